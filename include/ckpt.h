@@ -1,0 +1,148 @@
+/* include/ckpt.h — C ABI of the B200-native GPU Merkle-tree checkpoint de-duplication
+ * library (libckpt.so), after Tan et al., "Scalable Incremental Checkpointing using
+ * GPU-Accelerated De-Duplication", ICPP'23. "P:n" cites /root/reference/PAPER.md line n;
+ * "Rk" cites reading k in DESIGN.md §3.
+ *
+ * Problem statement: a process owns one GPU and repeatedly hands a
+ * device buffer to the library; it stops while the buffer is de-duplicated on the GPU
+ * ("stops during checkpointing to perform the de-duplication") and receives one
+ * consolidated difference — compact metadata followed by the first-occurrence chunks
+ * (P:81). Any checkpoint of the lineage can later be restored.
+ *
+ * General rules for every function:
+ *  - Return value: a CKPT_* status; 0 (CKPT_OK) on success. Nothing is silently degraded
+ *    and there is no CPU fallback: without a usable sm_100a GPU, calls fail.
+ *  - A handle is bound to the CUDA device current at ckpt_create and is not thread-safe;
+ *    different handles (one per GPU / process) are independent.
+ *  - After any CUDA failure the handle is poisoned: every later call except ckpt_destroy
+ *    returns CKPT_ESTATE.
+ *  - "stream" arguments are cudaStream_t values passed as void* (NULL = legacy default
+ *    stream) so this header needs no CUDA include.
+ */
+#ifndef CKPT_H_
+#define CKPT_H_
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define CKPT_API __attribute__((visibility("default")))
+#else
+#define CKPT_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct ckpt_ctx* ckpt_handle;
+
+enum {
+  CKPT_OK = 0,
+  CKPT_EINVAL = 1, /* bad argument / precondition violated; nothing changed           */
+  CKPT_ENOMEM = 2, /* device allocation (record growth, diff arena) failed; nothing committed */
+  CKPT_ECUDA = 3,  /* CUDA runtime/driver error; the handle is now poisoned            */
+  CKPT_ERANGE = 4, /* checkpoint id out of range                                       */
+  CKPT_ESTATE = 5, /* handle poisoned by an earlier CUDA error                          */
+  CKPT_ECOLLIDE = 6 /* a 128-bit digest collision was detected (R14: out of scope; the
+                       checkpoint is committed but its phase-2 record insert was skipped) */
+};
+
+/* Statistics and location of one consolidated difference. */
+typedef struct {
+  uint32_t id;              /* 0-based position in this handle's lineage (R19)               */
+  uint32_t chunk_bytes;     /* C                                                             */
+  const uint8_t* dev_ptr;   /* serialized diff in device memory, OWNED BY THE HANDLE, valid
+                               until ckpt_destroy (format: DESIGN.md §4, reading R13)        */
+  uint64_t bytes;           /* meta_bytes + data_bytes                                       */
+  uint64_t meta_bytes;      /* 64-B header + 4 B per FIRST region + 12 B per SHIFT region,
+                               zero-padded to 16 B                                            */
+  uint64_t data_bytes;      /* bytes of first-occurrence regions                      */
+  uint64_t buf_bytes;       /* B                                                             */
+  uint64_t n_leaves;        /* n = ceil(B / C)                                               */
+  uint64_t n_first_regions; /* Tree metadata entries for first occurrences            */
+  uint64_t n_shift_regions; /* Tree metadata entries for shifted duplicates                  */
+  uint64_t n_first;         /* leaves labelled FIRST_OCUR (Alg.1 l.9)                        */
+  uint64_t n_fixed;         /* leaves labelled FIXED_DUPL (Alg.1 l.4): unchanged             */
+  uint64_t n_spatial;       /* SHIFT_DUPL leaves whose source is this checkpoint            */
+  uint64_t n_temporal;      /* SHIFT_DUPL leaves whose source is an earlier checkpoint      */
+  uint64_t list_entries;    /* List-method entries = n_first + n_spatial + n_temporal*/
+  uint64_t record_size;     /* entries in the historical record after this checkpoint */
+  uint64_t record_capacity; /* slots of the device record table                              */
+  uint64_t phase2_inserts;  /* FIRST internal nodes inserted (Alg.1 l.29)                    */
+} ckpt_diff;
+
+/* Create a handle.  P:77: fixed-size chunks of "tens or hundreds of bytes".
+ *   chunk_bytes  C, a multiple of 16 with 32 <= C <= 65536 (C > 2 x 16-B digest).
+ *   out          receives the handle (owned by the caller; free with ckpt_destroy).
+ * Binds the handle to the current CUDA device.  Errors: CKPT_EINVAL (bad C / NULL out),
+ * CKPT_ECUDA (no usable sm_100 device). */
+CKPT_API int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out);
+
+/* De-duplicate one checkpoint (Alg.1; serialization P:81).
+ *   dev_ptr  device buffer of `bytes` bytes, 16-byte aligned, BORROWED for the call; the
+ *            caller must not modify it until the call returns.
+ *   bytes    B >= 1 with ceil(B / C) <= 2^31; every checkpoint of a handle must have the
+ *            same B (R17: the fixed-duplicate test is positional).
+ *   stream   cudaStream_t (as void*) all GPU work is enqueued on, in order.
+ *   diff     receives the statistics and the device pointer of the new diff.
+ * The call returns after exactly one host synchronisation with `stream` (the process
+ * "stops during checkpointing"). Capacity for the record table and the diff is
+ * reserved before the first kernel, so an error leaves the lineage unchanged.
+ * Errors: CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ESTATE, CKPT_ECOLLIDE. */
+CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff);
+
+/* Rebuild checkpoint `id` into the caller's device buffer ("start from the
+ * first-time occurrences, then fill the fixed duplicates and finally assemble the shifted
+ * duplicates from the corresponding checkpoint ID") by replaying diffs 0..id (R16).
+ *   dev_ptr  device buffer of B bytes, 16-byte aligned, owned by the caller; overwritten.
+ * Synchronous (runs on an internal stream of the handle).
+ * Errors: CKPT_ERANGE (id >= number of checkpoints), CKPT_EINVAL, CKPT_ECUDA, CKPT_ESTATE. */
+CKPT_API int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr);
+
+/* Statistics / device pointer of an earlier diff.  Errors: CKPT_ERANGE, CKPT_EINVAL. */
+CKPT_API int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff);
+
+/* Copy diff `id` to host memory with ONE device-to-host transfer ("initiating a
+ * single device-to-host data transfer is enough").
+ *   host_ptr  caller-owned host memory (pinned for full PCIe bandwidth) of >= capacity B.
+ * Synchronous. Errors: CKPT_ERANGE, CKPT_EINVAL (capacity < diff bytes), CKPT_ECUDA. */
+CKPT_API int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity);
+
+/* End-to-end convenience path over HOST memory (P:196's throughput definition: create
+ * the incremental checkpoint and copy it to host memory): copies `bytes` from host_ptr
+ * into a handle-owned device staging buffer, runs ckpt_checkpoint on `stream`, then
+ * copies the diff into host_diff (capacity host_diff_cap) — one H2D, one D2H.
+ * host_diff may be NULL to skip the D2H.  Errors as ckpt_checkpoint and ckpt_diff_to_host. */
+CKPT_API int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, void* stream,
+                         void* host_diff, uint64_t host_diff_cap, ckpt_diff* diff);
+
+/* Number of checkpoints taken so far. */
+CKPT_API int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count);
+
+/* Introspection for parity tests (not on the hot path):
+ * ckpt_leaf_digests copies the persistent leaf digests Tree(leaf) of the latest checkpoint
+ * (Alg.1 l.21; 16 B per chunk, h1 LE || h2 LE, R1) into device memory dev_out (16 n bytes).
+ * ckpt_record_dump copies the historical record to host arrays: keys (16 B each),
+ * node ids and checkpoint ids, at most `cap` entries; *count receives the record size. */
+CKPT_API int ckpt_leaf_digests(ckpt_handle h, void* dev_out);
+CKPT_API int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_nodes, uint32_t* host_ckpts,
+                     uint64_t cap, uint64_t* count);
+
+/* Per-phase device times (ms) of the latest ckpt_checkpoint, measured with CUDA events on
+ * the caller's stream when profiling is enabled (ckpt_set_profiling(h, 1)).
+ * times[0] leaf hash pass (K1), [1] record insert (K1b), [2] phase 2 (all stages),
+ * [3] phase 3 (all stages), [4] compaction (offsets + gather), [5] whole call (first
+ * kernel to last kernel). */
+CKPT_API int ckpt_set_profiling(ckpt_handle h, int enable);
+CKPT_API int ckpt_phase_times(ckpt_handle h, float* times, int n);
+
+/* Release all device memory of the handle (record, leaf digests, every diff). */
+CKPT_API int ckpt_destroy(ckpt_handle h);
+
+/* Static description of a status code. */
+CKPT_API const char* ckpt_strerror(int status);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CKPT_H_ */

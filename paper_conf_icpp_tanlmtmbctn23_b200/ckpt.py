@@ -1,0 +1,243 @@
+"""Thin Python binding of libckpt.so (include/ckpt.h) — argument marshalling only.
+
+Every step of the de-duplication path runs in the library's sm_100a kernels; this module
+only converts torch tensors / integers into the C ABI's pointers and sizes. There is no
+CPU fallback: if the extension is missing or no B200 is visible, calls raise.
+
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    ck = Checkpointer(chunk_bytes=128)
+    d = ck.checkpoint(buf)            # buf: torch.uint8 CUDA tensor (16-B aligned)
+    ck.restore(d["id"], out)          # out: torch.uint8 CUDA tensor of the same size
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import _build
+
+CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_ECOLLIDE = range(7)
+
+ABI_FUNCTIONS = [
+    "ckpt_create", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
+    "ckpt_checkpoint_host", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
+    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_destroy", "ckpt_strerror",
+]
+
+
+class CkptDiff(ctypes.Structure):
+    _fields_ = [
+        ("id", ctypes.c_uint32),
+        ("chunk_bytes", ctypes.c_uint32),
+        ("dev_ptr", ctypes.c_void_p),
+        ("bytes", ctypes.c_uint64),
+        ("meta_bytes", ctypes.c_uint64),
+        ("data_bytes", ctypes.c_uint64),
+        ("buf_bytes", ctypes.c_uint64),
+        ("n_leaves", ctypes.c_uint64),
+        ("n_first_regions", ctypes.c_uint64),
+        ("n_shift_regions", ctypes.c_uint64),
+        ("n_first", ctypes.c_uint64),
+        ("n_fixed", ctypes.c_uint64),
+        ("n_spatial", ctypes.c_uint64),
+        ("n_temporal", ctypes.c_uint64),
+        ("list_entries", ctypes.c_uint64),
+        ("record_size", ctypes.c_uint64),
+        ("record_capacity", ctypes.c_uint64),
+        ("phase2_inserts", ctypes.c_uint64),
+    ]
+
+    def as_dict(self) -> dict:
+        return {name: getattr(self, name) for name, _ in self._fields_}
+
+
+class CkptError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        super().__init__(f"{what}: {strerror(status)} (status {status})")
+        self.status = status
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load the in-tree libckpt.so (fails loudly if it is missing)."""
+    global _lib
+    if _lib is None:
+        path = _build.lib_path("libckpt.so")
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} missing: run __graft_entry__.build() (no CPU fallback exists)")
+        L = ctypes.CDLL(path)
+        vp, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+        P = ctypes.POINTER
+        sig = {
+            "ckpt_create": ([u32, P(vp)], i32),
+            "ckpt_checkpoint": ([vp, vp, u64, vp, P(CkptDiff)], i32),
+            "ckpt_restore": ([vp, u32, vp], i32),
+            "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
+            "ckpt_diff_to_host": ([vp, u32, vp, u64], i32),
+            "ckpt_checkpoint_host": ([vp, vp, u64, vp, vp, u64, P(CkptDiff)], i32),
+            "ckpt_num_checkpoints": ([vp, P(u32)], i32),
+            "ckpt_leaf_digests": ([vp, vp], i32),
+            "ckpt_record_dump": ([vp, vp, vp, vp, u64, P(u64)], i32),
+            "ckpt_set_profiling": ([vp, i32], i32),
+            "ckpt_phase_times": ([vp, P(ctypes.c_float), i32], i32),
+            "ckpt_destroy": ([vp], i32),
+            "ckpt_strerror": ([i32], ctypes.c_char_p),
+        }
+        for name, (args, res) in sig.items():
+            f = getattr(L, name)
+            f.argtypes = args
+            f.restype = res
+        _lib = L
+    return _lib
+
+
+def strerror(status: int) -> str:
+    return lib().ckpt_strerror(status).decode()
+
+
+def _ptr(x) -> int:
+    """Device/host pointer of a torch tensor, numpy array or raw integer."""
+    if isinstance(x, int):
+        return x
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if hasattr(x, "ctypes"):
+        return x.ctypes.data
+    raise TypeError(type(x))
+
+
+def _nbytes(x) -> int:
+    if hasattr(x, "element_size"):
+        return x.numel() * x.element_size()
+    if hasattr(x, "nbytes"):
+        return int(x.nbytes)
+    raise TypeError("pass nbytes explicitly")
+
+
+def _stream_handle(stream) -> int:
+    if stream is None:
+        try:
+            import torch
+            return torch.cuda.current_stream().cuda_stream
+        except Exception:
+            return 0
+    if hasattr(stream, "cuda_stream"):
+        return stream.cuda_stream
+    return int(stream)
+
+
+class Checkpointer:
+    """One de-duplication lineage on the current CUDA device (one per process / GPU)."""
+
+    def __init__(self, chunk_bytes: int):
+        h = ctypes.c_void_p()
+        rc = lib().ckpt_create(chunk_bytes, ctypes.byref(h))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_create")
+        self._h = h
+        self.chunk_bytes = chunk_bytes
+
+    # ------------------------------------------------------------------ core calls
+    def checkpoint(self, buf, nbytes: int | None = None, stream=None, raw: bool = False):
+        d = CkptDiff()
+        n = _nbytes(buf) if nbytes is None else nbytes
+        rc = lib().ckpt_checkpoint(self._h, _ptr(buf), n, _stream_handle(stream), ctypes.byref(d))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_checkpoint")
+        return d if raw else d.as_dict()
+
+    def checkpoint_host(self, host_buf, host_diff=None, nbytes: int | None = None, stream=None):
+        d = CkptDiff()
+        n = _nbytes(host_buf) if nbytes is None else nbytes
+        cap = _nbytes(host_diff) if host_diff is not None else 0
+        rc = lib().ckpt_checkpoint_host(self._h, _ptr(host_buf), n, _stream_handle(stream),
+                                        _ptr(host_diff) if host_diff is not None else None, cap, ctypes.byref(d))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_checkpoint_host")
+        return d.as_dict()
+
+    def restore(self, cid: int, out) -> None:
+        rc = lib().ckpt_restore(self._h, cid, _ptr(out))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_restore")
+
+    def diff_info(self, cid: int) -> dict:
+        d = CkptDiff()
+        rc = lib().ckpt_diff_info(self._h, cid, ctypes.byref(d))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_diff_info")
+        return d.as_dict()
+
+    def diff_to_host(self, cid: int, out=None) -> bytes:
+        """One D2H of the consolidated diff. Returns bytes (or fills `out`)."""
+        info = self.diff_info(cid)
+        if out is None:
+            buf = ctypes.create_string_buffer(max(info["bytes"], 1))
+            rc = lib().ckpt_diff_to_host(self._h, cid, ctypes.addressof(buf), info["bytes"])
+            if rc != CKPT_OK:
+                raise CkptError(rc, "ckpt_diff_to_host")
+            return buf.raw[: info["bytes"]]
+        rc = lib().ckpt_diff_to_host(self._h, cid, _ptr(out), _nbytes(out))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_diff_to_host")
+        return None
+
+    @property
+    def num_checkpoints(self) -> int:
+        c = ctypes.c_uint32()
+        rc = lib().ckpt_num_checkpoints(self._h, ctypes.byref(c))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_num_checkpoints")
+        return c.value
+
+    # ------------------------------------------------------------------ introspection
+    def leaf_digests(self, out) -> None:
+        rc = lib().ckpt_leaf_digests(self._h, _ptr(out))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_leaf_digests")
+
+    def record(self):
+        """Historical record as a set of (digest bytes, node, ckpt)."""
+        import numpy as np
+        cnt = ctypes.c_uint64()
+        rc = lib().ckpt_record_dump(self._h, None, None, None, 0, ctypes.byref(cnt))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_record_dump")
+        m = cnt.value + 16
+        keys = np.zeros((m, 16), dtype=np.uint8)
+        nodes = np.zeros(m, dtype=np.uint32)
+        ckpts = np.zeros(m, dtype=np.uint32)
+        rc = lib().ckpt_record_dump(self._h, keys.ctypes.data, nodes.ctypes.data, ckpts.ctypes.data, m,
+                                    ctypes.byref(cnt))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_record_dump")
+        k = cnt.value
+        return {(keys[i].tobytes(), int(nodes[i]), int(ckpts[i])) for i in range(k)}
+
+    def set_profiling(self, on: bool = True) -> None:
+        lib().ckpt_set_profiling(self._h, 1 if on else 0)
+
+    def phase_times(self) -> dict:
+        t = (ctypes.c_float * 6)()
+        lib().ckpt_phase_times(self._h, t, 6)
+        names = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total"]
+        return {names[i]: t[i] for i in range(6)}
+
+    def close(self) -> None:
+        if getattr(self, "_h", None):
+            lib().ckpt_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -1,0 +1,635 @@
+// engine.cu — host side of libckpt.so: the C ABI of include/ckpt.h.
+//
+// Owns, per handle (one process / GPU): the persistent leaf digests
+// Tree(leaf) (Alg.1 l.21, R5), the device record table, the per-stage tree
+// scratch, and an arena of consolidated diffs. ckpt_checkpoint enqueues the kernel
+// sequence of kernels.h on the caller's stream and synchronises exactly once, to read
+// the 128-byte totals record back (the process stops during checkpointing).
+// All capacity (record table, diff arena) is reserved before the first kernel, so a
+// failure never leaves a half-committed checkpoint (ckpt.h error contract).
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "../../include/ckpt.h"
+#include "kernels.h"
+
+using namespace ckpt;
+
+namespace {
+
+struct ArenaBlock {
+  uint8_t* ptr;
+  uint64_t size, used;
+};
+
+struct DiffRec {
+  ckpt_diff info;
+  uint8_t* ptr;
+  unsigned long long* Flo = nullptr;   // restore caches (lazy)
+  unsigned long long* Foff = nullptr;
+};
+
+constexpr double kMaxLoad = 0.8;     // reserve so that even a worst-case checkpoint stays below this
+constexpr double kGrowLoad = 0.6;    // load factor right after a growth
+constexpr uint64_t kArenaMin = 256ull << 20;
+
+}  // namespace
+
+struct ckpt_ctx {
+  int device = 0;
+  int num_sms = 148;
+  bool poisoned = false;
+  uint32_t C = 0;
+  // geometry (fixed after checkpoint 0, R17)
+  bool geo_set = false;
+  uint64_t B = 0, n = 0, m = 0;
+  int h = 0, t0 = 0;
+  int S = 0;
+  int Lin[kMaxStages] = {}, gsz[kMaxStages] = {};
+  uint64_t ngroups[kMaxStages] = {};
+  // device state
+  Digest* prev = nullptr;
+  uint32_t* cand = nullptr;
+  uint64_t nwords = 0;
+  uint32_t* slot_of = nullptr;
+  uint32_t* dirty[kMaxStages] = {};
+  uint32_t* wl[kMaxStages] = {};
+  LevelIO lvl[kMaxStages] = {};
+  uint4* scratch = nullptr;
+  uint4* tilecnt = nullptr;
+  uint4* toff = nullptr;
+  unsigned long long* blocksum = nullptr;
+  unsigned long long* freg_off = nullptr;
+  unsigned long long* freg_src = nullptr;
+  Totals* tot = nullptr;
+  Totals* tot_host = nullptr;   // pinned
+  Slot* tab = nullptr;
+  uint64_t cap = 0, live = 0;
+  std::vector<ArenaBlock> arena;
+  std::vector<DiffRec> diffs;
+  uint8_t* staging = nullptr;
+  uint64_t staging_size = 0;
+  cudaStream_t internal = nullptr;
+  bool prof = false;
+  cudaEvent_t ev[6] = {};
+  float times[6] = {};
+  PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  std::vector<void*> allocs;   // per-geometry allocations
+};
+
+#define CK(x)                                                                               \
+  do {                                                                                      \
+    cudaError_t e_ = (x);                                                                   \
+    if (e_ != cudaSuccess) {                                                                \
+      fprintf(stderr, "libckpt: CUDA error %s at %s:%d\n", cudaGetErrorString(e_), __FILE__, __LINE__); \
+      h->poisoned = true;                                                                   \
+      return CKPT_ECUDA;                                                                    \
+    }                                                                                       \
+  } while (0)
+
+namespace {
+
+template <class T>
+cudaError_t dalloc(ckpt_ctx* h, T** p, size_t count) {
+  void* q = nullptr;
+  cudaError_t e = cudaMalloc(&q, count * sizeof(T) > 0 ? count * sizeof(T) : 16);
+  if (e != cudaSuccess) return e;
+  h->allocs.push_back(q);
+  *p = static_cast<T*>(q);
+  return cudaSuccess;
+}
+
+int ceil_log2(uint64_t n) {
+  int h = 0;
+  while ((1ull << h) < n) ++h;
+  return h;
+}
+
+int setup_geometry(ckpt_ctx* h, uint64_t B) {
+  h->B = B;
+  h->n = (B + h->C - 1) / h->C;
+  h->h = ceil_log2(h->n);
+  h->m = 2 * h->n - (1ull << h->h);
+  h->t0 = std::min(kTileLog, h->h);
+  // stage plan: stage 0 covers heights 0..t0 (tiles); then groups of kGroupLog levels
+  h->S = 0;
+  int L = 0;
+  h->Lin[0] = 0;
+  h->gsz[0] = h->t0;
+  h->S = 1;
+  L = h->t0;
+  while (L < h->h) {
+    if (h->S >= kMaxStages) return CKPT_EINVAL;
+    const int g = std::min(kGroupLog, h->h - L);
+    h->Lin[h->S] = L;
+    h->gsz[h->S] = g;
+    ++h->S;
+    L += g;
+  }
+  for (int s = 0; s < h->S; ++s) h->ngroups[s] = 1ull << (h->h - h->Lin[s] - h->gsz[s]);
+
+  const uint64_t n = h->n;
+  const uint64_t n_tiles = h->ngroups[0];
+  h->nwords = (n + 31) / 32;
+  cudaError_t e = cudaSuccess;
+#define AL(ptr, cnt)                      \
+  do {                                    \
+    e = dalloc(h, &(ptr), (cnt));         \
+    if (e != cudaSuccess) return CKPT_ENOMEM; \
+  } while (0)
+  AL(h->prev, n);
+  AL(h->cand, h->nwords + 32);
+  AL(h->slot_of, n);
+  for (int s = 0; s < h->S; ++s) {
+    AL(h->dirty[s], h->ngroups[s]);
+    AL(h->wl[s], h->ngroups[s]);
+    if (cudaMemset(h->dirty[s], 0, h->ngroups[s] * 4) != cudaSuccess) return CKPT_ECUDA;
+    if (s >= 1) {
+      const uint64_t P = 1ull << (h->h - h->Lin[s]);
+      AL(h->lvl[s].lab2, P);
+      AL(h->lvl[s].lab3, P);
+      AL(h->lvl[s].dig, P);
+      AL(h->lvl[s].src, P);
+    }
+  }
+  AL(h->scratch, n_tiles << h->t0);
+  AL(h->tilecnt, n_tiles);
+  AL(h->toff, n_tiles);
+  AL(h->blocksum, 3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3);
+  AL(h->freg_off, n + 1);
+  AL(h->freg_src, n + 1);
+#undef AL
+  if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
+  h->geo_set = true;
+  return CKPT_OK;
+}
+
+Geo make_geo(const ckpt_ctx* h, uint32_t k) {
+  Geo g;
+  g.B = h->B;
+  g.n = h->n;
+  g.m = h->m;
+  g.C = h->C;
+  g.h = h->h;
+  g.t0 = h->t0;
+  g.k = k;
+  g.epoch = k + 1;
+  return g;
+}
+
+int ensure_table(ckpt_ctx* h, cudaStream_t st) {
+  const uint64_t need = h->live + 2 * h->n - 1;   // worst case: every node inserted
+  if (h->cap && (double)need <= kMaxLoad * (double)h->cap) return CKPT_OK;
+  uint64_t new_cap = (uint64_t)((double)need / kGrowLoad) + 1;
+  if (new_cap < 4096) new_cap = 4096;
+  if (new_cap >= (1ull << 32)) return CKPT_ENOMEM;   // slot ids are u32
+  Slot* nt = nullptr;
+  if (cudaMalloc(&nt, new_cap * sizeof(Slot)) != cudaSuccess) {
+    cudaGetLastError();
+    return CKPT_ENOMEM;
+  }
+  if (cudaMemsetAsync(nt, 0xFF, new_cap * sizeof(Slot), st) != cudaSuccess) return CKPT_ECUDA;
+  if (h->tab) {
+    if (launch_rehash(h->tab, h->cap, nt, new_cap, st) != cudaSuccess) return CKPT_ECUDA;
+    if (cudaStreamSynchronize(st) != cudaSuccess) return CKPT_ECUDA;
+    cudaFree(h->tab);
+  }
+  h->tab = nt;
+  h->cap = new_cap;
+  return CKPT_OK;
+}
+
+int reserve_arena(ckpt_ctx* h, uint64_t worst, uint8_t** out) {
+  if (!h->arena.empty()) {
+    ArenaBlock& b = h->arena.back();
+    if (b.size - b.used >= worst) {
+      *out = b.ptr + b.used;
+      return CKPT_OK;
+    }
+  }
+  const uint64_t size = std::max(worst, kArenaMin);
+  void* p = nullptr;
+  if (cudaMalloc(&p, size) != cudaSuccess) {
+    cudaGetLastError();
+    return CKPT_ENOMEM;
+  }
+  h->arena.push_back(ArenaBlock{static_cast<uint8_t*>(p), size, 0});
+  *out = static_cast<uint8_t*>(p);
+  return CKPT_OK;
+}
+
+int make_tmap(ckpt_ctx* h, const void* buf, const LeafParams& lp, CUtensorMap* map) {
+  cuuint64_t dims[3];
+  cuuint64_t strides[2];
+  cuuint32_t box[3];
+  cuuint32_t es[3] = {1, 1, 1};
+  cuuint32_t rank;
+  if (lp.mode3d) {
+    rank = 3;
+    dims[0] = 128; dims[1] = h->C / 128; dims[2] = lp.n_main;
+    strides[0] = 128; strides[1] = h->C;
+    box[0] = 128; box[1] = 1; box[2] = kLeafThreads;
+  } else {
+    rank = 2;
+    dims[0] = 128; dims[1] = lp.n_main * h->C / 128;
+    strides[0] = 128;
+    box[0] = 128; box[1] = lp.stage_bytes / 128;
+  }
+  CUresult r = h->encode(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, rank, const_cast<void*>(buf), dims, strides, box, es,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS ? CKPT_OK : CKPT_ECUDA;
+}
+
+void fill_diff(const ckpt_ctx* h, uint32_t id, const Totals& t, uint8_t* ptr, ckpt_diff* d) {
+  std::memset(d, 0, sizeof(*d));
+  d->id = id;
+  d->chunk_bytes = h->C;
+  d->dev_ptr = ptr;
+  d->meta_bytes = t.meta_bytes;
+  d->data_bytes = t.data_bytes;
+  d->bytes = t.meta_bytes + t.data_bytes;
+  d->buf_bytes = h->B;
+  d->n_leaves = h->n;
+  d->n_first_regions = t.nF;
+  d->n_shift_regions = t.nS;
+  d->n_first = t.n_first;
+  d->n_spatial = t.n_spatial;
+  d->n_temporal = t.n_temporal;
+  d->n_fixed = h->n - t.n_first - t.n_spatial - t.n_temporal;
+  d->list_entries = t.n_first + t.n_spatial + t.n_temporal;
+  d->record_size = h->live;
+  d->record_capacity = h->cap;
+  d->phase2_inserts = t.p2_inserts;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* ckpt_strerror(int status) {
+  switch (status) {
+    case CKPT_OK: return "ok";
+    case CKPT_EINVAL: return "invalid argument";
+    case CKPT_ENOMEM: return "out of device memory";
+    case CKPT_ECUDA: return "CUDA error";
+    case CKPT_ERANGE: return "checkpoint id out of range";
+    case CKPT_ESTATE: return "handle poisoned by an earlier CUDA error";
+    case CKPT_ECOLLIDE: return "128-bit digest collision detected";
+    default: return "unknown status";
+  }
+}
+
+int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
+  if (!out || chunk_bytes < 32 || chunk_bytes > 65536 || chunk_bytes % 16) return CKPT_EINVAL;
+  *out = nullptr;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, dev) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
+  if (prop.major != 10) return CKPT_ECUDA;   // built for sm_100a only; no fallback
+  ckpt_ctx* h = new (std::nothrow) ckpt_ctx();
+  if (!h) return CKPT_ENOMEM;
+  h->device = dev;
+  h->num_sms = prop.multiProcessorCount;
+  h->C = chunk_bytes;
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess || !fn) {
+    delete h;
+    return CKPT_ECUDA;
+  }
+  h->encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  if (cudaMallocHost(&h->tot_host, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  if (cudaMalloc(&h->tot, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ENOMEM; }
+  for (int i = 0; i < 6; ++i) cudaEventCreate(&h->ev[i]);
+  *out = h;
+  return CKPT_OK;
+}
+
+int ckpt_destroy(ckpt_handle h) {
+  if (!h) return CKPT_EINVAL;
+  cudaDeviceSynchronize();
+  for (void* p : h->allocs) cudaFree(p);
+  for (auto& b : h->arena) cudaFree(b.ptr);
+  for (auto& d : h->diffs) { if (d.Flo) cudaFree(d.Flo); if (d.Foff) cudaFree(d.Foff); }
+  if (h->tab) cudaFree(h->tab);
+  if (h->tot) cudaFree(h->tot);
+  if (h->tot_host) cudaFreeHost(h->tot_host);
+  if (h->staging) cudaFree(h->staging);
+  for (int i = 0; i < 6; ++i) if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+  if (h->internal) cudaStreamDestroy(h->internal);
+  cudaGetLastError();
+  delete h;
+  return CKPT_OK;
+}
+
+int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count) {
+  if (!h || !count) return CKPT_EINVAL;
+  *count = (uint32_t)h->diffs.size();
+  return CKPT_OK;
+}
+
+int ckpt_set_profiling(ckpt_handle h, int enable) {
+  if (!h) return CKPT_EINVAL;
+  h->prof = enable != 0;
+  return CKPT_OK;
+}
+
+int ckpt_phase_times(ckpt_handle h, float* times, int n) {
+  if (!h || !times) return CKPT_EINVAL;
+  for (int i = 0; i < n && i < 6; ++i) times[i] = h->times[i];
+  return CKPT_OK;
+}
+
+int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
+  if (!h) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (!dev_ptr || !diff || bytes == 0 || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
+  if ((bytes + h->C - 1) / h->C > (1ull << 31)) return CKPT_EINVAL;
+  if (h->geo_set && bytes != h->B) return CKPT_EINVAL;   // R17
+  {
+    cudaPointerAttributes pa;
+    if (cudaPointerGetAttributes(&pa, dev_ptr) != cudaSuccess) { cudaGetLastError(); return CKPT_EINVAL; }
+    if (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged) return CKPT_EINVAL;
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (!h->geo_set) {
+    const int r = setup_geometry(h, bytes);
+    if (r != CKPT_OK) return r;
+  }
+  const uint32_t k = (uint32_t)h->diffs.size();
+  int r = ensure_table(h, st);
+  if (r != CKPT_OK) return r;
+  const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
+  uint8_t* out = nullptr;
+  r = reserve_arena(h, worst, &out);
+  if (r != CKPT_OK) return r;
+
+  const Geo g = make_geo(h, k);
+  const uint8_t* buf = static_cast<const uint8_t*>(dev_ptr);
+
+  // ---- leaf pass configuration
+  LeafParams lp;
+  std::memset(&lp, 0, sizeof(lp));
+  lp.g = g;
+  lp.buf = buf;
+  lp.prev = h->prev;
+  lp.cand = h->cand;
+  const uint64_t n_full = h->B / h->C;
+  if (h->C % 128 == 0) {
+    lp.mode3d = 1;
+    lp.segs = (int)(h->C / 128);
+    lp.stage_bytes = 128 * kLeafThreads;
+    lp.nst = 3;
+    lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
+  } else if (h->C < 128) {
+    lp.mode3d = 0;
+    lp.segs = 1;
+    lp.stage_bytes = kLeafThreads * h->C;
+    lp.nst = (int)std::min<uint64_t>(8, std::max<uint64_t>(2, 98304 / (lp.stage_bytes + kLeafThreads * 16)));
+    lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
+  } else {
+    lp.n_main = 0;   // odd chunk sizes above 128 B: direct-load pass only
+  }
+  lp.tail_begin = lp.n_main;
+  CUtensorMap tmap;
+  if (lp.n_main) {
+    r = make_tmap(h, buf, lp, &tmap);
+    if (r != CKPT_OK) { h->poisoned = true; return r; }
+  }
+
+  CK(cudaMemsetAsync(h->tot, 0, sizeof(Totals), st));
+  if (h->prof) CK(cudaEventRecord(h->ev[0], st));
+  // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
+  CK(launch_leaf_tail(lp, st));
+  CK(launch_leaf(&tmap, lp, h->num_sms, st));
+  if (h->prof) CK(cudaEventRecord(h->ev[1], st));
+  // K1b: record insert + tie-break (l.6-19), dirty tiles
+  InsertParams ip;
+  ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
+  ip.tab = h->tab; ip.cap = h->cap; ip.slot_of = h->slot_of;
+  ip.dirty0 = h->dirty[0]; ip.wl0 = h->wl[0]; ip.tot = h->tot;
+  CK(launch_insert(ip, st));
+  if (h->prof) CK(cudaEventRecord(h->ev[2], st));
+
+  // ---- phase 2 (all stages), then phase 3 (all stages): R11
+  TreeParams tp;
+  std::memset(&tp, 0, sizeof(tp));
+  tp.g = g;
+  tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
+  tp.tab = h->tab; tp.cap = h->cap;
+  tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.tot = h->tot;
+  for (int phase = 2; phase <= 3; ++phase) {
+    for (int s = 0; s < h->S; ++s) {
+      tp.s = s;
+      tp.Lin = h->Lin[s];
+      tp.gsz = h->gsz[s];
+      tp.last = (s == h->S - 1);
+      tp.wl = h->wl[s];
+      tp.wl_slot = s;
+      tp.dirty_in = s >= 1 ? h->dirty[s - 1] : nullptr;
+      tp.in = s >= 1 ? h->lvl[s] : LevelIO{};
+      tp.out = !tp.last ? h->lvl[s + 1] : LevelIO{};
+      tp.dirty_next = !tp.last ? h->dirty[s + 1] : nullptr;
+      tp.wl_next = !tp.last ? h->wl[s + 1] : nullptr;
+      tp.g_next = !tp.last ? h->gsz[s + 1] : 0;
+      if (phase == 2) CK(launch_phase2(tp, h->ngroups[s], h->num_sms, st));
+      else CK(launch_phase3(tp, h->ngroups[s], h->num_sms, st));
+    }
+    if (h->prof) CK(cudaEventRecord(h->ev[phase == 2 ? 3 : 4], st));
+  }
+
+  // ---- compaction + serialisation
+  CompactParams cp;
+  cp.g = g;
+  cp.n_tiles = h->ngroups[0];
+  cp.tilecnt = h->tilecnt; cp.scratch = h->scratch; cp.blocksum = h->blocksum;
+  cp.toff = h->toff; cp.wl0 = h->wl[0]; cp.tot = h->tot;
+  cp.freg_off = h->freg_off; cp.freg_src = h->freg_src;
+  cp.out = out; cp.buf = buf;
+  CK(launch_compact(cp, h->num_sms, st));
+  if (h->prof) CK(cudaEventRecord(h->ev[5], st));
+  CK(cudaMemcpyAsync(h->tot_host, h->tot, sizeof(Totals), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));   // the one host synchronisation of the call
+
+  const Totals t = *h->tot_host;
+  if (h->prof) {
+    for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&h->times[i], h->ev[i], h->ev[i + 1]);
+    cudaEventElapsedTime(&h->times[5], h->ev[0], h->ev[5]);
+    // times: [0] K1 [1] K1b [2] phase 2 [3] phase 3 [4] compaction [5] total
+  }
+  h->live += t.n_first + t.p2_inserts;
+  DiffRec rec;
+  rec.ptr = out;
+  fill_diff(h, k, t, out, &rec.info);
+  ArenaBlock& blk = h->arena.back();
+  blk.used += (rec.info.bytes + 255) & ~255ull;
+  h->diffs.push_back(rec);
+  *diff = rec.info;
+  return t.collisions ? CKPT_ECOLLIDE : CKPT_OK;
+}
+
+int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff) {
+  if (!h || !diff) return CKPT_EINVAL;
+  if (id >= h->diffs.size()) return CKPT_ERANGE;
+  *diff = h->diffs[id].info;
+  return CKPT_OK;
+}
+
+int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity) {
+  if (!h || !host_ptr) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (id >= h->diffs.size()) return CKPT_ERANGE;
+  const DiffRec& d = h->diffs[id];
+  if (capacity < d.info.bytes) return CKPT_EINVAL;
+  CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, h->internal));   // one D2H
+  CK(cudaStreamSynchronize(h->internal));
+  return CKPT_OK;
+}
+
+int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, void* stream, void* host_diff,
+                         uint64_t host_diff_cap, ckpt_diff* diff) {
+  if (!h || !host_ptr || !diff || bytes == 0) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (h->geo_set && bytes != h->B) return CKPT_EINVAL;
+  if (h->staging_size < bytes) {
+    if (h->staging) cudaFree(h->staging);
+    h->staging = nullptr;
+    h->staging_size = 0;
+    if (cudaMalloc(&h->staging, bytes) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
+    h->staging_size = bytes;
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  CK(cudaMemcpyAsync(h->staging, host_ptr, bytes, cudaMemcpyHostToDevice, st));
+  int r = ckpt_checkpoint(h, h->staging, bytes, stream, diff);
+  if (r != CKPT_OK) return r;
+  if (host_diff) {
+    if (host_diff_cap < diff->bytes) return CKPT_EINVAL;
+    CK(cudaMemcpyAsync(host_diff, diff->dev_ptr, diff->bytes, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  }
+  return CKPT_OK;
+}
+
+int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
+  if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (id >= h->diffs.size()) return CKPT_ERANGE;
+  cudaStream_t st = h->internal;
+  const Geo g = make_geo(h, id);
+  uint64_t maxF = 1, maxS = 1;
+  for (uint32_t c = 0; c <= id; ++c) {
+    maxF = std::max<uint64_t>(maxF, h->diffs[c].info.n_first_regions);
+    maxS = std::max<uint64_t>(maxS, h->diffs[c].info.n_shift_regions);
+  }
+  const uint64_t maxN = std::max(maxF, maxS);
+  const size_t scan_bytes = scan_tmp_bytes_for(maxN);
+  unsigned long long *t_len = nullptr, *t_off = nullptr, *t_src = nullptr, *t_dst = nullptr;
+  void* scan_tmp = nullptr;
+  int* err = nullptr;
+  RestoreDiff* chain_dev = nullptr;
+  auto cleanup = [&]() {
+    cudaFree(t_len); cudaFree(t_off); cudaFree(t_src); cudaFree(t_dst);
+    cudaFree(scan_tmp); cudaFree(err); cudaFree(chain_dev);
+  };
+  if (cudaMalloc(&t_len, maxN * 8) != cudaSuccess || cudaMalloc(&t_off, maxN * 8) != cudaSuccess ||
+      cudaMalloc(&t_src, maxN * 8) != cudaSuccess || cudaMalloc(&t_dst, maxN * 8) != cudaSuccess ||
+      cudaMalloc(&scan_tmp, scan_bytes) != cudaSuccess || cudaMalloc(&err, sizeof(int)) != cudaSuccess ||
+      cudaMalloc(&chain_dev, sizeof(RestoreDiff) * (id + 1)) != cudaSuccess) {
+    cudaGetLastError();
+    cleanup();
+    return CKPT_ENOMEM;
+  }
+  std::vector<RestoreDiff> chain(id + 1);
+  int rc = CKPT_OK;
+  for (uint32_t c = 0; c <= id && rc == CKPT_OK; ++c) {
+    DiffRec& d = h->diffs[c];
+    RestoreDiff& rd = chain[c];
+    rd.base = d.ptr;
+    rd.nF = d.info.n_first_regions;
+    rd.nS = d.info.n_shift_regions;
+    rd.meta_bytes = d.info.meta_bytes;
+    rd.data_bytes = d.info.data_bytes;
+    if (!d.Flo && rd.nF) {
+      if (cudaMalloc(&d.Flo, rd.nF * 8) != cudaSuccess || cudaMalloc(&d.Foff, rd.nF * 8) != cudaSuccess) {
+        cudaGetLastError();
+        rc = CKPT_ENOMEM;
+        break;
+      }
+      rd.Flo = d.Flo;
+      rd.Foff = d.Foff;
+      if (restore_prepare_first(g, rd, t_len, scan_tmp, scan_bytes, st) != cudaSuccess) rc = CKPT_ECUDA;
+    }
+    rd.Flo = d.Flo;
+    rd.Foff = d.Foff;
+  }
+  if (rc == CKPT_OK) {
+    if (cudaMemcpyAsync(chain_dev, chain.data(), sizeof(RestoreDiff) * (id + 1), cudaMemcpyHostToDevice, st) !=
+            cudaSuccess ||
+        cudaMemsetAsync(err, 0, sizeof(int), st) != cudaSuccess || cudaMemsetAsync(dev_ptr, 0, h->B, st) != cudaSuccess)
+      rc = CKPT_ECUDA;
+  }
+  uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
+  for (uint32_t c = 0; c <= id && rc == CKPT_OK; ++c) {
+    // first-time occurrences, then (implicitly) fixed, then shifted duplicates
+    if (restore_copy_first(g, chain[c], outp, h->num_sms, st) != cudaSuccess) rc = CKPT_ECUDA;
+    else if (restore_shift(g, chain[c], chain_dev, outp, t_len, t_off, t_src, t_dst, err, scan_tmp, scan_bytes,
+                           h->num_sms, st) != cudaSuccess)
+      rc = CKPT_ECUDA;
+  }
+  int herr = 0;
+  if (rc == CKPT_OK) {
+    if (cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+      rc = CKPT_ECUDA;
+  }
+  cleanup();
+  if (rc == CKPT_ECUDA) h->poisoned = true;
+  if (rc == CKPT_OK && herr) rc = CKPT_EINVAL;   // malformed chain (a source outside any FIRST region)
+  return rc;
+}
+
+int ckpt_leaf_digests(ckpt_handle h, void* dev_out) {
+  if (!h || !dev_out) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (!h->geo_set) return CKPT_ERANGE;
+  CK(cudaMemcpyAsync(dev_out, h->prev, h->n * 16, cudaMemcpyDeviceToDevice, h->internal));
+  CK(cudaStreamSynchronize(h->internal));
+  return CKPT_OK;
+}
+
+int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_nodes, uint32_t* host_ckpts, uint64_t cap,
+                     uint64_t* count) {
+  if (!h || !count) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  *count = h->live;
+  if (!h->tab || cap == 0) return CKPT_OK;
+  std::vector<Slot> all(h->cap);
+  CK(cudaMemcpyAsync(all.data(), h->tab, h->cap * sizeof(Slot), cudaMemcpyDeviceToHost, h->internal));
+  CK(cudaStreamSynchronize(h->internal));
+  uint64_t i = 0;
+  for (const Slot& s : all) {
+    if (s.klo == kEmpty && s.khi == kEmpty) continue;
+    if (i < cap) {
+      if (host_keys) {
+        std::memcpy(host_keys + 16 * i, &s.klo, 8);
+        std::memcpy(host_keys + 16 * i + 8, &s.khi, 8);
+      }
+      if (host_nodes) host_nodes[i] = (uint32_t)(s.val & 0xffffffffu);
+      if (host_ckpts) host_ckpts[i] = (uint32_t)(s.val >> 32);
+    }
+    ++i;
+  }
+  *count = i;
+  return CKPT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,209 @@
+// k_restore.cu — restore scatter (reading R16).
+//
+// "To restore a checkpoint from the differences, it is enough to start from the
+// first-time occurrences, then fill the fixed duplicates and finally assemble the
+// shifted duplicates from the corresponding checkpoint ID (which can be a previous
+// checkpoint or the current checkpoint to be restored)". The engine replays
+// diffs 0..id into the caller's buffer; per diff c:
+//   prepare_first: FIRST region i -> (first chunk, byte length); exclusive scan of the
+//                  lengths = offsets in c's data section (kept for later diffs).
+//   copy_first   : the data section streamed to its regions, warp per 8-KiB segment.
+//   prepare_shift: SHIFT (u, v, c') -> (dst offset, length, source address) where the
+//                  source is v's bytes inside the FIRST region of diff c' holding v's
+//                  first chunk (binary search over c''s sorted region starts).
+//   copy_shift   : the virtual concatenation of the SHIFT regions, same streaming.
+// FIXED chunks are simply left as diff c-1's replay wrote them.
+#include "kernels.h"
+
+namespace ckpt {
+
+namespace {
+constexpr int kRT = 256;
+constexpr int kScanPer = 4;
+constexpr uint64_t kScanBlock = kRT * kScanPer;   // 1024 elements per scan block
+constexpr unsigned long long kSeg = 8192;
+
+__device__ __forceinline__ void node_range(const Geo& g, uint32_t node, uint64_t& lo, uint64_t& hi) {
+  const int depth = 31 - __clz(node + 1);
+  chunk_range(g, g.h - depth, (uint64_t)node + 1 - (1ull << depth), lo, hi);
+}
+
+__device__ __forceinline__ uint32_t rd32(const uint8_t* p) { return *reinterpret_cast<const uint32_t*>(p); }
+
+// ------------------------------------------------------------------ scan
+__global__ void __launch_bounds__(kRT) scan_block_kernel(const unsigned long long* in, unsigned long long* out,
+                                                        uint64_t count, unsigned long long* bsum) {
+  __shared__ unsigned long long wt[kRT / 32];
+  const uint64_t base = (uint64_t)blockIdx.x * kScanBlock + threadIdx.x * kScanPer;
+  unsigned long long v[kScanPer], mine = 0;
+  for (int i = 0; i < kScanPer; ++i) {
+    v[i] = (base + i < count) ? in[base + i] : 0ull;
+    mine += v[i];
+  }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  unsigned long long incl = mine;
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += u;
+  }
+  if (lane == 31) wt[wid] = incl;
+  __syncthreads();
+  unsigned long long off = 0, tot = 0;
+  for (int i = 0; i < kRT / 32; ++i) {
+    if (i < wid) off += wt[i];
+    tot += wt[i];
+  }
+  off += incl - mine;
+  for (int i = 0; i < kScanPer; ++i) {
+    if (base + i < count) out[base + i] = off;
+    off += v[i];
+  }
+  if (threadIdx.x == 0 && bsum) bsum[blockIdx.x] = tot;
+}
+
+__global__ void scan_add_kernel(unsigned long long* out, uint64_t count, const unsigned long long* boff) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < count) out[i] += boff[i / kScanBlock];
+}
+
+// ------------------------------------------------------------------ restore kernels
+__global__ void prepare_first_kernel(Geo g, RestoreDiff d, unsigned long long* len) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= d.nF) return;
+  const uint32_t node = rd32(d.base + 64 + 4 * i);
+  uint64_t lo, hi;
+  node_range(g, node, lo, hi);
+  d.Flo[i] = lo;
+  len[i] = range_bytes(g, lo, hi);
+}
+
+// stream `total` bytes laid out as consecutive regions (offsets off[0..nr), sorted) to
+// dst + dst_off(r) + (o - off[r]) from src(r) + (o - off[r]).
+template <bool FIRST>
+__global__ void __launch_bounds__(kRT) copy_stream_kernel(Geo g, RestoreDiff d, uint8_t* out,
+                                                          const unsigned long long* off, const unsigned long long* len,
+                                                          const unsigned long long* srcaddr,
+                                                          const unsigned long long* dstoff, uint64_t nr,
+                                                          unsigned long long total_known) {
+  if (nr == 0) return;
+  const unsigned long long total = FIRST ? total_known : off[nr - 1] + len[nr - 1];
+  const uint8_t* data = d.base + d.meta_bytes;
+  const int lane = threadIdx.x & 31;
+  const unsigned long long nseg = (total + kSeg - 1) / kSeg;
+  const unsigned long long wg = ((unsigned long long)blockIdx.x * kRT + threadIdx.x) >> 5;
+  const unsigned long long nw = ((unsigned long long)gridDim.x * kRT) >> 5;
+  for (unsigned long long sg = wg; sg < nseg; sg += nw) {
+    const unsigned long long s0 = sg * kSeg;
+    unsigned long long lo = 0, hi = nr;
+    while (hi - lo > 1) {
+      const unsigned long long mid = (lo + hi) >> 1;
+      if (off[mid] <= s0) lo = mid; else hi = mid;
+    }
+    unsigned long long r = lo;
+    unsigned long long next = (r + 1 < nr) ? off[r + 1] : ~0ull;
+    const unsigned long long send = (s0 + kSeg < total) ? s0 + kSeg : total;
+    for (unsigned long long o = s0 + 16ull * lane; o < send; o += 512) {
+      while (o >= next) {
+        ++r;
+        next = (r + 1 < nr) ? off[r + 1] : ~0ull;
+      }
+      const unsigned long long rel = o - off[r];
+      const uint8_t* s;
+      uint8_t* t;
+      if (FIRST) {
+        s = data + o;
+        t = out + d.Flo[r] * (unsigned long long)g.C + rel;
+      } else {
+        s = reinterpret_cast<const uint8_t*>(srcaddr[r]) + rel;
+        t = out + dstoff[r] + rel;
+      }
+      const unsigned long long rem = (r + 1 < nr ? off[r + 1] : total) - o;
+      if (rem >= 16) {
+        *reinterpret_cast<uint4*>(t) = *reinterpret_cast<const uint4*>(s);
+      } else {
+        for (unsigned long long b = 0; b < rem; ++b) t[b] = s[b];
+      }
+    }
+  }
+}
+
+__global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* chain, unsigned long long* len,
+                                     unsigned long long* srcaddr, unsigned long long* dstoff, int* err) {
+  const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= d.nS) return;
+  const uint8_t* e = d.base + 64 + 4 * d.nF + 12 * i;
+  const uint32_t u = rd32(e), v = rd32(e + 4), c2 = rd32(e + 8);
+  uint64_t ulo, uhi, vlo, vhi;
+  node_range(g, u, ulo, uhi);
+  node_range(g, v, vlo, vhi);
+  const RestoreDiff& s = chain[c2];
+  // FIRST region r of diff c2 with Flo[r] <= vlo (the last such): it contains v
+  uint64_t lo = 0, hi = s.nF;
+  if (s.nF == 0) { atomicExch(err, 1); len[i] = 0; srcaddr[i] = 0; dstoff[i] = 0; return; }
+  while (hi - lo > 1) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (s.Flo[mid] <= vlo) lo = mid; else hi = mid;
+  }
+  len[i] = range_bytes(g, ulo, uhi);
+  dstoff[i] = ulo * (unsigned long long)g.C;
+  srcaddr[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + (vlo - s.Flo[lo]) * (unsigned long long)g.C);
+}
+}  // namespace
+
+size_t scan_tmp_bytes_for(uint64_t count) {
+  size_t b = 0;
+  uint64_t c = count;
+  while (c > kScanBlock) {
+    const uint64_t nb = (c + kScanBlock - 1) / kScanBlock;
+    b += 2 * nb * sizeof(unsigned long long);
+    c = nb;
+  }
+  return b + 256;
+}
+
+cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long* out, uint64_t count, void* tmp,
+                               size_t tmp_bytes, cudaStream_t st) {
+  if (count == 0) return cudaSuccess;
+  const uint64_t nb = (count + kScanBlock - 1) / kScanBlock;
+  if (nb == 1) {
+    scan_block_kernel<<<1, kRT, 0, st>>>(in, out, count, nullptr);
+    return cudaGetLastError();
+  }
+  unsigned long long* bsum = reinterpret_cast<unsigned long long*>(tmp);
+  unsigned long long* boff = bsum + nb;
+  const size_t used = 2 * nb * sizeof(unsigned long long);
+  if (used > tmp_bytes) return cudaErrorInvalidValue;
+  scan_block_kernel<<<(unsigned)nb, kRT, 0, st>>>(in, out, count, bsum);
+  cudaError_t e = scan_u64_exclusive(bsum, boff, nb, boff + nb, tmp_bytes - used, st);
+  if (e != cudaSuccess) return e;
+  scan_add_kernel<<<(unsigned)((count + 255) / 256), 256, 0, st>>>(out, count, boff);
+  return cudaGetLastError();
+}
+
+cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long long* tmp_len, void* scan_tmp,
+                                  size_t scan_tmp_bytes, cudaStream_t st) {
+  if (d.nF == 0) return cudaSuccess;
+  prepare_first_kernel<<<(unsigned)((d.nF + 255) / 256), 256, 0, st>>>(g, d, tmp_len);
+  return scan_u64_exclusive(tmp_len, d.Foff, d.nF, scan_tmp, scan_tmp_bytes, st);
+}
+
+cudaError_t restore_copy_first(const Geo& g, const RestoreDiff& d, uint8_t* out, int num_sms, cudaStream_t st) {
+  if (d.nF == 0) return cudaSuccess;
+  copy_stream_kernel<true><<<num_sms * 8, kRT, 0, st>>>(g, d, out, d.Foff, nullptr, nullptr, nullptr, d.nF,
+                                                       d.data_bytes);
+  return cudaGetLastError();
+}
+
+cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, uint8_t* out,
+                          unsigned long long* t_len, unsigned long long* t_off, unsigned long long* t_src,
+                          unsigned long long* t_dst, int* err, void* scan_tmp, size_t scan_tmp_bytes, int num_sms,
+                          cudaStream_t st) {
+  if (d.nS == 0) return cudaSuccess;
+  prepare_shift_kernel<<<(unsigned)((d.nS + 255) / 256), 256, 0, st>>>(g, d, chain_dev, t_len, t_src, t_dst, err);
+  cudaError_t e = scan_u64_exclusive(t_len, t_off, d.nS, scan_tmp, scan_tmp_bytes, st);
+  if (e != cudaSuccess) return e;
+  copy_stream_kernel<false><<<num_sms * 8, kRT, 0, st>>>(g, d, out, t_off, t_len, t_src, t_dst, d.nS, 0);
+  return cudaGetLastError();
+}
+
+}  // namespace ckpt

@@ -1,0 +1,135 @@
+// kernels.h — parameter blocks and host launchers of the sm_100a kernels (internal).
+//
+// Launch order per checkpoint:
+//   K1  leaf hash + fixed test (TMA-staged, persistent)      Alg.1 l.1-5, l.21
+//   K1t leaf pass for the ragged tail (direct loads)           same
+//   K1b record insert + dirty-tile worklist                    Alg.1 l.6-19 (R6)
+//   P2[s] phase-2 stages (tile, then upper levels)             Alg.1 l.24-32
+//   P3[s] phase-3 stages + emission                            Alg.1 l.33-46 (R7-R10)
+//   KR/KO/KG/KD tile reduce, offsets + header, entries, data
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+
+#include "dev.cuh"
+
+namespace ckpt {
+
+constexpr int kMaxStages = 8;
+constexpr int kTileLog = 10;    // stage-0 tile: 1024 virtual leaf slots
+constexpr int kGroupLog = 10;   // upper stages: 1024 positions per group
+constexpr int kLeafThreads = 256;
+constexpr int kTreeThreads = 256;
+constexpr int kTilesPerBlock = 1024;  // compaction: tiles per reduce/offsets CTA
+
+struct Totals {                      // per-checkpoint device counters (zeroed each call)
+  unsigned long long nF, nS, data_bytes, meta_bytes;
+  unsigned long long n_first, n_spatial, n_temporal, p2_inserts;
+  unsigned long long collisions, n_cand, pad0, pad1;
+  uint32_t wl_count[kMaxStages];
+};
+
+struct LeafParams {
+  Geo g;
+  const uint8_t* buf;
+  uint64_t n_main;       // chunks handled by the TMA pipeline (multiple of 256)
+  uint64_t tail_begin;   // first chunk of the direct-load tail pass
+  int segs;              // 128-B rows per chunk (C >= 128) or 1
+  int mode3d;            // 1: C % 128 == 0 (3-D map: row r of 256 chunks); 0: C < 128 (2-D rows)
+  uint32_t stage_bytes;  // TMA bytes per pipeline stage
+  int nst;               // pipeline stages
+  Digest* prev;          // persistent leaf digests Tree(leaf), 16 n bytes
+  uint32_t* cand;        // candidate (non-FIXED) bit per chunk
+};
+
+struct InsertParams {
+  Geo g;
+  const Digest* prev;
+  const uint32_t* cand;
+  uint64_t nwords;
+  Slot* tab;
+  uint64_t cap;
+  uint32_t* slot_of;
+  uint32_t* dirty0;
+  uint32_t* wl0;
+  Totals* tot;
+};
+
+struct LevelIO {               // per-position arrays at one height (stage boundary)
+  uint8_t* lab2;               // phase-2 label (FIRST or not)
+  uint8_t* lab3;               // phase-3 label (FIRST / FIXED / SHIFT / DONE)
+  Digest* dig;                 // digest of FIRST (phase 2) or SHIFT (phase 3) positions
+  unsigned long long* src;     // packed (ckpt<<32|node) source of SHIFT positions
+};
+
+struct TreeParams {
+  Geo g;
+  int s;                       // stage index
+  int Lin;                     // input height
+  int gsz;                     // group log (levels processed)
+  int last;                    // output height == h (this stage ends at the root)
+  const uint32_t* wl;          // worklist of dirty groups of this stage
+  int wl_slot;                 // Totals::wl_count index of this stage
+  const uint32_t* dirty_in;    // s >= 1: dirty marks of stage s-1 (per input position)
+  LevelIO in;                  // s >= 1
+  LevelIO out;                 // !last
+  uint32_t* dirty_next;        // phase 2: mark parent groups of stage s+1
+  uint32_t* wl_next;
+  int g_next;
+  // leaf level (s == 0)
+  const uint32_t* cand;
+  const uint32_t* slot_of;
+  const Digest* prev;
+  Slot* tab;
+  uint64_t cap;
+  // emission (phase 3)
+  uint4* scratch;              // per tile: up to 2^t0 region records {node, src_node, src_ckpt, kind}
+  uint4* tilecnt;              // per tile: {nF, nS, data_bytes, epoch}
+  Totals* tot;
+};
+
+struct CompactParams {
+  Geo g;
+  uint64_t n_tiles;
+  const uint4* tilecnt;
+  const uint4* scratch;
+  unsigned long long* blocksum;  // 3 per reduce block
+  uint4* toff;                   // per tile {F_off, S_off, data_off lo, data_off hi}
+  const uint32_t* wl0;
+  Totals* tot;
+  unsigned long long* freg_off;   // per FIRST region (global order): offset in the data section
+  unsigned long long* freg_src;   // per FIRST region: byte offset in the checkpoint buffer
+  uint8_t* out;                  // diff destination (device arena)
+  const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
+};
+
+// ---- launchers (return cudaGetLastError())
+cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
+cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
+cudaError_t launch_insert(const InsertParams& p, cudaStream_t st);
+cudaError_t launch_phase2(const TreeParams& p, uint64_t n_groups, int num_sms, cudaStream_t st);
+cudaError_t launch_phase3(const TreeParams& p, uint64_t n_groups, int num_sms, cudaStream_t st);
+cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st);
+cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st);
+cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
+
+// ---- restore (k_restore.cu)
+struct RestoreDiff {           // one diff of the chain, as the restore kernels see it
+  const uint8_t* base;         // diff bytes (device)
+  uint64_t nF, nS, meta_bytes, data_bytes;
+  unsigned long long* Flo;     // per FIRST region: first chunk (sorted)
+  unsigned long long* Foff;    // per FIRST region: offset in the data section
+};
+cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long long* tmp_len, void* scan_tmp,
+                                  size_t scan_tmp_bytes, cudaStream_t st);
+cudaError_t restore_copy_first(const Geo& g, const RestoreDiff& d, uint8_t* out, int num_sms, cudaStream_t st);
+cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, uint8_t* out,
+                          unsigned long long* t_len, unsigned long long* t_off, unsigned long long* t_src,
+                          unsigned long long* t_dst, int* err, void* scan_tmp, size_t scan_tmp_bytes, int num_sms,
+                          cudaStream_t st);
+size_t scan_tmp_bytes_for(uint64_t count);
+cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long* out, uint64_t count, void* tmp,
+                               size_t tmp_bytes, cudaStream_t st);
+
+}  // namespace ckpt

@@ -267,3 +267,68 @@ def lineage(cfg: int, nbytes: int, chunk_bytes: int, K: int, seed: int | None = 
             yield g.next()
     else:
         raise ValueError(cfg)
+
+
+# ------------------------------------------------------------------ device twins
+class DeviceGen:
+    """ctypes binding of libckptgen.so: the same generators, writing straight into a CUDA
+    buffer (torch tensor or raw device pointer) on a stream."""
+
+    _lib = None
+
+    @classmethod
+    def lib(cls):
+        if cls._lib is None:
+            import ctypes
+            import os
+            from .. import _build
+            path = _build.lib_path("libckptgen.so")
+            if not os.path.exists(path):
+                raise RuntimeError(f"{path} missing: run __graft_entry__.build()")
+            L = ctypes.CDLL(path)
+            vp, u32, u64 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64
+            L.gen_cfg1_initial.argtypes = [vp, u64, u64, vp]
+            L.gen_cfg1_mutate.argtypes = [vp, u64, u32, u32, u64, u64, vp]
+            L.gen_cfg2_initial.argtypes = [vp, u64, u64, u64, vp]
+            L.gen_cfg2_mutate.argtypes = [vp, u64, u32, u64, u64, vp]
+            L.gen_freq_orbits.argtypes = [vp]
+            for f in ("gen_cfg1_initial", "gen_cfg1_mutate", "gen_cfg2_initial", "gen_cfg2_mutate", "gen_freq_orbits"):
+                getattr(L, f).restype = ctypes.c_int
+            cls._lib = L
+        return cls._lib
+
+    @staticmethod
+    def _args(buf, stream):
+        ptr = buf.data_ptr() if hasattr(buf, "data_ptr") else int(buf)
+        st = stream.cuda_stream if hasattr(stream, "cuda_stream") else (int(stream) if stream else 0)
+        return ptr, st
+
+    @classmethod
+    def freq_orbits(cls):
+        arr = np.zeros(32, dtype=np.int32)
+        n = cls.lib().gen_freq_orbits(arr.ctypes.data)
+        return arr[:n].astype(np.int64)
+
+    @classmethod
+    def initial(cls, cfg: int, buf, nbytes: int, seed: int, stream=None):
+        ptr, st = cls._args(buf, stream)
+        if cfg == 1:
+            rc = cls.lib().gen_cfg1_initial(ptr, nbytes, seed, st)
+        elif cfg in (2, 3, 5):
+            rc = cls.lib().gen_cfg2_initial(ptr, nbytes, seed, threshold(0.3), st)
+        else:
+            raise ValueError(f"config {cfg} has no device generator (host only)")
+        if rc:
+            raise RuntimeError(f"generator launch failed ({rc})")
+
+    @classmethod
+    def mutate(cls, cfg: int, buf, nbytes: int, k: int, chunk_bytes: int, seed: int, p: float, stream=None):
+        ptr, st = cls._args(buf, stream)
+        if cfg == 1:
+            rc = cls.lib().gen_cfg1_mutate(ptr, nbytes, chunk_bytes, k, seed, threshold(p), st)
+        elif cfg in (2, 3, 5):
+            rc = cls.lib().gen_cfg2_mutate(ptr, nbytes, k, seed, threshold(p), st)
+        else:
+            raise ValueError(cfg)
+        if rc:
+            raise RuntimeError(f"generator launch failed ({rc})")
