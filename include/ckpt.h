@@ -132,7 +132,9 @@ CKPT_API int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_
  * the caller's stream when profiling is enabled (ckpt_set_profiling(h, 1)).
  * times[0] leaf hash pass (K1), [1] record insert (K1b), [2] phase 2 (all stages),
  * [3] phase 3 (all stages), [4] compaction (offsets + gather), [5] whole call (first
- * kernel to last kernel). */
+ * kernel to last kernel); host wall times of the same call (always recorded): [6] entry
+ * to first enqueue, [7] enqueue of the kernel sequence, [8] wait in the one stream
+ * synchronisation, [9] bookkeeping after it.  n <= 10 values are written. */
 CKPT_API int ckpt_set_profiling(ckpt_handle h, int enable);
 CKPT_API int ckpt_phase_times(ckpt_handle h, float* times, int n);
 

@@ -220,10 +220,11 @@ class Checkpointer:
         lib().ckpt_set_profiling(self._h, 1 if on else 0)
 
     def phase_times(self) -> dict:
-        t = (ctypes.c_float * 6)()
-        lib().ckpt_phase_times(self._h, t, 6)
-        names = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total"]
-        return {names[i]: t[i] for i in range(6)}
+        t = (ctypes.c_float * 10)()
+        lib().ckpt_phase_times(self._h, t, 10)
+        names = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total",
+                 "host_pre", "host_enqueue", "host_sync_wait", "host_post"]
+        return {names[i]: t[i] for i in range(10)}
 
     def close(self) -> None:
         if getattr(self, "_h", None):

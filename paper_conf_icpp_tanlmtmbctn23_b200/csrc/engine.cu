@@ -10,22 +10,19 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstring>
 #include <new>
 #include <vector>
 
 #include "../../include/ckpt.h"
+#include "arena.h"
 #include "kernels.h"
 
 using namespace ckpt;
 
 namespace {
-
-struct ArenaBlock {
-  uint8_t* ptr;
-  uint64_t size, used;
-};
 
 struct DiffRec {
   ckpt_diff info;
@@ -36,7 +33,7 @@ struct DiffRec {
 
 constexpr double kMaxLoad = 0.8;     // reserve so that even a worst-case checkpoint stays below this
 constexpr double kGrowLoad = 0.6;    // load factor right after a growth
-constexpr uint64_t kArenaMin = 256ull << 20;
+constexpr uint64_t kArenaVA[] = {4ull << 40, 1ull << 40, 256ull << 30, 64ull << 30};
 
 }  // namespace
 
@@ -70,14 +67,14 @@ struct ckpt_ctx {
   Totals* tot_host = nullptr;   // pinned
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
-  std::vector<ArenaBlock> arena;
+  DiffArena arena;
   std::vector<DiffRec> diffs;
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
   cudaStream_t internal = nullptr;
   bool prof = false;
   cudaEvent_t ev[6] = {};
-  float times[6] = {};
+  float times[12] = {};
   PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   std::vector<void*> allocs;   // per-geometry allocations
 };
@@ -165,6 +162,10 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->freg_src, n + 1);
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
+  bool reserved = false;
+  for (uint64_t va : kArenaVA)
+    if (va >= 4 * (h->B + 12 * n + 1024) && h->arena.reserve(va)) { reserved = true; break; }
+  if (!reserved) return CKPT_ENOMEM;
   h->geo_set = true;
   return CKPT_OK;
 }
@@ -201,25 +202,6 @@ int ensure_table(ckpt_ctx* h, cudaStream_t st) {
   }
   h->tab = nt;
   h->cap = new_cap;
-  return CKPT_OK;
-}
-
-int reserve_arena(ckpt_ctx* h, uint64_t worst, uint8_t** out) {
-  if (!h->arena.empty()) {
-    ArenaBlock& b = h->arena.back();
-    if (b.size - b.used >= worst) {
-      *out = b.ptr + b.used;
-      return CKPT_OK;
-    }
-  }
-  const uint64_t size = std::max(worst, kArenaMin);
-  void* p = nullptr;
-  if (cudaMalloc(&p, size) != cudaSuccess) {
-    cudaGetLastError();
-    return CKPT_ENOMEM;
-  }
-  h->arena.push_back(ArenaBlock{static_cast<uint8_t*>(p), size, 0});
-  *out = static_cast<uint8_t*>(p);
   return CKPT_OK;
 }
 
@@ -306,6 +288,10 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
     return CKPT_ECUDA;
   }
   h->encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  if (!h->arena.init(dev)) {
+    delete h;
+    return CKPT_ECUDA;
+  }
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaMallocHost(&h->tot_host, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaMalloc(&h->tot, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ENOMEM; }
@@ -318,7 +304,7 @@ int ckpt_destroy(ckpt_handle h) {
   if (!h) return CKPT_EINVAL;
   cudaDeviceSynchronize();
   for (void* p : h->allocs) cudaFree(p);
-  for (auto& b : h->arena) cudaFree(b.ptr);
+  h->arena.release_all();
   for (auto& d : h->diffs) { if (d.Flo) cudaFree(d.Flo); if (d.Foff) cudaFree(d.Foff); }
   if (h->tab) cudaFree(h->tab);
   if (h->tot) cudaFree(h->tot);
@@ -345,11 +331,14 @@ int ckpt_set_profiling(ckpt_handle h, int enable) {
 
 int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
-  for (int i = 0; i < n && i < 6; ++i) times[i] = h->times[i];
+  for (int i = 0; i < n && i < 12; ++i) times[i] = h->times[i];
   return CKPT_OK;
 }
 
 int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
+  using clk = std::chrono::steady_clock;
+  const auto t_entry = clk::now();
+  auto ms_since = [](clk::time_point a, clk::time_point b) { return std::chrono::duration<float, std::milli>(b - a).count(); };
   if (!h) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
   if (!dev_ptr || !diff || bytes == 0 || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
@@ -369,9 +358,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   int r = ensure_table(h, st);
   if (r != CKPT_OK) return r;
   const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
-  uint8_t* out = nullptr;
-  r = reserve_arena(h, worst, &out);
-  if (r != CKPT_OK) return r;
+  if (!h->arena.ensure(worst)) return CKPT_ENOMEM;
+  uint8_t* out = h->arena.top_ptr();
 
   const Geo g = make_geo(h, k);
   const uint8_t* buf = static_cast<const uint8_t*>(dev_ptr);
@@ -406,6 +394,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     if (r != CKPT_OK) { h->poisoned = true; return r; }
   }
 
+  const auto t_pre = clk::now();
   CK(cudaMemsetAsync(h->tot, 0, sizeof(Totals), st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
@@ -458,7 +447,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
   CK(cudaMemcpyAsync(h->tot_host, h->tot, sizeof(Totals), cudaMemcpyDeviceToHost, st));
+  const auto t_launched = clk::now();
   CK(cudaStreamSynchronize(st));   // the one host synchronisation of the call
+  const auto t_synced = clk::now();
 
   const Totals t = *h->tot_host;
   if (h->prof) {
@@ -470,10 +461,15 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   DiffRec rec;
   rec.ptr = out;
   fill_diff(h, k, t, out, &rec.info);
-  ArenaBlock& blk = h->arena.back();
-  blk.used += (rec.info.bytes + 255) & ~255ull;
+  h->arena.commit(rec.info.bytes);
   h->diffs.push_back(rec);
   *diff = rec.info;
+  // host-side timings: [6] entry->first enqueue, [7] enqueue of the sequence, [8] sync wait, [9] post
+  const auto t_exit = clk::now();
+  h->times[6] = ms_since(t_entry, t_pre);
+  h->times[7] = ms_since(t_pre, t_launched);
+  h->times[8] = ms_since(t_launched, t_synced);
+  h->times[9] = ms_since(t_synced, t_exit);
   return t.collisions ? CKPT_ECOLLIDE : CKPT_OK;
 }
 

@@ -143,24 +143,44 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
 }
 
 // ------------------------------------------------------------------ K1b
+// One warp per 32 candidate-mask words (1024 chunks). The warp's candidates are spread
+// evenly over its lanes (warp prefix over popcounts; lane j takes candidate j, j+32, ...)
+// so a clustered run of changed chunks costs ceil(count/32) dependent insert chains, not
+// one chain per candidate of the densest word.
 __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
-  const int lane = threadIdx.x & 31;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint64_t wbase = warp * 32;                 // first mask word of this warp
   __shared__ uint32_t s_cnt, s_base;
   __shared__ uint32_t s_tiles[256];
+  __shared__ uint32_t s_word[8][32], s_excl[8][32];
   if (threadIdx.x == 0) s_cnt = 0;
   __syncthreads();
 
-  uint32_t word = (wbase + lane < p.nwords) ? p.cand[wbase + lane] : 0u;
-  uint32_t nfound = 0;
-  while (__any_sync(0xffffffffu, word != 0)) {
-    const bool has = word != 0;
+  const uint32_t word = (wbase + lane < p.nwords) ? p.cand[wbase + lane] : 0u;
+  const uint32_t cnt = __popc(word);
+  uint32_t incl = cnt;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  s_word[wid][lane] = word;
+  s_excl[wid][lane] = incl - cnt;
+  __syncwarp();
+
+  for (uint32_t base = 0; base < total; base += 32) {
+    const uint32_t j = base + lane;
+    const bool has = j < total;
     const unsigned active = __ballot_sync(0xffffffffu, has);
     if (has) {
-      const int b = __ffs(word) - 1;
-      word &= word - 1;
-      const uint64_t c = (wbase + lane) * 32 + b;
+      // source lane: last l with excl[l] <= j
+      int lo = 0;
+#pragma unroll
+      for (int step = 16; step > 0; step >>= 1)
+        if (lo + step < 32 && s_excl[wid][lo + step] <= j) lo += step;
+      const uint32_t b = __fns(s_word[wid][lo], 0, (int)(j - s_excl[wid][lo]) + 1);
+      const uint64_t c = (wbase + lo) * 32 + b;
       const ulonglong2 v = reinterpret_cast<const ulonglong2*>(p.prev)[c];
       const Digest d{v.x, v.y};
       const uint32_t node = node_of_chunk(p.g, c);
@@ -172,8 +192,8 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
       uint32_t minnode = node;   // minimum node id of the group (every active lane shuffles)
       for (unsigned a = active; a; a &= a - 1) {
         const int sl = __ffs(a) - 1;
-        const uint32_t v = __shfl_sync(active, node, sl);
-        if ((grp >> sl) & 1u) minnode = v < minnode ? v : minnode;
+        const uint32_t vv = __shfl_sync(active, node, sl);
+        if ((grp >> sl) & 1u) minnode = vv < minnode ? vv : minnode;
       }
       uint32_t slot = 0;
       if (lane == leader) {
@@ -182,7 +202,6 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
       }
       slot = __shfl_sync(active, slot, leader);
       p.slot_of[c] = slot;
-      ++nfound;
       // dirty stage-0 tile of this chunk (R3 virtual positions)
       const uint32_t T = (uint32_t)(vpos_of_chunk(p.g, c) >> p.g.t0);
       const unsigned tg = __match_any_sync(active, T);
@@ -195,14 +214,12 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
       }
     }
   }
-  // candidate count (warp aggregate)
-  for (int o = 16; o > 0; o >>= 1) nfound += __shfl_xor_sync(0xffffffffu, nfound, o);
-  if (lane == 0 && nfound) atomicAdd(&p.tot->n_cand, (unsigned long long)nfound);
+  if (lane == 0 && total) atomicAdd(&p.tot->n_cand, (unsigned long long)total);
   __syncthreads();
-  const uint32_t cnt = s_cnt < 256 ? s_cnt : 256;
-  if (threadIdx.x == 0 && cnt) s_base = atomicAdd(&p.tot->wl_count[0], cnt);
+  const uint32_t nt = s_cnt < 256 ? s_cnt : 256;
+  if (threadIdx.x == 0 && nt) s_base = atomicAdd(&p.tot->wl_count[0], nt);
   __syncthreads();
-  if (threadIdx.x < cnt) p.wl0[s_base + threadIdx.x] = s_tiles[threadIdx.x];
+  if (threadIdx.x < nt) p.wl0[s_base + threadIdx.x] = s_tiles[threadIdx.x];
 }
 
 // ------------------------------------------------------------------ rehash
