@@ -26,29 +26,52 @@ namespace mm {
 constexpr uint64_t c1 = 0x87c37b91114253d5ull;
 constexpr uint64_t c2 = 0x4cf5ad432745937full;
 
+// 64-bit rotate as two 32-bit funnel shifts (SHF.L.W), r in 1..63 (compile-time).
+template <int R>
+__device__ __forceinline__ uint64_t rotl(uint64_t x) {
+  const uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+  uint32_t nlo, nhi;
+  if (R < 32) {
+    nhi = __funnelshift_l(lo, hi, R);
+    nlo = __funnelshift_l(hi, lo, R);
+  } else {
+    nhi = __funnelshift_l(hi, lo, R - 32);
+    nlo = __funnelshift_l(lo, hi, R - 32);
+  }
+  return ((uint64_t)nhi << 32) | nlo;
+}
 __device__ __forceinline__ uint64_t rotl(uint64_t x, int r) { return (x << r) | (x >> (64 - r)); }
+
+// x * C mod 2^64 as IMAD.WIDE.U32 + 2 IMAD (C a compile-time constant)
+template <uint64_t C>
+__device__ __forceinline__ uint64_t mulc(uint64_t x) {
+  const uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+  const uint64_t w = (uint64_t)lo * (uint32_t)C;
+  const uint32_t h = (uint32_t)(w >> 32) + hi * (uint32_t)C + lo * (uint32_t)(C >> 32);
+  return ((uint64_t)h << 32) | (uint32_t)w;
+}
 
 __device__ __forceinline__ uint64_t fmix(uint64_t k) {
   k ^= k >> 33;
-  k *= 0xff51afd7ed558ccdull;
+  k = mulc<0xff51afd7ed558ccdull>(k);
   k ^= k >> 33;
-  k *= 0xc4ceb9fe1a85ec53ull;
+  k = mulc<0xc4ceb9fe1a85ec53ull>(k);
   k ^= k >> 33;
   return k;
 }
 
 // One 16-byte body block (k1 = bytes 0..7 LE, k2 = bytes 8..15 LE).
 __device__ __forceinline__ void block(uint64_t& h1, uint64_t& h2, uint64_t k1, uint64_t k2) {
-  k1 *= c1; k1 = rotl(k1, 31); k1 *= c2; h1 ^= k1;
-  h1 = rotl(h1, 27); h1 += h2; h1 = h1 * 5 + 0x52dce729ull;
-  k2 *= c2; k2 = rotl(k2, 33); k2 *= c1; h2 ^= k2;
-  h2 = rotl(h2, 31); h2 += h1; h2 = h2 * 5 + 0x38495ab5ull;
+  k1 = mulc<c1>(k1); k1 = rotl<31>(k1); k1 = mulc<c2>(k1); h1 ^= k1;
+  h1 = rotl<27>(h1); h1 += h2; h1 = h1 * 5 + 0x52dce729ull;
+  k2 = mulc<c2>(k2); k2 = rotl<33>(k2); k2 = mulc<c1>(k2); h2 ^= k2;
+  h2 = rotl<31>(h2); h2 += h1; h2 = h2 * 5 + 0x38495ab5ull;
 }
 
 // Tail of 1..15 bytes already packed little-endian into t1 (bytes 0..7) / t2 (8..14).
 __device__ __forceinline__ void tail(uint64_t& h1, uint64_t& h2, uint64_t t1, uint64_t t2, unsigned rem) {
-  if (rem > 8) { t2 *= c2; t2 = rotl(t2, 33); t2 *= c1; h2 ^= t2; }
-  if (rem > 0) { t1 *= c1; t1 = rotl(t1, 31); t1 *= c2; h1 ^= t1; }
+  if (rem > 8) { t2 = mulc<c2>(t2); t2 = rotl<33>(t2); t2 = mulc<c1>(t2); h2 ^= t2; }
+  if (rem > 0) { t1 = mulc<c1>(t1); t1 = rotl<31>(t1); t1 = mulc<c2>(t1); h1 ^= t1; }
 }
 
 __device__ __forceinline__ Digest finish(uint64_t h1, uint64_t h2, uint64_t len) {

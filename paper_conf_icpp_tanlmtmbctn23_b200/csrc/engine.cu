@@ -57,13 +57,21 @@ struct ckpt_ctx {
   uint32_t* dirty[kMaxStages] = {};
   uint32_t* wl[kMaxStages] = {};
   LevelIO lvl[kMaxStages] = {};
+  Digest* tdig[kMaxStages] = {};
+  unsigned long long* tsrc[kMaxStages] = {};
+  uint32_t* cnt[kMaxStages] = {};
+  uint32_t* done2[kMaxStages] = {};
+  uint32_t* done3[kMaxStages] = {};
+  uint8_t* ctr = nullptr;        // Totals + per-stage counters, zeroed by one memset per call
+  size_t ctr_bytes = 0;
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
+  uint32_t* lmask = nullptr;
   uint4* toff = nullptr;
   unsigned long long* blocksum = nullptr;
-  unsigned long long* freg_off = nullptr;
-  unsigned long long* freg_src = nullptr;
-  Totals* tot = nullptr;
+  ulonglong2* big = nullptr;
+  unsigned long long* big_len = nullptr;
+  Totals* tot = nullptr;         // = (Totals*)ctr
   Totals* tot_host = nullptr;   // pinned
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
@@ -153,13 +161,34 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
       AL(h->lvl[s].dig, P);
       AL(h->lvl[s].src, P);
     }
+    const uint64_t slots = h->ngroups[s] << h->gsz[s];
+    AL(h->tdig[s], slots);
+    AL(h->tsrc[s], 2 * slots);
+  }
+  // per-call counters: Totals, then cnt/done2/done3 of every stage s >= 1
+  {
+    size_t bytes = (sizeof(Totals) + 255) & ~size_t(255);
+    size_t off[kMaxStages] = {};
+    for (int s = 1; s < h->S; ++s) {
+      off[s] = bytes;
+      bytes += 3 * h->ngroups[s] * sizeof(uint32_t);
+    }
+    AL(h->ctr, bytes);
+    h->ctr_bytes = bytes;
+    h->tot = reinterpret_cast<Totals*>(h->ctr);
+    for (int s = 1; s < h->S; ++s) {
+      h->cnt[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
+      h->done2[s] = h->cnt[s] + h->ngroups[s];
+      h->done3[s] = h->done2[s] + h->ngroups[s];
+    }
   }
   AL(h->scratch, n_tiles << h->t0);
   AL(h->tilecnt, n_tiles);
+  AL(h->lmask, n_tiles * 128);
   AL(h->toff, n_tiles);
   AL(h->blocksum, 3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3);
-  AL(h->freg_off, n + 1);
-  AL(h->freg_src, n + 1);
+  AL(h->big, B / (1 << 20) + 2);
+  AL(h->big_len, B / (1 << 20) + 2);
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
   bool reserved = false;
@@ -294,7 +323,6 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
   }
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaMallocHost(&h->tot_host, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  if (cudaMalloc(&h->tot, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ENOMEM; }
   for (int i = 0; i < 6; ++i) cudaEventCreate(&h->ev[i]);
   *out = h;
   return CKPT_OK;
@@ -307,7 +335,6 @@ int ckpt_destroy(ckpt_handle h) {
   h->arena.release_all();
   for (auto& d : h->diffs) { if (d.Flo) cudaFree(d.Flo); if (d.Foff) cudaFree(d.Foff); }
   if (h->tab) cudaFree(h->tab);
-  if (h->tot) cudaFree(h->tot);
   if (h->tot_host) cudaFreeHost(h->tot_host);
   if (h->staging) cudaFree(h->staging);
   for (int i = 0; i < 6; ++i) if (h->ev[i]) cudaEventDestroy(h->ev[i]);
@@ -395,7 +422,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   }
 
   const auto t_pre = clk::now();
-  CK(cudaMemsetAsync(h->tot, 0, sizeof(Totals), st));
+  CK(cudaMemsetAsync(h->ctr, 0, h->ctr_bytes, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
   CK(launch_leaf_tail(lp, st));
@@ -405,36 +432,42 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   InsertParams ip;
   ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
   ip.tab = h->tab; ip.cap = h->cap; ip.slot_of = h->slot_of;
-  ip.dirty0 = h->dirty[0]; ip.wl0 = h->wl[0]; ip.tot = h->tot;
+  ip.wl0 = h->wl[0]; ip.tot = h->tot;
+  ip.S = h->S;
+  for (int s = 0; s < kMaxStages; ++s) {
+    ip.dirty[s] = h->dirty[s];
+    ip.cnt[s] = h->cnt[s];
+    ip.gsz[s] = h->gsz[s];
+  }
   CK(launch_insert(ip, st));
   if (h->prof) CK(cudaEventRecord(h->ev[2], st));
 
-  // ---- phase 2 (all stages), then phase 3 (all stages): R11
+  // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11
   TreeParams tp;
   std::memset(&tp, 0, sizeof(tp));
   tp.g = g;
+  tp.S = h->S;
+  tp.n_tiles = h->ngroups[0];
+  tp.wl0 = h->wl[0];
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
-  tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.tot = h->tot;
-  for (int phase = 2; phase <= 3; ++phase) {
-    for (int s = 0; s < h->S; ++s) {
-      tp.s = s;
-      tp.Lin = h->Lin[s];
-      tp.gsz = h->gsz[s];
-      tp.last = (s == h->S - 1);
-      tp.wl = h->wl[s];
-      tp.wl_slot = s;
-      tp.dirty_in = s >= 1 ? h->dirty[s - 1] : nullptr;
-      tp.in = s >= 1 ? h->lvl[s] : LevelIO{};
-      tp.out = !tp.last ? h->lvl[s + 1] : LevelIO{};
-      tp.dirty_next = !tp.last ? h->dirty[s + 1] : nullptr;
-      tp.wl_next = !tp.last ? h->wl[s + 1] : nullptr;
-      tp.g_next = !tp.last ? h->gsz[s + 1] : 0;
-      if (phase == 2) CK(launch_phase2(tp, h->ngroups[s], h->num_sms, st));
-      else CK(launch_phase3(tp, h->ngroups[s], h->num_sms, st));
-    }
-    if (h->prof) CK(cudaEventRecord(h->ev[phase == 2 ? 3 : 4], st));
+  tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
+  for (int s = 0; s < h->S; ++s) {
+    StageParams& sp = tp.st[s];
+    sp.Lin = h->Lin[s];
+    sp.gsz = h->gsz[s];
+    sp.dirty_in = s >= 1 ? h->dirty[s - 1] : nullptr;
+    sp.in = s >= 1 ? h->lvl[s] : LevelIO{};
+    sp.tdig = h->tdig[s];
+    sp.tsrc = h->tsrc[s];
+    sp.cnt = h->cnt[s];
+    sp.done2 = h->done2[s];
+    sp.done3 = h->done3[s];
   }
+  CK(launch_tree(tp, 2, h->num_sms, st));
+  if (h->prof) CK(cudaEventRecord(h->ev[3], st));
+  CK(launch_tree(tp, 3, h->num_sms, st));
+  if (h->prof) CK(cudaEventRecord(h->ev[4], st));
 
   // ---- compaction + serialisation
   CompactParams cp;
@@ -442,7 +475,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.n_tiles = h->ngroups[0];
   cp.tilecnt = h->tilecnt; cp.scratch = h->scratch; cp.blocksum = h->blocksum;
   cp.toff = h->toff; cp.wl0 = h->wl[0]; cp.tot = h->tot;
-  cp.freg_off = h->freg_off; cp.freg_src = h->freg_src;
+  cp.big = h->big; cp.big_len = h->big_len;
   cp.out = out; cp.buf = buf;
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));

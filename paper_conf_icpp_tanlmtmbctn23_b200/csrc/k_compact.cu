@@ -126,108 +126,144 @@ __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
   }
 }
 
+// KG: one WARP per dirty tile (work-stealing cursor). Writes the tile's metadata entries
+// and copies its FIRST bytes: the tile's FIRST regions are taken 32 at a time (lane i ->
+// region i), a warp scan gives their data offsets, and the batch's bytes are copied as
+// one lane-strided stream of 16-byte units (coalesced; the region of a unit is found by
+// a 5-step search in the warp's shared table). Regions above kBig bytes are deferred to
+// KD, which spreads each over the whole grid.
+constexpr unsigned long long kBig = 1ull << 20;
+constexpr int kGW = kCT / 32;
+
+struct GatherWarp {
+  unsigned long long off[33];    // batch-relative offsets of the inline stream
+  unsigned long long dst[32];    // data-section offset of each region
+  unsigned long long src[32];    // source byte offset in the checkpoint buffer
+};
+
 __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
-  __shared__ uint4 recs[1 << kTileLog];
-  __shared__ unsigned long long wtot[kCT / 32];
+  __shared__ GatherWarp gsm[kGW];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  GatherWarp& gw = gsm[wid];
   const Geo& g = p.g;
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   const unsigned long long nF_tot = p.tot->nF;
   uint8_t* const ent_f = p.out + 64;
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint8_t* const dat = p.out + p.tot->meta_bytes;
 
-  for (uint32_t w = blockIdx.x; w < count; w += gridDim.x) {
+  for (;;) {
+    uint32_t w = 0;
+    if (lane == 0) w = atomicAdd(&p.tot->gather_next, 1u);
+    w = __shfl_sync(0xffffffffu, w, 0);
+    if (w >= count) break;
     const uint32_t T = p.wl0[w];
     const uint4 cnt = p.tilecnt[T];
+    if (cnt.w != g.epoch) continue;
     const uint32_t nF = cnt.x, nS = cnt.y;
-    if (nF + nS == 0) continue;   // uniform across the CTA
+    if (nF + nS == 0) continue;
     const uint4 off = p.toff[T];
     const unsigned long long doff = (unsigned long long)off.z | ((unsigned long long)off.w << 32);
-    const uint4* src = p.scratch + ((uint64_t)T << g.t0);
-    for (uint32_t i = threadIdx.x; i < nF + nS; i += kCT) recs[i] = src[i];
-    __syncthreads();
-    // metadata entries (R13): FIRST = u32 node; SHIFT = u32 node, u32 src node, u32 src ckpt
-    for (uint32_t i = threadIdx.x; i < nF; i += kCT)
-      *reinterpret_cast<uint32_t*>(ent_f + 4ull * (off.x + i)) = recs[i].x;
-    for (uint32_t i = threadIdx.x; i < nS; i += kCT) {
-      uint32_t* e = reinterpret_cast<uint32_t*>(ent_s + 12ull * (off.y + i));
+    const uint4* recs = p.scratch + ((uint64_t)T << g.t0);
+    // SHIFT entries (R13): u32 node, u32 src node, u32 src ckpt
+    for (uint32_t i = lane; i < nS; i += 32) {
       const uint4 r = recs[nF + i];
+      uint32_t* e = reinterpret_cast<uint32_t*>(ent_s + 12ull * (off.y + i));
       e[0] = r.x; e[1] = r.y; e[2] = r.z;
     }
-    // FIRST regions: global data offset and source offset, for the data pass (KD)
+    // FIRST entries + data, 32 regions per batch
     unsigned long long carry = doff;
-    for (uint32_t b0 = 0; b0 < nF; b0 += kCT) {
-      const uint32_t i = b0 + threadIdx.x;
+    for (uint32_t b0 = 0; b0 < nF; b0 += 32) {
+      const uint32_t i = b0 + lane;
       unsigned long long len = 0, s0 = 0;
       if (i < nF) {
         const uint32_t node = recs[i].x;
+        *reinterpret_cast<uint32_t*>(ent_f + 4ull * (off.x + i)) = node;
         const int depth = 31 - __clz(node + 1);
-        const int L = g.h - depth;
         uint64_t lo, hi;
-        chunk_range(g, L, (uint64_t)node + 1 - (1ull << depth), lo, hi);
+        chunk_range(g, g.h - depth, (uint64_t)node + 1 - (1ull << depth), lo, hi);
         len = range_bytes(g, lo, hi);
         s0 = lo * (unsigned long long)g.C;
       }
-      unsigned long long incl = len;
+      const bool big = len > kBig;
+      const unsigned long long leff = big ? 0 : len;
+      unsigned long long incl = len, ieff = leff;
+#pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
         const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += u;
+        const unsigned long long v = __shfl_up_sync(0xffffffffu, ieff, o);
+        if (lane >= o) { incl += u; ieff += v; }
       }
-      if (lane == 31) wtot[wid] = incl;
-      __syncthreads();
-      unsigned long long wo = 0, bt = 0;
-      for (int k = 0; k < kCT / 32; ++k) {
-        if (k < wid) wo += wtot[k];
-        bt += wtot[k];
+      const unsigned long long my_dst = carry + incl - len;
+      if (big) {
+        const uint32_t slot = atomicAdd(&p.tot->big_count, 1u);
+        p.big[slot] = make_ulonglong2(my_dst, s0);
+        p.big_len[slot] = len;
       }
-      if (i < nF) {
-        p.freg_off[off.x + i] = carry + wo + incl - len;
-        p.freg_src[off.x + i] = s0;
+      gw.off[lane] = ieff - leff;
+      gw.dst[lane] = my_dst;
+      gw.src[lane] = s0;
+      const unsigned long long btot = __shfl_sync(0xffffffffu, ieff, 31);
+      if (lane == 31) gw.off[32] = btot;
+      carry += __shfl_sync(0xffffffffu, incl, 31);
+      __syncwarp();
+      const uint32_t nreg = (nF - b0) < 32 ? (nF - b0) : 32;
+      // stream copy of the inline bytes: unit x covers [16x, 16x+16)
+      const unsigned long long nunits = (btot + 15) / 16;
+      for (unsigned long long x0 = 0; x0 < nunits; x0 += 128) {
+        uint4 v[4];
+        uint8_t* d[4];
+        unsigned long long rem[4];
+        const uint8_t* sp[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const unsigned long long x = x0 + u * 32 + lane;
+          rem[u] = 0;
+          if (x < nunits) {
+            const unsigned long long o = 16 * x;
+            int r = 0;
+#pragma unroll
+            for (int step = 16; step > 0; step >>= 1)
+              if (r + step < (int)nreg && gw.off[r + step] <= o) r += step;
+            // skip zero-length (deferred big) regions that share this offset
+            while (r + 1 < (int)nreg && gw.off[r + 1] <= o) ++r;
+            const unsigned long long rel = o - gw.off[r];
+            sp[u] = p.buf + gw.src[r] + rel;
+            d[u] = dat + gw.dst[r] + rel;
+            rem[u] = gw.off[r + 1 <= (int)nreg ? r + 1 : nreg] - o;
+            if (r + 1 >= (int)nreg) rem[u] = btot - o;
+            if (rem[u] >= 16) v[u] = __ldg(reinterpret_cast<const uint4*>(sp[u]));
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          if (rem[u] >= 16) *reinterpret_cast<uint4*>(d[u]) = v[u];
+          else
+            for (unsigned long long b = 0; b < rem[u]; ++b) d[u][b] = sp[u][b];
+        }
       }
-      carry += bt;
-      __syncthreads();
+      __syncwarp();
     }
-    __syncthreads();   // recs[] is reused by the next tile
   }
 }
 
-// KD: copy all first-occurrence bytes into the data section. Each warp owns an 8-KiB
-// segment of the data stream, finds the FIRST region holding the segment start by
-// binary search once, then walks forward with coalesced 16-byte loads/stores.
-constexpr unsigned long long kSeg = 8192;
-
+// KD: first-occurrence regions above kBig bytes (e.g. a fully new checkpoint is one
+// region), each spread over the whole grid with coalesced 16-byte units.
 __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
-  const unsigned long long D = p.tot->data_bytes;
-  const unsigned long long nF = p.tot->nF;
-  if (D == 0) return;
+  const uint32_t nbig = *(volatile uint32_t*)&p.tot->big_count;
+  if (nbig == 0) return;
   uint8_t* const dat = p.out + p.tot->meta_bytes;
-  const int lane = threadIdx.x & 31;
-  const unsigned long long nseg = (D + kSeg - 1) / kSeg;
-  const unsigned long long wglobal = ((unsigned long long)blockIdx.x * kCT + threadIdx.x) >> 5;
-  const unsigned long long nwarps = ((unsigned long long)gridDim.x * kCT) >> 5;
-  for (unsigned long long sg = wglobal; sg < nseg; sg += nwarps) {
-    const unsigned long long s0 = sg * kSeg;
-    unsigned long long lo = 0, hi = nF;            // last region with off <= s0
-    while (hi - lo > 1) {
-      const unsigned long long mid = (lo + hi) >> 1;
-      if (__ldg(p.freg_off + mid) <= s0) lo = mid; else hi = mid;
-    }
-    unsigned long long r = lo;
-    unsigned long long next = (r + 1 < nF) ? __ldg(p.freg_off + r + 1) : ~0ull;
-    const unsigned long long send = (s0 + kSeg < D) ? s0 + kSeg : D;
-    for (unsigned long long o = s0 + 16ull * lane; o < send; o += 512) {
-      while (o >= next) {
-        ++r;
-        next = (r + 1 < nF) ? __ldg(p.freg_off + r + 1) : ~0ull;
-      }
-      const unsigned long long s = __ldg(p.freg_src + r) + (o - __ldg(p.freg_off + r));
-      uint8_t* d = dat + o;
-      if (o + 16 <= D) {
-        *reinterpret_cast<uint4*>(d) = __ldg(reinterpret_cast<const uint4*>(p.buf + s));
-      } else {
-        for (unsigned long long b = 0; b < D - o; ++b) d[b] = p.buf[s + b];
-      }
-    }
+  const unsigned long long stride = (unsigned long long)gridDim.x * kCT * 16;
+  for (uint32_t b = 0; b < nbig; ++b) {
+    const ulonglong2 e = p.big[b];
+    const unsigned long long len = p.big_len[b];
+    const uint8_t* s = p.buf + e.y;
+    uint8_t* d = dat + e.x;
+    const unsigned long long full = len & ~15ull;
+    for (unsigned long long o = ((unsigned long long)blockIdx.x * kCT + threadIdx.x) * 16; o < full; o += stride)
+      *reinterpret_cast<uint4*>(d + o) = __ldg(reinterpret_cast<const uint4*>(s + o));
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+      for (unsigned long long o = full; o < len; ++o) d[o] = s[o];
   }
 }
 
@@ -235,10 +271,10 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
   const unsigned nblk = (unsigned)((p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock);
   reduce_kernel<<<nblk, kCT, 0, st>>>(p);
   offsets_kernel<<<nblk, kCT, 0, st>>>(p);
-  uint64_t grid = (uint64_t)num_sms * 4;
-  if (grid > p.n_tiles) grid = p.n_tiles;
+  uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
+  if (grid > (uint64_t)num_sms * 8) grid = (uint64_t)num_sms * 8;
   gather_kernel<<<(unsigned)grid, kCT, 0, st>>>(p);
-  data_kernel<<<(unsigned)(num_sms * 8), kCT, 0, st>>>(p);
+  data_kernel<<<(unsigned)(num_sms * 4), kCT, 0, st>>>(p);
   return cudaGetLastError();
 }
 

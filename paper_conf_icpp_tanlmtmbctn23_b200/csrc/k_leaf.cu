@@ -31,19 +31,19 @@ __device__ __forceinline__ bool leaf_is_candidate(const Geo& g, const Digest& d,
 template <int MODE3D>
 __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  // 1024-B alignment for the 128B swizzle atom
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
+  const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
+  uint8_t* const data = smem_raw + pad;                                    // nst * stage_bytes
   const int nst = p.nst;
   const uint32_t stage_bytes = p.stage_bytes;
-  uint8_t* data = smem;                                            // nst * stage_bytes
-  Digest* prevbuf = reinterpret_cast<Digest*>(smem + nst * stage_bytes);  // nst * 256 digests
-  uint64_t* bars = reinterpret_cast<uint64_t*>(prevbuf + nst * kLeafThreads);
+  Digest* const prevbuf = reinterpret_cast<Digest*>(data + nst * stage_bytes);   // nst * 256 digests
+  uint64_t* const bars = reinterpret_cast<uint64_t*>(prevbuf + nst * kLeafThreads);
 
   const int tid = threadIdx.x;
-  const uint64_t n_tiles = p.n_main / kLeafThreads;
+  const uint32_t n_tiles = (uint32_t)(p.n_main / kLeafThreads);
   const int segs = p.segs;
-  const uint64_t my_tiles = (blockIdx.x < n_tiles) ? (n_tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-  const uint64_t total = my_tiles * (uint64_t)segs;
+  const uint32_t my_tiles = (blockIdx.x < n_tiles) ? (n_tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+  const uint32_t total = my_tiles * (uint32_t)segs;
   const bool use_prev = p.g.k > 0;
 
   if (tid == 0) {
@@ -53,32 +53,34 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   }
   __syncthreads();
 
-  auto issue = [&](uint64_t step) {
-    const int st = (int)(step % nst);
-    const uint64_t tile = blockIdx.x + (step / segs) * gridDim.x;
-    const int seg = (int)(step % segs);
-    const bool with_prev = use_prev && seg == segs - 1;
-    mbar_arrive_expect_tx(&bars[st], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
+  // producer state (thread 0): next step to issue, as (stage, tile, seg) counters
+  int is_st = 0, is_seg = 0;
+  uint32_t is_tile = blockIdx.x, issued = 0;
+  auto issue_next = [&]() {
+    const bool with_prev = use_prev && is_seg == segs - 1;
+    mbar_arrive_expect_tx(&bars[is_st], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
     if (MODE3D)
-      tma_load_3d(data + (size_t)st * stage_bytes, &tmap, &bars[st], 0, seg, (int)(tile * kLeafThreads));
+      tma_load_3d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, is_seg, (int)(is_tile * kLeafThreads));
     else
-      tma_load_2d(data + (size_t)st * stage_bytes, &tmap, &bars[st], 0, (int)(tile * (stage_bytes / 128)));
-    if (with_prev) bulk_load(prevbuf + st * kLeafThreads, p.prev + tile * kLeafThreads, kLeafThreads * 16u, &bars[st]);
+      tma_load_2d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, (int)(is_tile * (stage_bytes / 128)));
+    if (with_prev)
+      bulk_load(prevbuf + is_st * kLeafThreads, p.prev + (uint64_t)is_tile * kLeafThreads, kLeafThreads * 16u, &bars[is_st]);
+    ++issued;
+    if (++is_st == nst) is_st = 0;
+    if (++is_seg == segs) { is_seg = 0; is_tile += gridDim.x; }
   };
-
   if (tid == 0)
-    for (uint64_t s = 0; s < (uint64_t)nst && s < total; ++s) issue(s);
+    while (issued < (uint32_t)nst && issued < total) issue_next();
 
   const int units = MODE3D ? 8 : (int)(p.g.C / 16);   // 16-byte blocks of this thread per stage
+  const uint32_t ubase = (uint32_t)tid * (uint32_t)units;
   uint64_t h1 = 0, h2 = 0;
-  for (uint64_t step = 0; step < total; ++step) {
-    const int st = (int)(step % nst);
-    const int seg = (int)(step % segs);
-    const uint64_t tile = blockIdx.x + (step / segs) * gridDim.x;
-    mbar_wait(&bars[st], (uint32_t)((step / nst) & 1));
+  int st = 0, seg = 0;
+  uint32_t phase = 0, tile = blockIdx.x;
+  for (uint32_t step = 0; step < total; ++step) {
+    mbar_wait(&bars[st], phase);
     if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
     const uint8_t* sd = data + (size_t)st * stage_bytes;
-    const uint32_t ubase = (uint32_t)tid * (uint32_t)units;
 #pragma unroll 8
     for (int j = 0; j < units; ++j) {
       const uint32_t u = ubase + j;
@@ -89,7 +91,7 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
     }
     if (seg == segs - 1) {
       const Digest d = mm::finish(h1, h2, p.g.C);
-      const uint64_t c = tile * kLeafThreads + tid;
+      const uint64_t c = (uint64_t)tile * kLeafThreads + tid;
       Digest pd{0, 0};
       if (use_prev) pd = prevbuf[st * kLeafThreads + tid];
       const bool cand = leaf_is_candidate(p.g, d, pd);
@@ -98,7 +100,9 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
       if (cand) reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
     }
     __syncthreads();   // every thread is done with stage st
-    if (tid == 0 && step + nst < total) issue(step + nst);
+    if (tid == 0 && issued < total) issue_next();
+    if (++st == nst) { st = 0; phase ^= 1u; }
+    if (++seg == segs) { seg = 0; tile += gridDim.x; }
   }
 }
 
@@ -206,10 +210,18 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
       const uint32_t T = (uint32_t)(vpos_of_chunk(p.g, c) >> p.g.t0);
       const unsigned tg = __match_any_sync(active, T);
       if (lane == __ffs(tg) - 1) {
-        if (atomicExch(&p.dirty0[T], p.g.epoch) != p.g.epoch) {
+        if (atomicExch(&p.dirty[0][T], p.g.epoch) != p.g.epoch) {
           const uint32_t i = atomicAdd(&s_cnt, 1u);
           if (i < 256) s_tiles[i] = T;
           else p.wl0[atomicAdd(&p.tot->wl_count[0], 1u)] = T;   // overflow: direct append
+          // count dirty children up the stage hierarchy (the tree kernels' climb target)
+          uint64_t x = T;
+          for (int s = 1; s < p.S; ++s) {
+            const uint64_t P = x >> p.gsz[s];
+            if (atomicAdd(&p.cnt[s][P], 1u) != 0) break;
+            p.dirty[s][P] = p.g.epoch;
+            x = P;
+          }
         }
       }
     }

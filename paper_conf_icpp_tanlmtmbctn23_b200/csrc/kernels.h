@@ -4,8 +4,8 @@
 //   K1  leaf hash + fixed test (TMA-staged, persistent)      Alg.1 l.1-5, l.21
 //   K1t leaf pass for the ragged tail (direct loads)           same
 //   K1b record insert + dirty-tile worklist                    Alg.1 l.6-19 (R6)
-//   P2[s] phase-2 stages (tile, then upper levels)             Alg.1 l.24-32
-//   P3[s] phase-3 stages + emission                            Alg.1 l.33-46 (R7-R10)
+//   P2  phase 2, all stages in one launch (warp per group)     Alg.1 l.24-32
+//   P3  phase 3 + emission, all stages in one launch           Alg.1 l.33-46 (R7-R10)
 //   KR/KO/KG/KD tile reduce, offsets + header, entries, data
 #pragma once
 #include <cuda.h>
@@ -28,6 +28,10 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   unsigned long long n_first, n_spatial, n_temporal, p2_inserts;
   unsigned long long collisions, n_cand, pad0, pad1;
   uint32_t wl_count[kMaxStages];
+  uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
+  uint32_t gather_next;              // work-stealing cursor of the gather kernel
+  uint32_t big_count;                // FIRST regions deferred to the grid-wide data pass
+  uint32_t pad2[4];
 };
 
 struct LeafParams {
@@ -51,9 +55,12 @@ struct InsertParams {
   Slot* tab;
   uint64_t cap;
   uint32_t* slot_of;
-  uint32_t* dirty0;
   uint32_t* wl0;
   Totals* tot;
+  int S;                         // tree stages
+  uint32_t* dirty[kMaxStages];   // per stage: epoch mark of dirty groups
+  uint32_t* cnt[kMaxStages];     // per stage s >= 1: dirty children of each group
+  int gsz[kMaxStages];
 };
 
 struct LevelIO {               // per-position arrays at one height (stage boundary)
@@ -63,30 +70,33 @@ struct LevelIO {               // per-position arrays at one height (stage bound
   unsigned long long* src;     // packed (ckpt<<32|node) source of SHIFT positions
 };
 
+struct StageParams {
+  int Lin;                     // input height
+  int gsz;                     // log2 positions per group (levels processed)
+  const uint32_t* dirty_in;    // s >= 1: dirty marks of stage s-1 (per input position)
+  LevelIO in;                  // s >= 1: input arrays (written by stage s-1)
+  Digest* tdig;                // per group: digests of internal nodes (2^gsz entries)
+  unsigned long long* tsrc;    // per group: sources of SHIFT nodes (2 * 2^gsz entries)
+  uint32_t* cnt;               // s >= 1: dirty children per group (K1b)
+  uint32_t* done2;             // s >= 1: finished children per group, phase 2
+  uint32_t* done3;             //                                      phase 3
+};
+
 struct TreeParams {
   Geo g;
-  int s;                       // stage index
-  int Lin;                     // input height
-  int gsz;                     // group log (levels processed)
-  int last;                    // output height == h (this stage ends at the root)
-  const uint32_t* wl;          // worklist of dirty groups of this stage
-  int wl_slot;                 // Totals::wl_count index of this stage
-  const uint32_t* dirty_in;    // s >= 1: dirty marks of stage s-1 (per input position)
-  LevelIO in;                  // s >= 1
-  LevelIO out;                 // !last
-  uint32_t* dirty_next;        // phase 2: mark parent groups of stage s+1
-  uint32_t* wl_next;
-  int g_next;
-  // leaf level (s == 0)
+  int S;
+  uint64_t n_tiles;
+  const uint32_t* wl0;         // stage-0 worklist (dirty tiles)
   const uint32_t* cand;
   const uint32_t* slot_of;
   const Digest* prev;
   Slot* tab;
   uint64_t cap;
-  // emission (phase 3)
   uint4* scratch;              // per tile: up to 2^t0 region records {node, src_node, src_ckpt, kind}
   uint4* tilecnt;              // per tile: {nF, nS, data_bytes, epoch}
+  uint32_t* lmask;             // per tile: resolved leaf masks (phase 2 -> phase 3), 128 words
   Totals* tot;
+  StageParams st[kMaxStages];
 };
 
 struct CompactParams {
@@ -98,8 +108,8 @@ struct CompactParams {
   uint4* toff;                   // per tile {F_off, S_off, data_off lo, data_off hi}
   const uint32_t* wl0;
   Totals* tot;
-  unsigned long long* freg_off;   // per FIRST region (global order): offset in the data section
-  unsigned long long* freg_src;   // per FIRST region: byte offset in the checkpoint buffer
+  ulonglong2* big;               // deferred big FIRST regions: {data offset, source offset}
+  unsigned long long* big_len;   //                              byte length
   uint8_t* out;                  // diff destination (device arena)
   const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
 };
@@ -108,8 +118,7 @@ struct CompactParams {
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
 cudaError_t launch_insert(const InsertParams& p, cudaStream_t st);
-cudaError_t launch_phase2(const TreeParams& p, uint64_t n_groups, int num_sms, cudaStream_t st);
-cudaError_t launch_phase3(const TreeParams& p, uint64_t n_groups, int num_sms, cudaStream_t st);
+cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st);
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st);
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
