@@ -207,8 +207,9 @@ __device__ __forceinline__ unsigned long long table_lookup(const Slot* tab, uint
   uint64_t s = slot_home(d.lo, cap);
   for (;;) {
     const Slot* p = tab + s;
-    ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p));
-    if (kv.x == d.lo && kv.y == d.hi) return __ldcg(&p->val);
+    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p));   // key and value: one sector,
+    const unsigned long long val = __ldcg(&p->val);                         // both loads in flight
+    if (kv.x == d.lo && kv.y == d.hi) return val;
     if (kv.x == kEmpty && kv.y == kEmpty) return kEmpty;
     if (++s == cap) s = 0;
   }

@@ -12,6 +12,7 @@
 #include <algorithm>
 #include <chrono>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -85,6 +86,11 @@ struct ckpt_ctx {
   float times[12] = {};
   PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   std::vector<void*> allocs;   // per-geometry allocations
+  // diagnostics: CKPT_TRACE=<file prefix> records per-group tree timings of each call
+  const char* trace_path = nullptr;
+  int dbg = 0;
+  ulonglong4* trace = nullptr;
+  uint32_t* trace_n = nullptr;
 };
 
 #define CK(x)                                                                               \
@@ -184,13 +190,17 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   }
   AL(h->scratch, n_tiles << h->t0);
   AL(h->tilecnt, n_tiles);
-  AL(h->lmask, n_tiles * 128);
+  AL(h->lmask, n_tiles * 192);   // k_tree.cu kLmWords
   AL(h->toff, n_tiles);
   AL(h->blocksum, 3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3);
   AL(h->big, B / (1 << 20) + 2);
   AL(h->big_len, B / (1 << 20) + 2);
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
+  if (h->trace_path) {
+    if (dalloc(h, &h->trace, 24 * n_tiles + 64) != cudaSuccess || dalloc(h, &h->trace_n, 4) != cudaSuccess)
+      return CKPT_ENOMEM;
+  }
   bool reserved = false;
   for (uint64_t va : kArenaVA)
     if (va >= 4 * (h->B + 12 * n + 1024) && h->arena.reserve(va)) { reserved = true; break; }
@@ -309,6 +319,8 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
   h->device = dev;
   h->num_sms = prop.multiProcessorCount;
   h->C = chunk_bytes;
+  h->trace_path = getenv("CKPT_TRACE");
+  if (const char* d = getenv("CKPT_DBG")) h->dbg = atoi(d);
   void* fn = nullptr;
   cudaDriverEntryPointQueryResult q;
   if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) != cudaSuccess ||
@@ -317,6 +329,10 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
     return CKPT_ECUDA;
   }
   h->encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  if (leaf_setup_attributes() != cudaSuccess || tree_setup_attributes() != cudaSuccess) {
+    delete h;
+    return CKPT_ECUDA;
+  }
   if (!h->arena.init(dev)) {
     delete h;
     return CKPT_ECUDA;
@@ -452,6 +468,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
+  tp.trace = h->trace; tp.trace_n = h->trace_n;
+  tp.dbg = h->dbg;
+  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
   for (int s = 0; s < h->S; ++s) {
     StageParams& sp = tp.st[s];
     sp.Lin = h->Lin[s];
@@ -485,6 +504,17 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   const auto t_synced = clk::now();
 
   const Totals t = *h->tot_host;
+  if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
+    uint32_t nt = 0, ne = 0;
+    cudaMemcpy(&nt, h->trace_n, 4, cudaMemcpyDeviceToHost);
+    cudaMemcpy(&ne, h->trace_n + 1, 4, cudaMemcpyDeviceToHost);
+    (void)ne;
+    std::vector<ulonglong4> tr(nt);
+    cudaMemcpy(tr.data(), h->trace, nt * sizeof(ulonglong4), cudaMemcpyDeviceToHost);
+    char path[512];
+    snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
+    if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), nt, f); fclose(f); }
+  }
   if (h->prof) {
     for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&h->times[i], h->ev[i], h->ev[i + 1]);
     cudaEventElapsedTime(&h->times[5], h->ev[0], h->ev[5]);

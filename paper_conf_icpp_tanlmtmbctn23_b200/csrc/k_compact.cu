@@ -15,6 +15,7 @@
 //                      segment, coalesced 16-byte loads/stores (balanced even when one
 //                      region is the whole buffer).
 #include "kernels.h"
+#include "tma.cuh"
 
 namespace ckpt {
 
@@ -38,6 +39,8 @@ constexpr int kPer = kTilesPerBlock / kCT;
 
 __global__ void __launch_bounds__(kCT) reduce_kernel(CompactParams p) {
   __shared__ unsigned long long sh[3 * (kCT / 32)];
+  pdl_launch_dependents();
+  pdl_wait();
   unsigned long long a = 0, b = 0, c = 0;
   const uint64_t t0 = (uint64_t)blockIdx.x * kTilesPerBlock + threadIdx.x * kPer;
   for (int i = 0; i < kPer; ++i) {
@@ -58,6 +61,8 @@ __global__ void __launch_bounds__(kCT) reduce_kernel(CompactParams p) {
 __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
   __shared__ unsigned long long sh[3 * (kCT / 32)];
   __shared__ unsigned long long wx[kCT / 32], wy[kCT / 32], wz[kCT / 32];
+  pdl_launch_dependents();
+  pdl_wait();
   // prefix of earlier blocks
   unsigned long long a = 0, b = 0, c = 0;
   for (uint32_t i = threadIdx.x; i < blockIdx.x; i += kCT) {
@@ -146,6 +151,8 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   GatherWarp& gw = gsm[wid];
   const Geo& g = p.g;
+  pdl_launch_dependents();
+  pdl_wait();
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   const unsigned long long nF_tot = p.tot->nF;
   uint8_t* const ent_f = p.out + 64;
@@ -250,6 +257,7 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
 // KD: first-occurrence regions above kBig bytes (e.g. a fully new checkpoint is one
 // region), each spread over the whole grid with coalesced 16-byte units.
 __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
+  pdl_wait();
   const uint32_t nbig = *(volatile uint32_t*)&p.tot->big_count;
   if (nbig == 0) return;
   uint8_t* const dat = p.out + p.tot->meta_bytes;
@@ -269,13 +277,14 @@ __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
 
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st) {
   const unsigned nblk = (unsigned)((p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock);
-  reduce_kernel<<<nblk, kCT, 0, st>>>(p);
-  offsets_kernel<<<nblk, kCT, 0, st>>>(p);
+  cudaError_t e = launch_pdl(reduce_kernel, nblk, kCT, 0, st, p);
+  if (e == cudaSuccess) e = launch_pdl(offsets_kernel, nblk, kCT, 0, st, p);
+  if (e != cudaSuccess) return e;
   uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
   if (grid > (uint64_t)num_sms * 8) grid = (uint64_t)num_sms * 8;
-  gather_kernel<<<(unsigned)grid, kCT, 0, st>>>(p);
-  data_kernel<<<(unsigned)(num_sms * 4), kCT, 0, st>>>(p);
-  return cudaGetLastError();
+  e = launch_pdl(gather_kernel, (unsigned)grid, kCT, 0, st, p);
+  if (e == cudaSuccess) e = launch_pdl(data_kernel, (unsigned)(num_sms * 4), kCT, 0, st, p);
+  return e;
 }
 
 }  // namespace ckpt

@@ -46,6 +46,7 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   const uint32_t total = my_tiles * (uint32_t)segs;
   const bool use_prev = p.g.k > 0;
 
+  pdl_launch_dependents();
   if (tid == 0) {
     prefetch_tmap(&tmap);
     for (int s = 0; s < nst; ++s) mbar_init(&bars[s], 1);
@@ -56,15 +57,20 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   // producer state (thread 0): next step to issue, as (stage, tile, seg) counters
   int is_st = 0, is_seg = 0;
   uint32_t is_tile = blockIdx.x, issued = 0;
+  const uint64_t pol_stream = policy_evict_first();
+  const uint64_t pol_keep = policy_evict_last();
   auto issue_next = [&]() {
     const bool with_prev = use_prev && is_seg == segs - 1;
     mbar_arrive_expect_tx(&bars[is_st], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
     if (MODE3D)
-      tma_load_3d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, is_seg, (int)(is_tile * kLeafThreads));
+      tma_load_3d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, is_seg, (int)(is_tile * kLeafThreads),
+                  pol_stream);
     else
-      tma_load_2d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, (int)(is_tile * (stage_bytes / 128)));
+      tma_load_2d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, (int)(is_tile * (stage_bytes / 128)),
+                  pol_stream);
     if (with_prev)
-      bulk_load(prevbuf + is_st * kLeafThreads, p.prev + (uint64_t)is_tile * kLeafThreads, kLeafThreads * 16u, &bars[is_st]);
+      bulk_load(prevbuf + is_st * kLeafThreads, p.prev + (uint64_t)is_tile * kLeafThreads, kLeafThreads * 16u, &bars[is_st],
+                pol_stream);
     ++issued;
     if (++is_st == nst) is_st = 0;
     if (++is_seg == segs) { is_seg = 0; is_tile += gridDim.x; }
@@ -96,8 +102,8 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
       if (use_prev) pd = prevbuf[st * kLeafThreads + tid];
       const bool cand = leaf_is_candidate(p.g, d, pd);
       const unsigned mask = __ballot_sync(0xffffffffu, cand);
-      if ((tid & 31) == 0) p.cand[c >> 5] = mask;
-      if (cand) reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
+      if ((tid & 31) == 0) st_evict_last_u32(p.cand + (c >> 5), mask, pol_keep);
+      if (cand) st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
     }
     __syncthreads();   // every thread is done with stage st
     if (tid == 0 && issued < total) issue_next();
@@ -152,6 +158,7 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
 // so a clustered run of changed chunks costs ceil(count/32) dependent insert chains, not
 // one chain per candidate of the densest word.
 __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
+  pdl_launch_dependents();
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint64_t wbase = warp * 32;                 // first mask word of this warp
@@ -160,6 +167,7 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
   __shared__ uint32_t s_word[8][32], s_excl[8][32];
   if (threadIdx.x == 0) s_cnt = 0;
   __syncthreads();
+  pdl_wait();
 
   const uint32_t word = (wbase + lane < p.nwords) ? p.cand[wbase + lane] : 0u;
   const uint32_t cnt = __popc(word);
@@ -205,7 +213,7 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
         slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed);
       }
       slot = __shfl_sync(active, slot, leader);
-      p.slot_of[c] = slot;
+      st_evict_last_u32(p.slot_of + c, slot, policy_evict_last());
       // dirty stage-0 tile of this chunk (R3 virtual positions)
       const uint32_t T = (uint32_t)(vpos_of_chunk(p.g, c) >> p.g.t0);
       const unsigned tg = __match_any_sync(active, T);
@@ -258,13 +266,8 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   const uint64_t n_tiles = p.n_main / kLeafThreads;
   uint64_t grid = (uint64_t)num_sms * 2;
   if (grid > n_tiles) grid = n_tiles;
-  if (p.mode3d) {
-    cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    leaf_hash_kernel<1><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
-  } else {
-    cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    leaf_hash_kernel<0><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
-  }
+  if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
+  else leaf_hash_kernel<0><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
   return cudaGetLastError();
 }
 
@@ -278,8 +281,16 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
 cudaError_t launch_insert(const InsertParams& p, cudaStream_t st) {
   const uint64_t warps = (p.nwords + 31) / 32;
   const uint64_t blocks = (warps + 7) / 8;
-  if (blocks) insert_kernel<<<(unsigned)blocks, 256, 0, st>>>(p);
-  return cudaGetLastError();
+  if (blocks) return launch_pdl(insert_kernel, (unsigned)blocks, 256, 0, st, p);
+  return cudaSuccess;
+}
+
+cudaError_t leaf_setup_attributes() {
+  // the largest dynamic smem any leaf configuration asks for (C >= 128: 3 x 36 KB; C < 128: <= 96 KB)
+  const int smem = 1024 + 110 * 1024;
+  cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  return e;
 }
 
 cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st) {

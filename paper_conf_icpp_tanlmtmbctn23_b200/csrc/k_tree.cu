@@ -7,15 +7,21 @@
 //
 // Work unit: one WARP per group of up to 1024 positions of one height (a stage-0 tile
 // of the virtual leaf level, R3 geometry in dev.cuh, or 1024 roots of the stage below).
-// The labels of a level are bitmasks — lane w holds positions 32w..32w+31 of each class
-// (FIRST, SHIFT, FIXED) — so a level step is two shuffles and an even/odd bit split:
-// a parent is FIRST iff both children are, FIXED iff both are (R7), "SHIFT pair" iff both
-// are SHIFT, otherwise DONE (mixed). Only the set bits that need a digest (phase 2:
-// FIRST pairs -> hash + insert, Alg.1 l.28-29; phase 3: SHIFT pairs -> hash + lookup,
-// l.38-39) do memory work, spread evenly over the 32 lanes. Groups holding no
-// non-FIXED leaf are never visited (K1b builds the stage-0 worklist and counts dirty
-// children per upper group); the warp that finishes the LAST dirty child of an upper
-// group climbs and processes that group too, so every stage runs in the same launch.
+// Labels are bitmasks (FIRST, SHIFT, FIXED), one bit per position, 32 positions per
+// lane. Each level is kept in BIT-REVERSED position order, so the two children of the
+// node at index r sit at indices r and r + N/2 of the level below: a level step is one
+// shuffle and an AND (parent FIRST iff both children FIRST; FIXED iff both FIXED, R7;
+// "SHIFT pair" iff both SHIFT; otherwise DONE), with no bit compression. Leaf masks enter
+// that order once per group through a 32-ballot bit transpose.
+//
+// Digest work is batched per group instead of per level: pass 1 computes every digest
+// the group needs bottom-up from on-chip data (phase 2: FIRST pairs, Alg.1 l.28; phase 3:
+// every POTENTIAL shifted pair, l.38 — a superset of the pairs Alg.1 looks up); pass 2
+// issues all record operations at once (phase 2: insert, l.29; phase 3: lookup, l.39);
+// pass 3 (phase 3) replays the labels with the lookup results and emits the regions.
+// Groups holding no non-FIXED leaf are never visited (K1b builds the stage-0 worklist and
+// counts dirty children per upper group); the warp that finishes the LAST dirty child of
+// an upper group climbs and processes that group too, so every stage runs in this launch.
 //
 // Phase-3 emission ("save roots", R8/R10): a FIRST/SHIFT child of a DONE parent (or the
 // FIRST/SHIFT root) becomes a region. Stage 0 records its regions per tile in leaf
@@ -23,32 +29,25 @@
 // and is recorded in the tile holding its first leaf, so the per-tile lists in tile
 // order are the regions sorted by first chunk (R13) — k_compact.cu relies on it.
 #include "kernels.h"
+#include "tma.cuh"
 
 namespace ckpt {
 
 namespace {
 
 constexpr int kWarps = kTreeThreads / 32;
+constexpr int kDigCap = 256;   // on-chip digests per warp (4 KB); dense groups spill to global
+constexpr int kLmWords = 192;  // per tile: F0 S0 X0 F1 S1 leaf1 (rev order), 32 words each
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
 
 // ------------------------------------------------------------------ bit helpers
-__device__ __forceinline__ uint32_t even_bits64(uint64_t x) {   // bits 0,2,...,62 -> 0..31
-  x &= 0x5555555555555555ull;
-  x = (x | (x >> 1)) & 0x3333333333333333ull;
-  x = (x | (x >> 2)) & 0x0F0F0F0F0F0F0F0Full;
-  x = (x | (x >> 4)) & 0x00FF00FF00FF00FFull;
-  x = (x | (x >> 8)) & 0x0000FFFF0000FFFFull;
-  x = (x | (x >> 16)) & 0x00000000FFFFFFFFull;
-  return (uint32_t)x;
-}
-__device__ __forceinline__ uint32_t spread16(uint32_t x) {      // bit i -> bits 2i and 2i+1
-  x &= 0xFFFFu;
-  x = (x | (x << 8)) & 0x00FF00FFu;
-  x = (x | (x << 4)) & 0x0F0F0F0Fu;
-  x = (x | (x << 2)) & 0x33333333u;
-  x = (x | (x << 1)) & 0x55555555u;
-  return x | (x << 1);
-}
 __device__ __forceinline__ uint32_t low_mask(uint64_t nbits) { return nbits >= 32 ? 0xFFFFFFFFu : ((1u << nbits) - 1u); }
+__device__ __forceinline__ uint32_t rev_n(uint32_t x, int n) { return n ? (__brev(x) >> (32 - n)) : 0u; }
 
 // 32 bits of the candidate bitmap starting at chunk c (c may be unaligned)
 __device__ __forceinline__ uint32_t cand_bits(const uint32_t* cand, uint64_t c) {
@@ -63,18 +62,67 @@ __device__ __forceinline__ uint32_t cand_bits(const uint32_t* cand, uint64_t c) 
 struct WarpSmem {
   uint32_t pw[32];      // words of the current work mask
   uint32_t px[32];      // exclusive prefix of their popcounts
-  uint32_t hitF[32];    // result bits written by work items (FIRST / lookup hit)
-  uint32_t hitS[32];    // result bits (SHIFT leaves)
-  uint32_t stF[32];     // stage-0 emission: FIRST region start slots
+  uint32_t hitF[32];    // result bits written by work items (resolve: FIRST)
+  uint32_t hitS[32];    // result bits (resolve: SHIFT)
+  uint32_t T[32];       // scatter-transpose scratch
+  uint32_t stF[32];     // stage-0 emission: FIRST region start slots (natural order)
   uint32_t stS[32];     //                   SHIFT region start slots
+  uint32_t W[32];       // pass-1 nodes of all levels (layout below)
+  uint32_t WP[32];      // exclusive prefix of popc(W): a pass-1 node's rank = its compact digest index
+  uint32_t H[32];       // pass-2 lookup hits (same layout)
+  Digest dig[kDigCap];  // compact on-chip digests of pass-1 nodes (rank < kDigCap; others: global)
   uint8_t lvl[1 << kTileLog];   // level of the region starting at each slot
+  unsigned long long tp[8];     // diagnostics: intra-group timestamps
 };
 
+// One 32-word layout holding a bit for every internal node of a 1024-slot group:
+// level 1 -> words 0..15, level 2 -> 16..23, level 3 -> 24..27, level 4 -> 28..29,
+// level 5 -> word 30, levels 6..10 packed in word 31 at bits 0, 16, 24, 28, 30.
+__device__ __forceinline__ int lay_base(int lv) {
+  return lv == 1 ? 0 : lv == 2 ? 16 : lv == 3 ? 24 : lv == 4 ? 28 : lv == 5 ? 30 : 31;
+}
+__device__ __forceinline__ int lay_shift(int lv) {
+  return lv <= 6 ? 0 : lv == 7 ? 16 : lv == 8 ? 24 : lv == 9 ? 28 : 30;
+}
+__device__ __forceinline__ void lay_decode(uint32_t w, uint32_t b, int& lv, uint32_t& q) {
+  if (w < 16) { lv = 1; q = 32 * w + b; }
+  else if (w < 24) { lv = 2; q = 32 * (w - 16) + b; }
+  else if (w < 28) { lv = 3; q = 32 * (w - 24) + b; }
+  else if (w < 30) { lv = 4; q = 32 * (w - 28) + b; }
+  else if (w == 30) { lv = 5; q = b; }
+  else if (b < 16) { lv = 6; q = b; }
+  else if (b < 24) { lv = 7; q = b - 16; }
+  else if (b < 28) { lv = 8; q = b - 24; }
+  else if (b < 30) { lv = 9; q = b - 28; }
+  else { lv = 10; q = b - 30; }
+}
+__device__ __forceinline__ void lay_pos(int lv, uint32_t q, uint32_t& w, uint32_t& b) {
+  if (lv <= 5) { w = lay_base(lv) + (q >> 5); b = q & 31; }
+  else { w = 31; b = lay_shift(lv) + q; }
+}
+__device__ __forceinline__ uint32_t lay_rank(const WarpSmem& ws, int lv, uint32_t q) {
+  uint32_t w, b;
+  lay_pos(lv, q, w, b);
+  return ws.WP[w] + __popc(ws.W[w] & ((1u << b) - 1u));
+}
+__device__ __forceinline__ Digest dig_load(const WarpSmem& ws, const Digest* spill, uint32_t idx) {
+  if (idx < kDigCap) return ws.dig[idx];
+  const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(spill) + idx);
+  return Digest{v.x, v.y};
+}
+__device__ __forceinline__ void dig_store(WarpSmem& ws, Digest* spill, uint32_t idx, const Digest& d) {
+  if (idx < kDigCap) ws.dig[idx] = d;
+  else reinterpret_cast<ulonglong2*>(spill)[idx] = make_ulonglong2(d.lo, d.hi);
+}
+
+__device__ __forceinline__ uint64_t lvl_off(uint64_t P0, int lv) { return P0 - (P0 >> (lv - 1)); }  // lv >= 1
+
 // Balanced distribution of the set bits of per-lane words `m` (word index = lane) over
-// the 32 lanes: calls f(word, bit, position) once per set bit.
+// the 32 lanes: calls f(word, bit, index) once per set bit.
 template <class F>
 __device__ __forceinline__ void for_each_bit_balanced(WarpSmem& ws, uint32_t m, F&& f) {
   const int lane = threadIdx.x & 31;
+  if (!__any_sync(0xffffffffu, m != 0)) return;   // most levels have no work: one vote, no scan
   const uint32_t cnt = __popc(m);
   uint32_t incl = cnt;
 #pragma unroll
@@ -83,7 +131,6 @@ __device__ __forceinline__ void for_each_bit_balanced(WarpSmem& ws, uint32_t m, 
     if (lane >= o) incl += v;
   }
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  if (total == 0) return;
   ws.pw[lane] = m;
   ws.px[lane] = incl - cnt;
   __syncwarp();
@@ -101,7 +148,76 @@ __device__ __forceinline__ void for_each_bit_balanced(WarpSmem& ws, uint32_t m, 
   __syncwarp();
 }
 
-__device__ __forceinline__ uint64_t lvl_off(uint64_t P0, int lv) { return P0 - (P0 >> (lv - 1)); }  // lv >= 1
+// ---- natural order -> bit-reversed order for a level of N = 2^n positions.
+// n == 10: 32-ballot transpose (lane w first fetches natural word rev5(w)); smaller
+// levels: scatter through shared memory (small groups only).
+__device__ __forceinline__ void to_rev3(WarpSmem& ws, int n, uint32_t a, uint32_t b, uint32_t c, uint32_t& ra,
+                                        uint32_t& rb, uint32_t& rc) {
+  const int lane = threadIdx.x & 31;
+  if (n == 10) {
+    const int src = (int)rev_n((uint32_t)lane, 5);
+    a = __shfl_sync(0xffffffffu, a, src);
+    b = __shfl_sync(0xffffffffu, b, src);
+    c = __shfl_sync(0xffffffffu, c, src);
+    ra = rb = rc = 0;
+#pragma unroll
+    for (int bit = 0; bit < 32; ++bit) {
+      const uint32_t ma = __ballot_sync(0xffffffffu, (a >> bit) & 1u);
+      const uint32_t mb = __ballot_sync(0xffffffffu, (b >> bit) & 1u);
+      const uint32_t mc = __ballot_sync(0xffffffffu, (c >> bit) & 1u);
+      if (src == bit) { ra = ma; rb = mb; rc = mc; }   // rev5 is an involution: lane == rev5(bit)
+    }
+    return;
+  }
+  uint32_t* out[3] = {&ra, &rb, &rc};
+  const uint32_t in[3] = {a, b, c};
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    ws.T[lane] = 0;
+    __syncwarp();
+    for (uint32_t m = in[k]; m; m &= m - 1) {
+      const uint32_t q = lane * 32 + (__ffs(m) - 1);
+      const uint32_t r = rev_n(q, n);
+      atomicOr(&ws.T[r >> 5], 1u << (r & 31));
+    }
+    __syncwarp();
+    *out[k] = ws.T[lane];
+    __syncwarp();
+  }
+}
+
+// Children masks of this lane's parent word: left children (index r) and right children
+// (index r + Np) of a level with Nc positions in bit-reversed order.
+__device__ __forceinline__ void lr(uint32_t M, uint64_t Nc, uint32_t& l, uint32_t& r) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t Np = Nc >> 1;
+  if (Np >= 32) {
+    const int wp = (int)(Np >> 5);
+    l = M;
+    r = __shfl_sync(0xffffffffu, M, (lane + wp) & 31);
+  } else {
+    const uint32_t x = __shfl_sync(0xffffffffu, M, 0);
+    l = x & low_mask(Np);
+    r = (x >> Np) & low_mask(Np);
+  }
+}
+
+// Parent bits (this level, Np positions) seen from the children words of the level below.
+__device__ __forceinline__ uint32_t to_children(uint32_t D, uint64_t Nc) {
+  const int lane = threadIdx.x & 31;
+  const uint64_t Np = Nc >> 1;
+  if (Np >= 32) {
+    const int wp = (int)(Np >> 5);
+    return __shfl_sync(0xffffffffu, D, lane % wp);
+  }
+  const uint32_t d = __shfl_sync(0xffffffffu, D, 0) & low_mask(Np);
+  return lane == 0 ? (d | (d << Np)) : 0u;
+}
+
+__device__ __forceinline__ uint32_t valid_word(uint64_t N) {
+  const uint64_t q0 = (uint64_t)(threadIdx.x & 31) * 32;
+  return q0 < N ? low_mask(N - q0) : 0u;
+}
 
 struct Ctx {
   const TreeParams* p;
@@ -110,53 +226,52 @@ struct Ctx {
   int Lin, gsz;
   uint64_t P0;       // positions at the input height
   bool leaf;         // stage 0
-  Digest* tdig;      // this group's internal digests (P0 entries)
-  unsigned long long* tsrc;   // this group's sources (2 P0 entries: level 0, then internal)
+  Digest* tdig;      // this group's spilled digests (P0 entries)
+  unsigned long long* tsrc;   // this group's sources (2 P0 entries, bit-reversed indices)
 };
 
-// digest of the child at (lv, pos) of the current group
-__device__ __forceinline__ Digest child_digest(const Ctx& c, int lv, uint64_t pos) {
+// digest of the node at (lv, rev index r) of the current group: leaves / inputs from
+// global memory, internal pass-1 nodes from the warp's compact store
+__device__ __forceinline__ Digest child_digest(const Ctx& c, const WarpSmem& ws, int lv, uint32_t r) {
   const TreeParams& p = *c.p;
   if (lv == 0) {
-    if (c.leaf) {
-      const ulonglong2 v = __ldg(reinterpret_cast<const ulonglong2*>(p.prev) + ((c.G << c.gsz) + pos));
-      return Digest{v.x, v.y};
-    }
-    const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(p.st[c.s].in.dig) + ((c.G << c.gsz) + pos));
+    const uint64_t q = rev_n(r, c.gsz);
+    const ulonglong2* base =
+        c.leaf ? reinterpret_cast<const ulonglong2*>(p.prev) : reinterpret_cast<const ulonglong2*>(p.st[c.s].in.dig);
+    const ulonglong2 v = c.leaf ? __ldg(base + ((c.G << c.gsz) + q)) : __ldcg(base + ((c.G << c.gsz) + q));
     return Digest{v.x, v.y};
   }
   if (lv == 1 && c.leaf) {
-    const uint64_t gq = (c.G << (c.gsz - 1)) + pos;
+    const uint64_t gq = (c.G << (c.gsz - 1)) + rev_n(r, c.gsz - 1);
     if (2 * gq >= p.g.m) {
       const ulonglong2 v = __ldg(reinterpret_cast<const ulonglong2*>(p.prev) + (gq + p.g.m / 2));
       return Digest{v.x, v.y};
     }
   }
-  const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(c.tdig) + (lvl_off(c.P0, lv) + pos));
-  return Digest{v.x, v.y};
+  return dig_load(ws, c.tdig, lay_rank(ws, lv, r));
 }
 
-__device__ __forceinline__ unsigned long long child_src(const Ctx& c, int lv, uint64_t pos) {
+__device__ __forceinline__ unsigned long long child_src(const Ctx& c, int lv, uint32_t r) {
   const TreeParams& p = *c.p;
   if (lv == 0) {
-    if (c.leaf) return __ldcg(c.tsrc + pos);
-    return __ldcg(p.st[c.s].in.src + ((c.G << c.gsz) + pos));
+    if (c.leaf) return __ldcg(c.tsrc + r);
+    return __ldcg(p.st[c.s].in.src + ((c.G << c.gsz) + rev_n(r, c.gsz)));
   }
-  return __ldcg(c.tsrc + c.P0 + lvl_off(c.P0, lv) + pos);
+  return __ldcg(c.tsrc + c.P0 + lvl_off(c.P0, lv) + r);
 }
 
-// Leaf labels of a chunk range mapped onto one level's words (stage 0, phase 2): every
-// candidate is resolved against the record (R6: FIRST iff the record's entry is this
-// leaf; otherwise SHIFT with that entry as its source), the rest are FIXED. Sets masks
-// F/S/X (lane word) for positions [0, npos); SHIFT sources go to tsrc[src_base + pos].
+// Leaf labels of a chunk range (stage 0, phase 2): every candidate is resolved against
+// the record (R6: FIRST iff the record's entry is this leaf; otherwise SHIFT with that
+// entry as its source), the rest are FIXED. Returns NATURAL-order masks for positions
+// [0, npos) (word = lane); the SHIFT sources go to tsrc[src_base + rev_n(pos0 + pos)].
 // The leaf classes (first / spatial / temporal) are counted here.
 struct LeafCount {
   uint32_t f, s, t;
 };
 
 __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint64_t chunk0, uint64_t npos,
-                                               uint64_t src_base, uint32_t& F, uint32_t& S, uint32_t& X,
-                                               LeafCount& lc) {
+                                               uint64_t src_base, uint32_t pos0, int nrev, uint32_t& F, uint32_t& S,
+                                               uint32_t& X, LeafCount& lc) {
   const TreeParams& p = *c.p;
   const int lane = threadIdx.x & 31;
   uint32_t valid = 0, cand = 0;
@@ -178,7 +293,7 @@ __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint6
       ++lc.f;
     } else {
       atomicOr(&ws.hitS[w], 1u << b);
-      c.tsrc[src_base + pos] = val;
+      c.tsrc[src_base + rev_n(pos0 + pos, nrev)] = val;
       if ((uint32_t)(val >> 32) == k) ++lc.s; else ++lc.t;
     }
   });
@@ -203,18 +318,19 @@ __device__ __forceinline__ bool insert_new(Slot* tab, uint64_t cap, const Digest
   }
 }
 
-// Emit the region (lv, pos) of the current group (phase 3).
-__device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, uint64_t pos, bool first,
+// Emit the region (lv, rev index r) of the current group (phase 3).
+__device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, uint32_t r, bool first,
                                            unsigned long long src) {
   const TreeParams& p = *c.p;
+  const uint32_t q = rev_n(r, c.gsz - lv);   // natural position
   if (c.leaf) {
-    const uint32_t slot = (uint32_t)(pos << lv);
+    const uint32_t slot = q << lv;
     atomicOr(first ? &ws.stF[slot >> 5] : &ws.stS[slot >> 5], 1u << (slot & 31));
     ws.lvl[slot] = (uint8_t)lv;
     return;
   }
   const int Lc = c.Lin + lv;
-  const uint64_t gpos = (c.G << (c.gsz - lv)) + pos;
+  const uint64_t gpos = (c.G << (c.gsz - lv)) + q;
   const uint32_t node = node_id(p.g, Lc, gpos);
   const uint64_t tile = (gpos << Lc) >> p.g.t0;
   uint32_t bytes = 0;
@@ -236,203 +352,233 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
   const Geo& g = p.g;
   const int lane = threadIdx.x & 31;
   const uint64_t P0 = c.P0;
-  uint32_t F = 0, S = 0, X = 0;    // current level's masks (lane word)
-  uint32_t* lm = c.leaf ? p.lmask + (c.G << 7) : nullptr;   // per tile: F0 S0 F1 S1 (32 words each)
+  const int gsz = c.gsz;
+  uint32_t F = 0, S = 0, X = 0;                      // current level (bit-reversed order)
+  uint32_t leafm1 = 0, lF1 = 0, lS1 = 0, lX1 = 0;   // level-1 leaves of depth h-1 (R3)
+  uint32_t* lm = c.leaf ? p.lmask + c.G * kLmWords : nullptr;
 
   // ---- input level
   if (c.leaf) {
-    const uint64_t base = c.G << c.gsz;
+    const uint64_t base = c.G << gsz;
     const uint64_t npos0 = base < g.m ? (g.m - base < P0 ? g.m - base : P0) : 0;   // real leaves at height 0
+    const uint64_t Np1 = P0 >> 1;
+    const uint64_t pbase1 = c.G << (gsz - 1);
+    const uint64_t first_leaf = gsz >= 1 ? ((g.m / 2 > pbase1) ? g.m / 2 - pbase1 : 0) : Np1;   // local, level 1
+    const bool has_l1 = gsz >= 1 && first_leaf < Np1;
     if (PHASE == 2) {
-      resolve_leaves(c, ws, base, npos0, 0, F, S, X, lc);
+      uint32_t nF, nS, nX;
+      resolve_leaves(c, ws, base, npos0, 0, 0, gsz, nF, nS, nX, lc);
+      to_rev3(ws, gsz, nF, nS, nX, F, S, X);
       lm[lane] = F;
       lm[32 + lane] = S;
+      lm[64 + lane] = X;
+      if (has_l1) {
+        // chunks gq + m/2 for level-1 local positions [first_leaf, Np1)
+        uint32_t tF, tS, tX;
+        resolve_leaves(c, ws, pbase1 + first_leaf + g.m / 2, Np1 - first_leaf, P0 + lvl_off(P0, 1),
+                       (uint32_t)first_leaf, gsz - 1, tF, tS, tX, lc);
+        // natural words relative to first_leaf -> natural words of level 1
+        const uint32_t sh = (uint32_t)(first_leaf & 31);
+        const int wsrc = (int)(first_leaf >> 5);
+        auto realign = [&](uint32_t m) {
+          const int a = lane - wsrc;
+          const uint32_t cur = __shfl_sync(0xffffffffu, m, a < 0 ? 0 : (a & 31));
+          const uint32_t prv = __shfl_sync(0xffffffffu, m, (a - 1) < 0 ? 0 : ((a - 1) & 31));
+          uint32_t r = 0;
+          if (a >= 0) r = cur << sh;
+          if (a >= 1 && sh) r |= prv >> (32 - sh);
+          return r;
+        };
+        const uint32_t v1 = valid_word(Np1);
+        const uint32_t q0 = lane * 32;
+        const uint32_t lmn = (q0 + 32 > first_leaf) ? (v1 & ~low_mask(first_leaf > q0 ? first_leaf - q0 : 0)) : 0u;
+        to_rev3(ws, gsz - 1, realign(tF) & lmn, realign(tS) & lmn, lmn, lF1, lS1, leafm1);
+        lm[96 + lane] = lF1;
+        lm[128 + lane] = lS1;
+        lm[160 + lane] = leafm1;
+      }
     } else {
-      const uint32_t valid = ((uint64_t)lane * 32 < npos0) ? low_mask(npos0 - (uint64_t)lane * 32) : 0u;
       F = __ldcg(lm + lane);
       S = __ldcg(lm + 32 + lane);
-      X = valid & ~(F | S);
+      X = __ldcg(lm + 64 + lane);
+      if (has_l1) {
+        lF1 = __ldcg(lm + 96 + lane);
+        lS1 = __ldcg(lm + 128 + lane);
+        leafm1 = __ldcg(lm + 160 + lane);
+      }
       ws.stF[lane] = 0;
       ws.stS[lane] = 0;
     }
+    lX1 = leafm1 & ~(lF1 | lS1);
   } else {
-    // 32 positions per lane: dirty marks (128 B) and labels (32 B) as vector loads
+    // 32 positions per lane (natural order): dirty marks and labels as vector loads
     const StageParams& sp = p.st[c.s];
-    const uint64_t j0 = (c.G << c.gsz) + (uint64_t)lane * 32;
+    const uint64_t j0 = (c.G << gsz) + (uint64_t)lane * 32;
     const uint8_t* labs = PHASE == 2 ? sp.in.lab2 : sp.in.lab3;
+    uint32_t nF = 0, nS = 0, nX = 0;
     if (P0 >= 32) {
-      uint4 dv[8], lv2[2];
+      if ((uint64_t)lane * 32 < P0) {
+        uint4 dv[8], lv2[2];
 #pragma unroll
-      for (int i = 0; i < 8; ++i) dv[i] = __ldcg(reinterpret_cast<const uint4*>(sp.dirty_in + j0) + i);
+        for (int i = 0; i < 8; ++i) dv[i] = __ldcg(reinterpret_cast<const uint4*>(sp.dirty_in + j0) + i);
 #pragma unroll
-      for (int i = 0; i < 2; ++i) lv2[i] = __ldcg(reinterpret_cast<const uint4*>(labs + j0) + i);
-      const uint32_t* dw = reinterpret_cast<const uint32_t*>(dv);
-      const uint8_t* lb = reinterpret_cast<const uint8_t*>(lv2);
+        for (int i = 0; i < 2; ++i) lv2[i] = __ldcg(reinterpret_cast<const uint4*>(labs + j0) + i);
+        const uint32_t* dw = reinterpret_cast<const uint32_t*>(dv);
+        const uint8_t* lb = reinterpret_cast<const uint8_t*>(lv2);
 #pragma unroll
-      for (int b = 0; b < 32; ++b) {
-        const uint8_t L = (dw[b] == g.epoch) ? lb[b] : (uint8_t)L_FIXED;
-        F |= (uint32_t)(L == L_FIRST) << b;
-        S |= (uint32_t)(L == L_SHIFT) << b;
-        X |= (uint32_t)(L == L_FIXED) << b;
+        for (int b = 0; b < 32; ++b) {
+          const uint8_t L = (dw[b] == g.epoch) ? lb[b] : (uint8_t)L_FIXED;
+          nF |= (uint32_t)(L == L_FIRST) << b;
+          nS |= (uint32_t)(L == L_SHIFT) << b;
+          nX |= (uint32_t)(L == L_FIXED) << b;
+        }
       }
-    } else if (lane == 0) {
-      for (uint32_t b = 0; b < P0; ++b) {
-        const uint8_t L = (__ldcg(sp.dirty_in + j0 + b) == g.epoch) ? __ldcg(labs + j0 + b) : (uint8_t)L_FIXED;
-        F |= (uint32_t)(L == L_FIRST) << b;
-        S |= (uint32_t)(L == L_SHIFT) << b;
-        X |= (uint32_t)(L == L_FIXED) << b;
+    } else {
+      // fewer than 32 positions: lane b loads position b, ballots build lane 0's words
+      const uint64_t jb = (c.G << gsz) + lane;
+      uint8_t L = L_ABSENT;
+      if ((uint64_t)lane < P0) L = (__ldcg(sp.dirty_in + jb) == g.epoch) ? __ldcg(labs + jb) : (uint8_t)L_FIXED;
+      const uint32_t bf = __ballot_sync(0xffffffffu, L == L_FIRST);
+      const uint32_t bs = __ballot_sync(0xffffffffu, L == L_SHIFT);
+      const uint32_t bx = __ballot_sync(0xffffffffu, L == L_FIXED);
+      if (lane == 0) { nF = bf; nS = bs; nX = bx; }
+    }
+    to_rev3(ws, gsz, nF, nS, nX, F, S, X);
+  }
+  __syncwarp();
+  if (p.trace && lane == 0) ws.tp[0] = gtimer();
+
+  // ---- pass 1: digests bottom-up, no record traffic (see file header)
+  ws.W[lane] = 0;
+  __syncwarp();
+  {
+    uint32_t P = PHASE == 2 ? F : S;
+    for (int lv = 1; lv <= gsz; ++lv) {
+      const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
+      uint32_t l, r;
+      lr(P, Nc, l, r);
+      const uint32_t work = l & r & valid_word(Np) & (lv == 1 ? ~leafm1 : 0xFFFFFFFFu);
+      const uint32_t inj = lv == 1 ? (PHASE == 2 ? lF1 : lS1) : 0u;
+      if (!__any_sync(0xffffffffu, work != 0)) {
+        P = inj;
+        continue;
       }
+      if (lv <= 5) {
+        if ((uint64_t)lane * 32 < Np) ws.W[lay_base(lv) + lane] = work;
+      } else if (lane == 0) {
+        ws.W[31] |= work << lay_shift(lv);
+      }
+      __syncwarp();
+      {   // ranks: exclusive prefix of the layout popcounts
+        const uint32_t cnt = __popc(ws.W[lane]);
+        uint32_t incl = cnt;
+#pragma unroll
+        for (int o2 = 1; o2 < 32; o2 <<= 1) {
+          const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o2);
+          if (lane >= o2) incl += v;
+        }
+        ws.WP[lane] = incl - cnt;
+      }
+      __syncwarp();
+      for_each_bit_balanced(ws, work, [&](uint32_t, uint32_t, uint32_t q) {
+        const Digest d = mm::node(child_digest(c, ws, lv - 1, q), child_digest(c, ws, lv - 1, q + (uint32_t)Np));
+        dig_store(ws, c.tdig, lay_rank(ws, lv, q), d);
+      });
+      P = work | inj;
     }
   }
   __syncwarp();
+  if (p.trace && lane == 0) ws.tp[1] = gtimer();
 
-  // ---- levels
-  for (int lv = 1; lv <= c.gsz; ++lv) {
-    const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
-    uint32_t eF, oF, eS, oS, eX, oX;
-    if (Nc > 32) {
-      const int s0 = (2 * lane) & 31, s1 = (2 * lane + 1) & 31;
-      const uint32_t fl = __shfl_sync(0xffffffffu, F, s0), fh = __shfl_sync(0xffffffffu, F, s1);
-      const uint32_t sl = __shfl_sync(0xffffffffu, S, s0), sh = __shfl_sync(0xffffffffu, S, s1);
-      const uint32_t xl = __shfl_sync(0xffffffffu, X, s0), xh = __shfl_sync(0xffffffffu, X, s1);
-      const uint64_t f64 = (uint64_t)fl | ((uint64_t)fh << 32);
-      const uint64_t s64 = (uint64_t)sl | ((uint64_t)sh << 32);
-      const uint64_t x64 = (uint64_t)xl | ((uint64_t)xh << 32);
-      eF = even_bits64(f64); oF = even_bits64(f64 >> 1);
-      eS = even_bits64(s64); oS = even_bits64(s64 >> 1);
-      eX = even_bits64(x64); oX = even_bits64(x64 >> 1);
-    } else {
-      const uint32_t f = __shfl_sync(0xffffffffu, F, 0), s = __shfl_sync(0xffffffffu, S, 0),
-                     x = __shfl_sync(0xffffffffu, X, 0);
-      eF = even_bits64(f); oF = even_bits64(f >> 1);
-      eS = even_bits64(s); oS = even_bits64(s >> 1);
-      eX = even_bits64(x); oX = even_bits64(x >> 1);
-    }
-    const uint32_t valid = ((uint64_t)lane * 32 < Np) ? low_mask(Np - (uint64_t)lane * 32) : 0u;
-    const uint32_t bothF = eF & oF & valid;
-    const uint32_t bothX = eX & oX & valid;
-    const uint32_t bothS = eS & oS & valid;
-    const uint64_t pbase = c.G << (c.gsz - lv);     // global position of this level's first node
-
-    // height-1 leaves of depth h-1 (R3): their labels come from the record, not children
-    uint32_t leafm = 0, lF = 0, lS = 0, lX = 0;
-    if (c.leaf && lv == 1) {
-      const uint64_t first_leaf = (g.m / 2 > pbase) ? g.m / 2 - pbase : 0;   // local position
-      if (first_leaf < Np) {
-        const uint64_t q0 = (uint64_t)lane * 32;
-        if (q0 + 32 > first_leaf && q0 < Np) {
-          const uint64_t lo = first_leaf > q0 ? first_leaf - q0 : 0;
-          leafm = valid & ~low_mask(lo);
-        }
-        if (PHASE == 2) {
-          // resolve chunks gq + m/2 for local positions [first_leaf, Np); sources land at
-          // tsrc[P0 + off(1) + pos]
-          uint32_t tF, tS, tX;
-          resolve_leaves(c, ws, pbase + first_leaf + g.m / 2, Np - first_leaf, c.P0 + lvl_off(c.P0, 1) + first_leaf,
-                         tF, tS, tX, lc);
-          // realign: resolve_leaves numbered positions from first_leaf
-          const uint32_t sh = (uint32_t)(first_leaf & 31);
-          const int wsrc = (int)(first_leaf >> 5);
-          auto realign = [&](uint32_t m) {
-            const int a = lane - wsrc;
-            const uint32_t cur = __shfl_sync(0xffffffffu, m, a < 0 ? 0 : (a & 31));
-            const uint32_t prv = __shfl_sync(0xffffffffu, m, (a - 1) < 0 ? 0 : ((a - 1) & 31));
-            uint32_t r = 0;
-            if (a >= 0) r = cur << sh;
-            if (a >= 1 && sh) r |= prv >> (32 - sh);
-            return r & leafm;
-          };
-          lF = realign(tF);
-          lS = realign(tS);
-          lm[64 + lane] = lF;
-          lm[96 + lane] = lS;
-        } else {
-          lF = __ldcg(lm + 64 + lane);
-          lS = __ldcg(lm + 96 + lane);
-        }
-        lX = leafm & ~(lF | lS);
-      }
-    }
-
-    uint32_t nF, nS, nX, nD;
+  // ---- pass 2: record operations for all pass-1 nodes at once
+  ws.H[lane] = 0;
+  __syncwarp();
+  for_each_bit_balanced(ws, ws.W[lane], [&](uint32_t w, uint32_t b, uint32_t) {
+    int lv;
+    uint32_t r;
+    lay_decode(w, b, lv, r);
+    const Digest d = dig_load(ws, c.tdig, ws.WP[w] + __popc(ws.W[w] & ((1u << b) - 1u)));
     if (PHASE == 2) {
-      // Alg.1 l.24-32: FIRST pairs -> hash, label FIRST, insert (node, chkptID)
-      const uint32_t work = bothF & ~leafm;
-      for_each_bit_balanced(ws, work, [&](uint32_t, uint32_t, uint32_t q) {
-        const Digest d = mm::node(child_digest(c, lv - 1, 2 * (uint64_t)q), child_digest(c, lv - 1, 2 * (uint64_t)q + 1));
-        if (insert_new(p.tab, p.cap, d, pack_entry(g.k, node_id(g, c.Lin + lv, pbase + q)))) ++ins_cnt;
-        else ++coll_cnt;   // R14: a FIRST-FIRST digest already in the record = 128-bit collision
-        reinterpret_cast<ulonglong2*>(c.tdig)[lvl_off(P0, lv) + q] = make_ulonglong2(d.lo, d.hi);
-      });
-      nF = (work) | lF;
-      nS = 0; nX = 0; nD = 0;
-      (void)lS; (void)lX;
+      // Alg.1 l.29: Map[Tree(node)] <- (node, chkptID)
+      const uint64_t gpos = (c.G << (gsz - lv)) + rev_n(r, gsz - lv);
+      if (insert_new(p.tab, p.cap, d, pack_entry(g.k, node_id(g, c.Lin + lv, gpos)))) ++ins_cnt;
+      else ++coll_cnt;   // R14: a FIRST-FIRST digest already in the record = 128-bit collision
     } else {
-      // Alg.1 l.33-46 on non-FIRST nodes
-      const uint32_t work = bothS & ~leafm;
-      ws.hitF[lane] = 0;
-      __syncwarp();
-      for_each_bit_balanced(ws, work, [&](uint32_t w, uint32_t b, uint32_t q) {
-        const Digest d = mm::node(child_digest(c, lv - 1, 2 * (uint64_t)q), child_digest(c, lv - 1, 2 * (uint64_t)q + 1));
-        const unsigned long long v = table_lookup(p.tab, p.cap, d);
-        if (v != kEmpty) {
-          atomicOr(&ws.hitF[w], 1u << b);
-          reinterpret_cast<ulonglong2*>(c.tdig)[lvl_off(P0, lv) + q] = make_ulonglong2(d.lo, d.hi);
-          c.tsrc[P0 + lvl_off(P0, lv) + q] = v;
-        }
-      });
-      const uint32_t hit = ws.hitF[lane];
-      nF = (bothF & ~leafm) | lF;
-      nX = (bothX & ~leafm) | lX;
-      nS = hit | lS;
-      nD = valid & ~leafm & ~bothF & ~bothX & ~hit;
-      // emission of the children of DONE parents: spread parent bits onto child words
-      uint32_t dchild;
-      if (Nc > 32) {
-        const uint32_t dp = __shfl_sync(0xffffffffu, nD, lane >> 1);
-        dchild = spread16((lane & 1) ? (dp >> 16) : dp);
-      } else {
-        const uint32_t dp = __shfl_sync(0xffffffffu, nD, 0);
-        dchild = lane == 0 ? spread16(dp) : 0u;
+      // Alg.1 l.39: Tree(node) in Map ?
+      const unsigned long long v = table_lookup(p.tab, p.cap, d);
+      if (v != kEmpty) {
+        atomicOr(&ws.H[w], 1u << b);
+        c.tsrc[P0 + lvl_off(P0, lv) + r] = v;
       }
-      const uint32_t emF = dchild & F, emS = dchild & S;
-      for (uint32_t m = emF | emS; m; m &= m - 1) {
-        const uint32_t b = __ffs(m) - 1;
-        const uint64_t pos = (uint64_t)lane * 32 + b;
-        const bool isF = (emF >> b) & 1u;
-        emit_region(c, ws, lv - 1, pos, isF, isF ? 0ull : child_src(c, lv - 1, pos));
-      }
-      __syncwarp();
     }
-    F = nF; S = nS; X = nX;
-    (void)nD;
+  });
+  if (p.trace && lane == 0) ws.tp[2] = gtimer();
+
+  if (PHASE == 2) {
+    // the FIRST label chain up to the group root
+    for (int lv = 1; lv <= gsz; ++lv) {
+      const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
+      uint32_t l, r;
+      lr(F, Nc, l, r);
+      F = (l & r & valid_word(Np) & (lv == 1 ? ~leafm1 : 0xFFFFFFFFu)) | (lv == 1 ? lF1 : 0u);
+    }
+  } else {
+    // ---- pass 3: Alg.1 l.33-46 with the lookup results; emission of "roots" (R8)
+    for (int lv = 1; lv <= gsz; ++lv) {
+      const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
+      uint32_t lF, rF, lS, rS, lX, rX;
+      lr(F, Nc, lF, rF);
+      lr(S, Nc, lS, rS);
+      lr(X, Nc, lX, rX);
+      const uint32_t leafm = lv == 1 ? leafm1 : 0u;
+      const uint32_t valid = valid_word(Np) & ~leafm;
+      uint32_t hw;
+      if (lv <= 5) hw = ((uint64_t)lane * 32 < Np) ? ws.H[lay_base(lv) + lane] : 0u;
+      else hw = lane == 0 ? (ws.H[31] >> lay_shift(lv)) & low_mask(Np) : 0u;
+      const uint32_t bothF = lF & rF & valid;
+      const uint32_t bothX = lX & rX & valid;
+      const uint32_t hitS = lS & rS & valid & hw;        // both children SHIFT and found
+      const uint32_t nD = valid & ~bothF & ~bothX & ~hitS;
+      // the FIRST/SHIFT children of DONE parents are regions
+      const uint32_t dchild = to_children(nD, Nc);
+      const uint32_t emF = dchild & F, emS = dchild & S;
+      if (__any_sync(0xffffffffu, (emF | emS) != 0)) {
+        for (uint32_t m = emF | emS; m; m &= m - 1) {
+          const uint32_t b = __ffs(m) - 1;
+          const uint32_t rr = (uint32_t)lane * 32 + b;
+          const bool isF = (emF >> b) & 1u;
+          emit_region(c, ws, lv - 1, rr, isF, (isF || c.leaf) ? 0ull : child_src(c, lv - 1, rr));
+        }
+        __syncwarp();
+      }
+      F = bothF | (lv == 1 ? lF1 : 0u);
+      X = bothX | (lv == 1 ? lX1 : 0u);
+      S = hitS | (lv == 1 ? lS1 : 0u);
+    }
   }
 
-  // ---- group root (single position at level gsz, lane 0 bit 0)
+  // ---- group root (single position at level gsz: lane 0 bit 0)
   const uint32_t rF = __shfl_sync(0xffffffffu, F, 0) & 1u;
   const uint32_t rS = __shfl_sync(0xffffffffu, S, 0) & 1u;
   const uint32_t rX = __shfl_sync(0xffffffffu, X, 0) & 1u;
   const bool last = (c.s == p.S - 1);
   if (last) {
     if (PHASE == 3 && lane == 0 && (rF | rS))
-      emit_region(c, ws, c.gsz, 0, rF != 0, rS ? child_src(c, c.gsz, 0) : 0ull);   // R10
+      emit_region(c, ws, gsz, 0, rF != 0, rS ? child_src(c, gsz, 0) : 0ull);   // R10
   } else if (lane == 0) {
     const StageParams& nx = p.st[c.s + 1];
-    uint8_t L;
     if (PHASE == 2) {
-      L = rF ? L_FIRST : L_FIXED;
-      nx.in.lab2[c.G] = L;
+      nx.in.lab2[c.G] = rF ? L_FIRST : L_FIXED;
       if (rF) {
-        const Digest d = child_digest(c, c.gsz, 0);
+        const Digest d = child_digest(c, ws, gsz, 0);
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
       }
     } else {
-      L = rF ? L_FIRST : (rS ? L_SHIFT : (rX ? L_FIXED : L_DONE));
-      nx.in.lab3[c.G] = L;
+      nx.in.lab3[c.G] = rF ? L_FIRST : (rS ? L_SHIFT : (rX ? L_FIXED : L_DONE));
       if (rS) {
-        const Digest d = child_digest(c, c.gsz, 0);
+        const Digest d = child_digest(c, ws, gsz, 0);
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
-        nx.in.src[c.G] = child_src(c, c.gsz, 0);
+        nx.in.src[c.G] = child_src(c, gsz, 0);
       }
     }
   }
@@ -452,22 +598,38 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     uint32_t bytes = 0;
     uint4* out = p.scratch + (c.G << g.t0);
     for (uint32_t m = wF; m; m &= m - 1) {
-      const uint32_t b = __ffs(m) - 1;
-      const uint32_t slot = lane * 32 + b;
+      const uint32_t slot = lane * 32 + (__ffs(m) - 1);
       const int lv = ws.lvl[slot];
-      const uint64_t gpos = (c.G << (c.gsz - lv)) + (slot >> lv);
+      const uint64_t gpos = (c.G << (gsz - lv)) + (slot >> lv);
       uint64_t lo, hi;
       chunk_range(g, lv, gpos, lo, hi);
       bytes += (uint32_t)range_bytes(g, lo, hi);
       out[rf++] = make_uint4(node_id(g, lv, gpos), 0u, 0u, L_FIRST);
     }
-    for (uint32_t m = wS; m; m &= m - 1) {
-      const uint32_t b = __ffs(m) - 1;
-      const uint32_t slot = lane * 32 + b;
-      const int lv = ws.lvl[slot];
-      const uint64_t gpos = (c.G << (c.gsz - lv)) + (slot >> lv);
-      const unsigned long long src = child_src(c, lv, slot >> lv);
-      out[rs++] = make_uint4(node_id(g, lv, gpos), (uint32_t)(src & 0xffffffffu), (uint32_t)(src >> 32), L_SHIFT);
+    for (uint32_t m = wS; m;) {   // batches of 4: issue the source loads first
+      uint32_t slots[4];
+      unsigned long long src[4];
+      int nb = 0;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        if (m) {
+          const uint32_t b = __ffs(m) - 1;
+          m &= m - 1;
+          slots[u] = lane * 32 + b;
+          const int lv = ws.lvl[slots[u]];
+          src[u] = child_src(c, lv, rev_n(slots[u] >> lv, gsz - lv));
+          nb = u + 1;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        if (u < nb) {
+          const int lv = ws.lvl[slots[u]];
+          const uint64_t gpos = (c.G << (gsz - lv)) + (slots[u] >> lv);
+          out[rs++] = make_uint4(node_id(g, lv, gpos), (uint32_t)(src[u] & 0xffffffffu), (uint32_t)(src[u] >> 32),
+                                 L_SHIFT);
+        }
+      }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
@@ -481,13 +643,16 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
 // ================================================================= kernel
 template <int PHASE>
 __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constant__ TreeParams p) {
-  __shared__ WarpSmem sm[kWarps];
+  extern __shared__ __align__(16) uint8_t tree_smem[];
+  WarpSmem* sm = reinterpret_cast<WarpSmem*>(tree_smem);
   __shared__ unsigned long long s_cnt[4];
   LeafCount lc{0, 0, 0};
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   WarpSmem& ws = sm[wid];
+  pdl_launch_dependents();
   if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
   __syncthreads();
+  pdl_wait();
   unsigned long long ins = 0, coll = 0;
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   unsigned* next = &p.tot->tree_next[PHASE - 2];
@@ -506,7 +671,13 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
     c.leaf = true;
     c.tdig = p.st[0].tdig + (c.G << c.gsz);
     c.tsrc = p.st[0].tsrc + ((c.G << c.gsz) << 1);
+    unsigned long long t0 = p.trace ? gtimer() : 0;
     process_group<PHASE>(c, ws, ins, coll, lc);
+    if (p.trace && lane == 0) {
+      const uint32_t i = atomicAdd(p.trace_n, 2u);
+      p.trace[i] = make_ulonglong4(t0, gtimer(), (unsigned long long)c.G, PHASE);
+      p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 10 + PHASE);
+    }
     // climb: the warp finishing the last dirty child of a group processes that group
     while (c.s < p.S - 1) {
       const StageParams& up = p.st[c.s + 1];
@@ -526,7 +697,12 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
       c.leaf = false;
       c.tdig = up.tdig + (P << c.gsz);
       c.tsrc = up.tsrc + ((P << c.gsz) << 1);
+      t0 = p.trace ? gtimer() : 0;
       process_group<PHASE>(c, ws, ins, coll, lc);
+      if (p.trace && lane == 0) {
+        const uint32_t i = atomicAdd(p.trace_n, 1u);
+        p.trace[i] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
+      }
     }
   }
   if (ins) atomicAdd(&s_cnt[3], ins);
@@ -549,9 +725,18 @@ cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_
   uint64_t grid = (uint64_t)num_sms * 8;
   const uint64_t need = (p.n_tiles + kWarps - 1) / kWarps;
   if (grid > need) grid = need ? need : 1;
-  if (phase == 2) tree_kernel<2><<<(unsigned)grid, kTreeThreads, 0, st>>>(p);
-  else tree_kernel<3><<<(unsigned)grid, kTreeThreads, 0, st>>>(p);
-  return cudaGetLastError();
+  const size_t smem = kWarps * sizeof(WarpSmem);
+  if (phase == 2) return launch_pdl(tree_kernel<2>, (unsigned)grid, kTreeThreads, smem, st, p);
+  return launch_pdl(tree_kernel<3>, (unsigned)grid, kTreeThreads, smem, st, p);
 }
+
+cudaError_t tree_setup_attributes() {
+  const int smem = (int)(kWarps * sizeof(WarpSmem));
+  cudaError_t e = cudaFuncSetAttribute(tree_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tree_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  return e;
+}
+
+size_t tree_lmask_words() { return kLmWords; }
 
 }  // namespace ckpt

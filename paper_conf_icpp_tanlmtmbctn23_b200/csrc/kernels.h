@@ -96,6 +96,9 @@ struct TreeParams {
   uint4* tilecnt;              // per tile: {nF, nS, data_bytes, epoch}
   uint32_t* lmask;             // per tile: resolved leaf masks (phase 2 -> phase 3), 128 words
   Totals* tot;
+  int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
+  ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
+  uint32_t* trace_n;
   StageParams st[kMaxStages];
 };
 
@@ -114,7 +117,27 @@ struct CompactParams {
   const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
 };
 
+// Launch with programmatic stream serialization (PDL): the kernel may be scheduled while
+// its predecessor drains; it must call pdl_wait() before touching the predecessor's output.
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
 // ---- launchers (return cudaGetLastError())
+cudaError_t leaf_setup_attributes();
+cudaError_t tree_setup_attributes();
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
 cudaError_t launch_insert(const InsertParams& p, cudaStream_t st);
