@@ -115,12 +115,18 @@ def dist_setup(n_gpus):
     return ws, rank, local
 
 
+def _coll_device():
+    import torch.distributed as dist
+    return "cpu" if dist.get_backend() == "gloo" else "cuda"
+
+
 def max_over_ranks(x, ws):
+    """Max over ranks (the box time of P:232: slowest process)."""
     if ws == 1:
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    t = torch.tensor([x], dtype=torch.float64, device=_coll_device())
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -130,7 +136,7 @@ def sum_over_ranks(x, ws):
         return x
     import torch
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    t = torch.tensor([x], dtype=torch.float64, device=_coll_device())
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
 
@@ -148,7 +154,7 @@ def allgather_sizes(records, ws):
     if ws == 1:
         return [records]
     import torch.distributed as dist
-    t = torch.tensor(records, dtype=torch.int64, device="cuda")
+    t = torch.tensor(records, dtype=torch.int64, device=_coll_device())
     out = [torch.empty_like(t) for _ in range(ws)]
     dist.all_gather(out, t)
     return [o.cpu().tolist() for o in out]
