@@ -30,13 +30,14 @@ constexpr uint64_t c2 = 0x4cf5ad432745937full;
 template <int R>
 __device__ __forceinline__ uint64_t rotl(uint64_t x) {
   const uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+  constexpr unsigned sh = R < 32 ? (unsigned)R : (unsigned)(R - 32);
   uint32_t nlo, nhi;
   if (R < 32) {
-    nhi = __funnelshift_l(lo, hi, R);
-    nlo = __funnelshift_l(hi, lo, R);
+    nhi = __funnelshift_l(lo, hi, sh);
+    nlo = __funnelshift_l(hi, lo, sh);
   } else {
-    nhi = __funnelshift_l(hi, lo, R - 32);
-    nlo = __funnelshift_l(lo, hi, R - 32);
+    nhi = __funnelshift_l(hi, lo, sh);
+    nlo = __funnelshift_l(lo, hi, sh);
   }
   return ((uint64_t)nhi << 32) | nlo;
 }
@@ -192,10 +193,23 @@ __device__ __forceinline__ uint64_t table_find_or_claim(Slot* tab, uint64_t cap,
   }
 }
 
+// Find-or-claim by CAS first (no plain read): one round trip when the key is new, which
+// is the common case after checkpoint 0; hot repeated keys should use the read-first form.
+__device__ __forceinline__ uint64_t table_claim_cas(Slot* tab, uint64_t cap, const Digest& d, bool* claimed) {
+  uint64_t s = slot_home(d.lo, cap);
+  for (;;) {
+    unsigned long long olo, ohi;
+    cas128(tab + s, kEmpty, kEmpty, d.lo, d.hi, olo, ohi);
+    if (olo == kEmpty && ohi == kEmpty) { *claimed = true; return s; }
+    if (olo == d.lo && ohi == d.hi) { *claimed = false; return s; }
+    if (++s == cap) s = 0;
+  }
+}
+
 // Insert-or-min: Map.insert(digest, entry) of Alg.1 l.7 with the R6 tie-break.
 __device__ __forceinline__ uint64_t table_insert_min(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed,
-                                                    bool* claimed) {
-  uint64_t s = table_find_or_claim(tab, cap, d, claimed);
+                                                    bool* claimed, bool cas_first = false) {
+  uint64_t s = cas_first ? table_claim_cas(tab, cap, d, claimed) : table_find_or_claim(tab, cap, d, claimed);
   Slot* p = tab + s;
   if (*claimed || ld_val_relaxed(p) > packed) atomicMin(&p->val, packed);
   return s;

@@ -56,18 +56,20 @@ struct ckpt_ctx {
   uint64_t nwords = 0;
   uint32_t* slot_of = nullptr;
   uint32_t* dirty[kMaxStages] = {};
-  uint32_t* wl[kMaxStages] = {};
   LevelIO lvl[kMaxStages] = {};
   Digest* tdig[kMaxStages] = {};
   unsigned long long* tsrc[kMaxStages] = {};
-  uint32_t* cnt[kMaxStages] = {};
-  uint32_t* done2[kMaxStages] = {};
-  uint32_t* done3[kMaxStages] = {};
+  uint32_t* arr2[kMaxStages] = {};
+  uint32_t* arr3[kMaxStages] = {};
+  uint32_t* dcnt[kMaxStages] = {};
+  uint32_t* wl0 = nullptr;
+  uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
   uint8_t* ctr = nullptr;        // Totals + per-stage counters, zeroed by one memset per call
   size_t ctr_bytes = 0;
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
+  uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b
   uint4* toff = nullptr;
   unsigned long long* blocksum = nullptr;
   ulonglong2* big = nullptr;
@@ -158,7 +160,6 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->slot_of, n);
   for (int s = 0; s < h->S; ++s) {
     AL(h->dirty[s], h->ngroups[s]);
-    AL(h->wl[s], h->ngroups[s]);
     if (cudaMemset(h->dirty[s], 0, h->ngroups[s] * 4) != cudaSuccess) return CKPT_ECUDA;
     if (s >= 1) {
       const uint64_t P = 1ull << (h->h - h->Lin[s]);
@@ -174,6 +175,9 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   // per-call counters: Totals, then cnt/done2/done3 of every stage s >= 1
   {
     size_t bytes = (sizeof(Totals) + 255) & ~size_t(255);
+    const size_t dbits_off = bytes;
+    bytes += ((n_tiles + 31) / 32) * sizeof(uint32_t);
+    bytes = (bytes + 255) & ~size_t(255);
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
@@ -182,15 +186,18 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     AL(h->ctr, bytes);
     h->ctr_bytes = bytes;
     h->tot = reinterpret_cast<Totals*>(h->ctr);
+    h->dbits = reinterpret_cast<uint32_t*>(h->ctr + dbits_off);
     for (int s = 1; s < h->S; ++s) {
-      h->cnt[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
-      h->done2[s] = h->cnt[s] + h->ngroups[s];
-      h->done3[s] = h->done2[s] + h->ngroups[s];
+      h->arr2[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
+      h->arr3[s] = h->arr2[s] + h->ngroups[s];
+      h->dcnt[s] = h->arr3[s] + h->ngroups[s];
     }
   }
   AL(h->scratch, n_tiles << h->t0);
   AL(h->tilecnt, n_tiles);
+  AL(h->wl0, n_tiles);
   AL(h->lmask, n_tiles * 192);   // k_tree.cu kLmWords
+  AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
   AL(h->toff, n_tiles);
   AL(h->blocksum, 3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3);
   AL(h->big, B / (1 << 20) + 2);
@@ -198,7 +205,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
   if (h->trace_path) {
-    if (dalloc(h, &h->trace, 24 * n_tiles + 64) != cudaSuccess || dalloc(h, &h->trace_n, 4) != cudaSuccess)
+    if (dalloc(h, &h->trace, 24 * n_tiles + n / 16 + 64) != cudaSuccess || dalloc(h, &h->trace_n, 4) != cudaSuccess)
       return CKPT_ENOMEM;
   }
   bool reserved = false;
@@ -223,7 +230,8 @@ Geo make_geo(const ckpt_ctx* h, uint32_t k) {
 }
 
 int ensure_table(ckpt_ctx* h, cudaStream_t st) {
-  const uint64_t need = h->live + 2 * h->n - 1;   // worst case: every node inserted
+  uint64_t need = h->live + 2 * h->n - 1;   // worst case: every node inserted
+  if (h->dbg & 256) need = h->live + h->n / 2;   // diagnostics only: undersized table experiment
   if (h->cap && (double)need <= kMaxLoad * (double)h->cap) return CKPT_OK;
   uint64_t new_cap = (uint64_t)((double)need / kGrowLoad) + 1;
   if (new_cap < 4096) new_cap = 4096;
@@ -407,6 +415,23 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   const Geo g = make_geo(h, k);
   const uint8_t* buf = static_cast<const uint8_t*>(dev_ptr);
 
+  // ---- record-insert state (K1's insert warp and K1b)
+  InsertParams ip;
+  std::memset(&ip, 0, sizeof(ip));
+  ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
+  ip.tab = h->tab; ip.cap = h->cap; ip.slot_of = h->slot_of;
+  ip.tot = h->tot;
+  ip.defer = h->defer;
+  ip.dbits = h->dbits;
+  ip.n_tiles = h->ngroups[0];
+  ip.wl0 = h->wl0;
+  ip.S = h->S;
+  for (int s = 0; s < kMaxStages; ++s) {
+    ip.gsz[s] = h->gsz[s];
+    ip.dcnt[s] = h->dcnt[s];
+  }
+  ip.trace = h->trace; ip.trace_n = h->trace_n;
+
   // ---- leaf pass configuration
   LeafParams lp;
   std::memset(&lp, 0, sizeof(lp));
@@ -414,6 +439,10 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   lp.buf = buf;
   lp.prev = h->prev;
   lp.cand = h->cand;
+  lp.ins = ip;
+  // K1's insert warp overlaps the inserts with the stream but lengthens K1 by about as
+  // much as it saves (measured); it stays available (CKPT_DBG bit 128) and off by default.
+  lp.insert_warp = (k > 0 && (h->dbg & 128)) ? 1 : 0;
   const uint64_t n_full = h->B / h->C;
   if (h->C % 128 == 0) {
     lp.mode3d = 1;
@@ -439,23 +468,14 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   const auto t_pre = clk::now();
   CK(cudaMemsetAsync(h->ctr, 0, h->ctr_bytes, st));
+  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
   CK(launch_leaf_tail(lp, st));
   CK(launch_leaf(&tmap, lp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[1], st));
   // K1b: record insert + tie-break (l.6-19), dirty tiles
-  InsertParams ip;
-  ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
-  ip.tab = h->tab; ip.cap = h->cap; ip.slot_of = h->slot_of;
-  ip.wl0 = h->wl[0]; ip.tot = h->tot;
-  ip.S = h->S;
-  for (int s = 0; s < kMaxStages; ++s) {
-    ip.dirty[s] = h->dirty[s];
-    ip.cnt[s] = h->cnt[s];
-    ip.gsz[s] = h->gsz[s];
-  }
-  CK(launch_insert(ip, st));
+  CK(launch_insert(ip, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[2], st));
 
   // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11
@@ -464,13 +484,13 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.g = g;
   tp.S = h->S;
   tp.n_tiles = h->ngroups[0];
-  tp.wl0 = h->wl[0];
+  tp.wl0 = h->wl0;
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
   tp.trace = h->trace; tp.trace_n = h->trace_n;
   tp.dbg = h->dbg;
-  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
+
   for (int s = 0; s < h->S; ++s) {
     StageParams& sp = tp.st[s];
     sp.Lin = h->Lin[s];
@@ -479,9 +499,10 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.in = s >= 1 ? h->lvl[s] : LevelIO{};
     sp.tdig = h->tdig[s];
     sp.tsrc = h->tsrc[s];
-    sp.cnt = h->cnt[s];
-    sp.done2 = h->done2[s];
-    sp.done3 = h->done3[s];
+    sp.dirty = h->dirty[s];
+    sp.arr2 = h->arr2[s];
+    sp.arr3 = h->arr3[s];
+    sp.dcnt = h->dcnt[s];
   }
   CK(launch_tree(tp, 2, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[3], st));
@@ -493,7 +514,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.g = g;
   cp.n_tiles = h->ngroups[0];
   cp.tilecnt = h->tilecnt; cp.scratch = h->scratch; cp.blocksum = h->blocksum;
-  cp.toff = h->toff; cp.wl0 = h->wl[0]; cp.tot = h->tot;
+  cp.toff = h->toff; cp.wl0 = h->wl0; cp.tot = h->tot;
   cp.big = h->big; cp.big_len = h->big_len;
   cp.out = out; cp.buf = buf;
   CK(launch_compact(cp, h->num_sms, st));

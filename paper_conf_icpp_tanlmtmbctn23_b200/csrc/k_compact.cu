@@ -131,7 +131,7 @@ __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
   }
 }
 
-// KG: one WARP per dirty tile (work-stealing cursor). Writes the tile's metadata entries
+// KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata entries
 // and copies its FIRST bytes: the tile's FIRST regions are taken 32 at a time (lane i ->
 // region i), a warp scan gives their data offsets, and the batch's bytes are copied as
 // one lane-strided stream of 16-byte units (coalesced; the region of a unit is found by
@@ -153,18 +153,15 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
   const Geo& g = p.g;
   pdl_launch_dependents();
   pdl_wait();
-  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   const unsigned long long nF_tot = p.tot->nF;
   uint8_t* const ent_f = p.out + 64;
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
   uint8_t* const dat = p.out + p.tot->meta_bytes;
 
-  for (;;) {
-    uint32_t w = 0;
-    if (lane == 0) w = atomicAdd(&p.tot->gather_next, 1u);
-    w = __shfl_sync(0xffffffffu, w, 0);
-    if (w >= count) break;
-    const uint32_t T = p.wl0[w];
+  const uint64_t nwarps = (uint64_t)gridDim.x * kGW;
+  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
+  for (uint64_t w = (uint64_t)blockIdx.x * kGW + wid; w < count; w += nwarps) {
+    const uint64_t T = __ldcg(p.wl0 + w);
     const uint4 cnt = p.tilecnt[T];
     if (cnt.w != g.epoch) continue;
     const uint32_t nF = cnt.x, nS = cnt.y;

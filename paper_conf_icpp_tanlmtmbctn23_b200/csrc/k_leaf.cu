@@ -13,9 +13,8 @@
 //     chunk hashed at its true length, R4) with direct loads.
 // K1b (insert_kernel): Map.insert(digest, (leaf, chkptID)) for every candidate
 //     (Alg.1 l.6-19) with the R6 tie-break (atomicMin over ckpt<<32|node), one warp per
-//     32 candidate-mask words, warp-level de-duplication of equal digests (__match_any)
-//     so a hot key (e.g. all-zero chunks) costs one atomic per warp; marks stage-0
-//     tiles dirty and appends them to the phase-2/3 worklist.
+//     round of 32 candidates of a 256-chunk tile, warp-level de-duplication of equal
+//     digests (__match_any) so a hot key (e.g. all-zero chunks) costs one atomic per warp.
 #include "kernels.h"
 #include "tma.cuh"
 
@@ -27,9 +26,105 @@ __device__ __forceinline__ bool leaf_is_candidate(const Geo& g, const Digest& d,
   return !(g.k > 0 && d == prevd);
 }
 
+// ------------------------------------------------------------------ record insert
+// Map.insert(digest, (leaf, chkptID)) for the candidates of one 256-chunk leaf tile
+// (Alg.1 l.6-19), by one warp: lane i < 8 holds candidate word i. The candidates are
+// spread evenly over the lanes (prefix over popcounts, __fns), identical digests within a
+// round are collapsed (__match_any) so a hot key costs one record operation per warp, the
+// R6 tie-break is atomicMin over (ckpt << 32 | node).
+__device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile, uint32_t word, uint32_t* s_word,
+                                            uint32_t* s_excl, unsigned long long& ncand, int only_round = -1) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t cnt = __popc(word);
+  uint32_t incl = cnt;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  if (total == 0) return;
+  s_word[lane] = word;
+  s_excl[lane] = incl - cnt;
+  __syncwarp();
+  const uint64_t c0 = (uint64_t)tile * 256;
+  const uint64_t pol = policy_evict_last();
+  const uint32_t b_begin = only_round < 0 ? 0u : 32u * (uint32_t)only_round;
+  const uint32_t b_end = only_round < 0 ? total : (b_begin + 32 < total ? b_begin + 32 : total);
+  for (uint32_t base = b_begin; base < b_end; base += 32) {
+    const uint32_t j = base + lane;
+    const bool has = j < b_end;
+    const unsigned active = __ballot_sync(0xffffffffu, has);
+    if (has) {
+      int lo = 0;   // source word: last w < 8 with excl[w] <= j
+#pragma unroll
+      for (int step = 4; step > 0; step >>= 1)
+        if (lo + step < 8 && s_excl[lo + step] <= j) lo += step;
+      const uint32_t b = __fns(s_word[lo], 0, (int)(j - s_excl[lo]) + 1);
+      const uint64_t c = c0 + (uint64_t)lo * 32 + b;
+      const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(p.prev) + c);
+      const Digest d{v.x, v.y};
+      const uint32_t node = node_of_chunk(p.g, c);
+      const unsigned m1 = __match_any_sync(active, d.lo);
+      const unsigned m2 = __match_any_sync(active, d.hi);
+      const unsigned grp = m1 & m2;
+      const int leader = __ffs(grp) - 1;
+      uint32_t minnode = node;   // minimum node id of the group (every active lane shuffles)
+      for (unsigned a = active; a; a &= a - 1) {
+        const int sl = __ffs(a) - 1;
+        const uint32_t vv = __shfl_sync(active, node, sl);
+        if ((grp >> sl) & 1u) minnode = vv < minnode ? vv : minnode;
+      }
+      uint32_t slot = 0;
+      if (lane == leader) {
+        bool claimed;
+        // checkpoint 0 is full of hot repeated keys (read first); later ones mostly insert new keys (CAS first)
+        slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed, p.g.k > 0);
+      }
+      slot = __shfl_sync(active, slot, leader);
+      st_evict_last_u32(p.slot_of + c, slot, pol);
+    }
+  }
+  ncand += b_end - b_begin;
+  __syncwarp();
+}
+
+// Mark the stage-0 tree tile(s) holding 256-chunk leaf tile `tile` dirty (fire-and-forget;
+// a tree tile marked without candidates is processed as all-FIXED, which is harmless).
+__device__ __forceinline__ void mark_tree_dirty(const InsertParams& p, uint32_t tile) {
+  const uint64_t c0 = (uint64_t)tile * 256;
+  uint64_t c1 = c0 + 255;
+  if (c1 >= p.g.n) c1 = p.g.n - 1;
+  const uint64_t t0 = vpos_of_chunk(p.g, c0) >> p.g.t0, t1 = vpos_of_chunk(p.g, c1) >> p.g.t0;
+  for (uint64_t t = t0; t <= t1; ++t) atomicOr(p.dbits + (t >> 5), 1u << (t & 31));
+}
+
+// Defer a tile's inserts to K1b as one entry (tile << 3 | round) per 32 candidates, so
+// the rounds of a dense tile run on different warps.
+__device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile, uint32_t ncand_tile) {
+  const uint32_t rounds = (ncand_tile + 31) / 32;
+  const uint32_t i = atomicAdd(&p.tot->defer_count, rounds);
+  for (uint32_t r = 0; r < rounds; ++r) p.defer[i + r] = (tile << 3) | r;
+}
+
 // ------------------------------------------------------------------ K1
+// 8 hashing warps + 1 insert warp. A finished tile's 8 candidate words go through a small
+// shared-memory ring to the insert warp, which runs the record inserts while the hashing
+// warps keep streaming; when the ring is full (or at checkpoint 0, when every chunk is a
+// candidate) the tile is deferred to K1b instead, so the stream never waits on inserts.
+constexpr int kRing = 16;
+constexpr int kK1Threads = kLeafThreads + 32;
+
+struct K1Ring {
+  uint32_t words[kRing][8];
+  uint32_t tile[kRing];
+  uint32_t stage_words[2][8];
+  uint32_t s_word[32], s_excl[32];
+  volatile uint32_t head, tail, done;
+};
+
 template <int MODE3D>
-__global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
+__global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
   const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -38,6 +133,7 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   const uint32_t stage_bytes = p.stage_bytes;
   Digest* const prevbuf = reinterpret_cast<Digest*>(data + nst * stage_bytes);   // nst * 256 digests
   uint64_t* const bars = reinterpret_cast<uint64_t*>(prevbuf + nst * kLeafThreads);
+  K1Ring& ring = *reinterpret_cast<K1Ring*>(bars + 8);
 
   const int tid = threadIdx.x;
   const uint32_t n_tiles = (uint32_t)(p.n_main / kLeafThreads);
@@ -46,15 +142,43 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   const uint32_t total = my_tiles * (uint32_t)segs;
   const bool use_prev = p.g.k > 0;
 
-  pdl_launch_dependents();
   if (tid == 0) {
     prefetch_tmap(&tmap);
     for (int s = 0; s < nst; ++s) mbar_init(&bars[s], 1);
     fence_mbar_init();
+    ring.head = 0;
+    ring.tail = 0;
+    ring.done = 0;
   }
   __syncthreads();
 
-  // producer state (thread 0): next step to issue, as (stage, tile, seg) counters
+  if (tid >= kLeafThreads) {
+    // ---------------- insert warp
+    const int lane = tid & 31;
+    unsigned long long ncand = 0;
+    uint32_t head = 0;
+    for (;;) {
+      const uint32_t t = ring.tail;
+      if (head == t) {
+        if (ring.done && head == ring.tail) break;
+        __nanosleep(128);
+        continue;
+      }
+      __threadfence_block();
+      const uint32_t slot = head % kRing;
+      const uint32_t tile = ring.tile[slot];
+      const uint32_t word = lane < 8 ? ring.words[slot][lane] : 0u;
+      __syncwarp();
+      insert_tile(p.ins, tile, word, ring.s_word, ring.s_excl, ncand);
+      ++head;
+      __syncwarp();
+      if (lane == 0) ring.head = head;
+    }
+    if (lane == 0 && ncand) atomicAdd(&p.ins.tot->n_cand, ncand);
+    return;
+  }
+
+  // ---------------- hashing warps (named barrier 1 over 256 threads)
   int is_st = 0, is_seg = 0;
   uint32_t is_tile = blockIdx.x, issued = 0;
   const uint64_t pol_stream = policy_evict_first();
@@ -82,7 +206,7 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
   const uint32_t ubase = (uint32_t)tid * (uint32_t)units;
   uint64_t h1 = 0, h2 = 0;
   int st = 0, seg = 0;
-  uint32_t phase = 0, tile = blockIdx.x;
+  uint32_t phase = 0, tile = blockIdx.x, ntile_done = 0;
   for (uint32_t step = 0; step < total; ++step) {
     mbar_wait(&bars[st], phase);
     if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
@@ -95,24 +219,55 @@ __global__ void __launch_bounds__(kLeafThreads, 2) leaf_hash_kernel(const __grid
       const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + off);
       mm::block(h1, h2, v.x, v.y);
     }
-    if (seg == segs - 1) {
+    const bool tile_end = (seg == segs - 1);
+    if (tile_end) {
       const Digest d = mm::finish(h1, h2, p.g.C);
       const uint64_t c = (uint64_t)tile * kLeafThreads + tid;
       Digest pd{0, 0};
       if (use_prev) pd = prevbuf[st * kLeafThreads + tid];
       const bool cand = leaf_is_candidate(p.g, d, pd);
       const unsigned mask = __ballot_sync(0xffffffffu, cand);
-      if ((tid & 31) == 0) st_evict_last_u32(p.cand + (c >> 5), mask, pol_keep);
+      if ((tid & 31) == 0) {
+        st_evict_last_u32(p.cand + (c >> 5), mask, pol_keep);
+        ring.stage_words[ntile_done & 1][tid >> 5] = mask;
+      }
       if (cand) st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
     }
-    __syncthreads();   // every thread is done with stage st
-    if (tid == 0 && issued < total) issue_next();
+    asm volatile("bar.sync 1, %0;" ::"n"(kLeafThreads) : "memory");   // every hashing thread is done with stage st
+    if (tid == 0) {
+      if (tile_end) {
+        // hand the tile's candidate words to the insert warp, or defer them to K1b
+        uint32_t w[8], any = 0, pc = 0;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) { w[i] = ring.stage_words[ntile_done & 1][i]; any |= w[i]; pc += __popc(w[i]); }
+        if (any) {
+          mark_tree_dirty(p.ins, tile);
+          const uint32_t t = ring.tail;
+          if (p.insert_warp && t - ring.head < (uint32_t)kRing) {
+#pragma unroll
+            for (int i = 0; i < 8; ++i) ring.words[t % kRing][i] = w[i];
+            ring.tile[t % kRing] = tile;
+            __threadfence_block();
+            ring.tail = t + 1;
+          } else {
+            defer_tile(p.ins, tile, pc);
+          }
+        }
+      }
+      if (issued < total) issue_next();
+    }
+    if (tile_end) ++ntile_done;
     if (++st == nst) { st = 0; phase ^= 1u; }
     if (++seg == segs) { seg = 0; tile += gridDim.x; }
+  }
+  if (tid == 0) {
+    __threadfence_block();
+    ring.done = 1;
   }
 }
 
 // ------------------------------------------------------------------ K1t
+// The ragged tail (direct loads): one block = one 256-chunk tile; its inserts are deferred.
 __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
   const uint64_t c = p.tail_begin + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const bool valid = c < p.g.n;
@@ -150,96 +305,107 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
   const unsigned mask = __ballot_sync(0xffffffffu, cand);
   if ((threadIdx.x & 31) == 0 && c < p.g.n) p.cand[c >> 5] = mask;
   if (cand) reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
+  const int pc = __syncthreads_count(cand);
+  if (pc && threadIdx.x == 0) {
+    const uint32_t tile = (uint32_t)((p.tail_begin >> 8) + blockIdx.x);
+    mark_tree_dirty(p.ins, tile);
+    defer_tile(p.ins, tile, (uint32_t)pc);
+  }
 }
 
 // ------------------------------------------------------------------ K1b
-// One warp per 32 candidate-mask words (1024 chunks). The warp's candidates are spread
-// evenly over its lanes (warp prefix over popcounts; lane j takes candidate j, j+32, ...)
-// so a clustered run of changed chunks costs ceil(count/32) dependent insert chains, not
-// one chain per candidate of the densest word.
+// Record inserts of the deferred 256-chunk tiles (all tiles at checkpoint 0, the ragged
+// tail, and whatever overflowed K1's ring): one warp per (tile, round of 32 candidates).
+// Block 0 of K1b turns the dirty-tile bitmap into the tree kernels' work description: the
+// compact list of dirty stage-0 tiles (block scan) and, per upper group, the number of
+// dirty children (the climb target of the tree kernels).
+__device__ void build_tree_work(const InsertParams& p) {
+  __shared__ uint32_t s_ws[8], s_carry;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const uint64_t nw = (p.n_tiles + 31) / 32;
+  if (tid == 0) s_carry = 0;
+  __syncthreads();
+  for (uint64_t base = 0; base < nw; base += 256) {
+    const uint64_t wi = base + tid;
+    uint32_t bits = wi < nw ? __ldcg(p.dbits + wi) : 0u;
+    if (wi == nw - 1 && (p.n_tiles & 31)) bits &= (1u << (p.n_tiles & 31)) - 1u;
+    const uint32_t pc = __popc(bits);
+    uint32_t incl = pc;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += v;
+    }
+    if (lane == 31) s_ws[wid] = incl;
+    __syncthreads();
+    uint32_t off = s_carry, tot = 0;
+    for (int i = 0; i < 8; ++i) {
+      if (i < wid) off += s_ws[i];
+      tot += s_ws[i];
+    }
+    off += incl - pc;
+    for (uint32_t m = bits; m; m &= m - 1) p.wl0[off++] = (uint32_t)(wi * 32 + (__ffs(m) - 1));
+    __syncthreads();
+    if (tid == 0) s_carry += tot;
+    __syncthreads();
+  }
+  if (tid == 0) p.tot->wl_count[0] = s_carry;
+  // dirty children per group, stage by stage
+  for (int s = 1; s < p.S; ++s) {
+    // groups of stage s: children are positions of stage s-1 (tiles for s == 1)
+    uint64_t nchild = p.n_tiles;
+    for (int t = 1; t < s; ++t) nchild >>= p.gsz[t];
+    const uint64_t ngroups = nchild >> p.gsz[s];
+    const uint32_t per = 1u << p.gsz[s];
+    for (uint64_t G = tid; G < ngroups; G += blockDim.x) {
+      uint32_t cnt = 0;
+      if (s == 1) {
+        const uint64_t b0 = G * per;
+        for (uint64_t b = b0; b < b0 + per;) {
+          if ((b & 31) == 0 && b + 32 <= b0 + per) { cnt += __popc(__ldcg(p.dbits + (b >> 5))); b += 32; }
+          else { cnt += (__ldcg(p.dbits + (b >> 5)) >> (b & 31)) & 1u; ++b; }
+        }
+      } else {
+        for (uint64_t ch = G * per; ch < (G + 1) * per; ++ch) cnt += p.dcnt[s - 1][ch] != 0;
+      }
+      p.dcnt[s][G] = cnt;
+    }
+    __syncthreads();
+  }
+}
+
 __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
   pdl_launch_dependents();
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const uint64_t warp = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t wbase = warp * 32;                 // first mask word of this warp
-  __shared__ uint32_t s_cnt, s_base;
-  __shared__ uint32_t s_tiles[256];
   __shared__ uint32_t s_word[8][32], s_excl[8][32];
-  if (threadIdx.x == 0) s_cnt = 0;
-  __syncthreads();
   pdl_wait();
-
-  const uint32_t word = (wbase + lane < p.nwords) ? p.cand[wbase + lane] : 0u;
-  const uint32_t cnt = __popc(word);
-  uint32_t incl = cnt;
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += v;
+  if (blockIdx.x == 0) {
+    build_tree_work(p);
+    return;
   }
-  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  s_word[wid][lane] = word;
-  s_excl[wid][lane] = incl - cnt;
-  __syncwarp();
-
-  for (uint32_t base = 0; base < total; base += 32) {
-    const uint32_t j = base + lane;
-    const bool has = j < total;
-    const unsigned active = __ballot_sync(0xffffffffu, has);
-    if (has) {
-      // source lane: last l with excl[l] <= j
-      int lo = 0;
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1)
-        if (lo + step < 32 && s_excl[wid][lo + step] <= j) lo += step;
-      const uint32_t b = __fns(s_word[wid][lo], 0, (int)(j - s_excl[wid][lo]) + 1);
-      const uint64_t c = (wbase + lo) * 32 + b;
-      const ulonglong2 v = reinterpret_cast<const ulonglong2*>(p.prev)[c];
-      const Digest d{v.x, v.y};
-      const uint32_t node = node_of_chunk(p.g, c);
-      // warp-level de-duplication of identical digests
-      const unsigned m1 = __match_any_sync(active, d.lo);
-      const unsigned m2 = __match_any_sync(active, d.hi);
-      const unsigned grp = m1 & m2;
-      const int leader = __ffs(grp) - 1;
-      uint32_t minnode = node;   // minimum node id of the group (every active lane shuffles)
-      for (unsigned a = active; a; a &= a - 1) {
-        const int sl = __ffs(a) - 1;
-        const uint32_t vv = __shfl_sync(active, node, sl);
-        if ((grp >> sl) & 1u) minnode = vv < minnode ? vv : minnode;
-      }
-      uint32_t slot = 0;
-      if (lane == leader) {
-        bool claimed;
-        slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed);
-      }
-      slot = __shfl_sync(active, slot, leader);
-      st_evict_last_u32(p.slot_of + c, slot, policy_evict_last());
-      // dirty stage-0 tile of this chunk (R3 virtual positions)
-      const uint32_t T = (uint32_t)(vpos_of_chunk(p.g, c) >> p.g.t0);
-      const unsigned tg = __match_any_sync(active, T);
-      if (lane == __ffs(tg) - 1) {
-        if (atomicExch(&p.dirty[0][T], p.g.epoch) != p.g.epoch) {
-          const uint32_t i = atomicAdd(&s_cnt, 1u);
-          if (i < 256) s_tiles[i] = T;
-          else p.wl0[atomicAdd(&p.tot->wl_count[0], 1u)] = T;   // overflow: direct append
-          // count dirty children up the stage hierarchy (the tree kernels' climb target)
-          uint64_t x = T;
-          for (int s = 1; s < p.S; ++s) {
-            const uint64_t P = x >> p.gsz[s];
-            if (atomicAdd(&p.cnt[s][P], 1u) != 0) break;
-            p.dirty[s][P] = p.g.epoch;
-            x = P;
-          }
-        }
+  unsigned long long tk0 = 0;
+  if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tk0));
+  const uint32_t count = *(volatile uint32_t*)&p.tot->defer_count;
+  const uint32_t nwarps = (gridDim.x - 1) * (blockDim.x >> 5);
+  unsigned long long ncand = 0;
+  for (uint32_t w = (blockIdx.x - 1) * (blockDim.x >> 5) + wid; w < count; w += nwarps) {
+    unsigned long long t1 = 0, t2 = 0, t3 = 0;
+    if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t1));
+    const uint32_t e = p.defer[w];
+    const uint32_t tile = e >> 3;
+    const uint64_t wi = (uint64_t)tile * 8 + lane;
+    const uint32_t word = (lane < 8 && wi < p.nwords) ? __ldcg(p.cand + wi) : 0u;
+    if (p.trace) { __syncwarp(); asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t2)); }
+    insert_tile(p, tile, word, s_word[wid], s_excl[wid], ncand, (int)(e & 7));
+    if (p.trace) {
+      asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t3));
+      if (lane == 0) {
+        const uint32_t i = atomicAdd(p.trace_n, 1u);
+        p.trace[i] = make_ulonglong4(tk0, t1, t2, t3);
       }
     }
   }
-  if (lane == 0 && total) atomicAdd(&p.tot->n_cand, (unsigned long long)total);
-  __syncthreads();
-  const uint32_t nt = s_cnt < 256 ? s_cnt : 256;
-  if (threadIdx.x == 0 && nt) s_base = atomicAdd(&p.tot->wl_count[0], nt);
-  __syncthreads();
-  if (threadIdx.x < nt) p.wl0[s_base + threadIdx.x] = s_tiles[threadIdx.x];
+  if (lane == 0 && ncand) atomicAdd(&p.tot->n_cand, ncand);
 }
 
 // ------------------------------------------------------------------ rehash
@@ -255,7 +421,7 @@ __global__ void rehash_kernel(const Slot* old_tab, uint64_t old_cap, Slot* new_t
 
 // ------------------------------------------------------------------ launchers
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes) {
-  *smem_bytes = 1024 + (size_t)p.nst * p.stage_bytes + (size_t)p.nst * kLeafThreads * 16 + (size_t)p.nst * 8;
+  *smem_bytes = 1008 + (size_t)p.nst * p.stage_bytes + (size_t)p.nst * kLeafThreads * 16 + 64 + sizeof(K1Ring);
   return cudaSuccess;
 }
 
@@ -266,8 +432,8 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   const uint64_t n_tiles = p.n_main / kLeafThreads;
   uint64_t grid = (uint64_t)num_sms * 2;
   if (grid > n_tiles) grid = n_tiles;
-  if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
-  else leaf_hash_kernel<0><<<(unsigned)grid, kLeafThreads, smem, st>>>(*tmap, p);
+  if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  else leaf_hash_kernel<0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   return cudaGetLastError();
 }
 
@@ -278,16 +444,17 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_insert(const InsertParams& p, cudaStream_t st) {
-  const uint64_t warps = (p.nwords + 31) / 32;
-  const uint64_t blocks = (warps + 7) / 8;
+cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st) {
+  const uint64_t tiles = (p.nwords + 7) / 8;
+  uint64_t blocks = (tiles + 7) / 8 + 1;   // + block 0: tree work description
+  if (blocks > (uint64_t)num_sms * 8) blocks = (uint64_t)num_sms * 8;
   if (blocks) return launch_pdl(insert_kernel, (unsigned)blocks, 256, 0, st, p);
   return cudaSuccess;
 }
 
 cudaError_t leaf_setup_attributes() {
   // the largest dynamic smem any leaf configuration asks for (C >= 128: 3 x 36 KB; C < 128: <= 96 KB)
-  const int smem = 1024 + 110 * 1024;
+  const int smem = 1008 + 3 * (32768 + 4096) + 64 + (int)sizeof(K1Ring);   // the largest leaf configuration
   cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;

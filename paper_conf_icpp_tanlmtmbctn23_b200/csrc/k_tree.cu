@@ -19,9 +19,10 @@
 // every POTENTIAL shifted pair, l.38 — a superset of the pairs Alg.1 looks up); pass 2
 // issues all record operations at once (phase 2: insert, l.29; phase 3: lookup, l.39);
 // pass 3 (phase 3) replays the labels with the lookup results and emits the regions.
-// Groups holding no non-FIXED leaf are never visited (K1b builds the stage-0 worklist and
-// counts dirty children per upper group); the warp that finishes the LAST dirty child of
-// an upper group climbs and processes that group too, so every stage runs in this launch.
+// Only dirty groups are visited: K1/K1t mark the tree tiles holding a non-FIXED leaf in a
+// bitmap, K1b compacts it into a worklist and counts the dirty children of every upper
+// group; the warp finishing the LAST dirty child of a group climbs and processes that
+// group too, so every stage runs in this launch.
 //
 // Phase-3 emission ("save roots", R8/R10): a FIRST/SHIFT child of a DONE parent (or the
 // FIRST/SHIFT root) becomes a region. Stage 0 records its regions per tile in leaf
@@ -654,17 +655,43 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
   __syncthreads();
   pdl_wait();
   unsigned long long ins = 0, coll = 0;
-  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
-  unsigned* next = &p.tot->tree_next[PHASE - 2];
-  for (;;) {
-    uint32_t w = 0;
-    if (lane == 0) w = atomicAdd(next, 1u);
-    w = __shfl_sync(0xffffffffu, w, 0);
-    if (w >= count) break;
+
+  // Climb from (stage s, group G) after it is finished: arrive at the parent; the warp of
+  // the last arrival processes the parent (phase 2: when any child was dirty; phase 3:
+  // the parent's dirty-children count was recorded by phase 2).
+  auto climb = [&](Ctx& c) {
+    while (c.s < p.S - 1) {
+      const StageParams& up = p.st[c.s + 1];
+      const uint64_t P = c.G >> up.gsz;
+      uint32_t old = 0;
+      __threadfence();
+      if (lane == 0) old = atomicAdd((PHASE == 2 ? up.arr2 : up.arr3) + P, 1u);
+      old = __shfl_sync(0xffffffffu, old, 0);
+      if (old + 1 != __ldcg(up.dcnt + P)) return;   // not the last dirty child
+      __threadfence();
+      c.s += 1;
+      c.G = P;
+      c.Lin = up.Lin;
+      c.gsz = up.gsz;
+      c.P0 = 1ull << c.gsz;
+      c.leaf = false;
+      c.tdig = up.tdig + (P << c.gsz);
+      c.tsrc = up.tsrc + ((P << c.gsz) << 1);
+      unsigned long long t0 = p.trace ? gtimer() : 0;
+      process_group<PHASE>(c, ws, ins, coll, lc);
+      if (PHASE == 2 && lane == 0) up.dirty[P] = p.g.epoch;
+      if (p.trace && lane == 0) {
+        const uint32_t i = atomicAdd(p.trace_n, 1u);
+        p.trace[i] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
+      }
+    }
+  };
+
+  auto run_tile = [&](uint64_t T) {
     Ctx c;
     c.p = &p;
     c.s = 0;
-    c.G = p.wl0[w];
+    c.G = T;
     c.Lin = 0;
     c.gsz = p.st[0].gsz;
     c.P0 = 1ull << c.gsz;
@@ -678,32 +705,17 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
       p.trace[i] = make_ulonglong4(t0, gtimer(), (unsigned long long)c.G, PHASE);
       p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 10 + PHASE);
     }
-    // climb: the warp finishing the last dirty child of a group processes that group
-    while (c.s < p.S - 1) {
-      const StageParams& up = p.st[c.s + 1];
-      const uint64_t P = c.G >> up.gsz;
-      uint32_t old = 0;
-      __threadfence();
-      if (lane == 0) old = atomicAdd((PHASE == 2 ? up.done2 : up.done3) + P, 1u);
-      old = __shfl_sync(0xffffffffu, old, 0);
-      const uint32_t need = __ldcg(up.cnt + P);
-      if (old + 1 != need) break;
-      __threadfence();
-      c.s += 1;
-      c.G = P;
-      c.Lin = up.Lin;
-      c.gsz = up.gsz;
-      c.P0 = 1ull << c.gsz;
-      c.leaf = false;
-      c.tdig = up.tdig + (P << c.gsz);
-      c.tsrc = up.tsrc + ((P << c.gsz) << 1);
-      t0 = p.trace ? gtimer() : 0;
-      process_group<PHASE>(c, ws, ins, coll, lc);
-      if (p.trace && lane == 0) {
-        const uint32_t i = atomicAdd(p.trace_n, 1u);
-        p.trace[i] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
-      }
-    }
+    return c;
+  };
+
+  // dirty stage-0 tiles (K1b's list); climb on the last DIRTY child of each group
+  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
+  const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
+  for (uint64_t w = (uint64_t)blockIdx.x * kWarps + wid; w < count; w += nwarps) {
+    const uint64_t T = __ldcg(p.wl0 + w);
+    Ctx c = run_tile(T);
+    if (PHASE == 2 && lane == 0) p.st[0].dirty[T] = p.g.epoch;
+    climb(c);
   }
   if (ins) atomicAdd(&s_cnt[3], ins);
   if (PHASE == 2 && coll) atomicAdd(&p.tot->collisions, coll);
@@ -721,9 +733,13 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
   }
 }
 
+static int g_tree_blocks_per_sm[2] = {0, 0};
+
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st) {
-  uint64_t grid = (uint64_t)num_sms * 8;
-  const uint64_t need = (p.n_tiles + kWarps - 1) / kWarps;
+  // all CTAs resident at once (static tile striding relies on it): occupancy-sized grid
+  const int bps = g_tree_blocks_per_sm[phase - 2] > 0 ? g_tree_blocks_per_sm[phase - 2] : 2;
+  uint64_t grid = (uint64_t)num_sms * bps;
+  const uint64_t need = (p.n_tiles + kWarps - 1) / kWarps;   // one warp per tile when it fits
   if (grid > need) grid = need ? need : 1;
   const size_t smem = kWarps * sizeof(WarpSmem);
   if (phase == 2) return launch_pdl(tree_kernel<2>, (unsigned)grid, kTreeThreads, smem, st, p);
@@ -734,6 +750,10 @@ cudaError_t tree_setup_attributes() {
   const int smem = (int)(kWarps * sizeof(WarpSmem));
   cudaError_t e = cudaFuncSetAttribute(tree_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tree_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_tree_blocks_per_sm[0], tree_kernel<2>, kTreeThreads, smem);
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_tree_blocks_per_sm[1], tree_kernel<3>, kTreeThreads, smem);
   return e;
 }
 

@@ -3,7 +3,7 @@
 // Launch order per checkpoint:
 //   K1  leaf hash + fixed test (TMA-staged, persistent)      Alg.1 l.1-5, l.21
 //   K1t leaf pass for the ragged tail (direct loads)           same
-//   K1b record insert + dirty-tile worklist                    Alg.1 l.6-19 (R6)
+//   K1b record inserts of the candidate chunks                 Alg.1 l.6-19 (R6)
 //   P2  phase 2, all stages in one launch (warp per group)     Alg.1 l.24-32
 //   P3  phase 3 + emission, all stages in one launch           Alg.1 l.33-46 (R7-R10)
 //   KR/KO/KG/KD tile reduce, offsets + header, entries, data
@@ -31,7 +31,30 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
   uint32_t gather_next;              // work-stealing cursor of the gather kernel
   uint32_t big_count;                // FIRST regions deferred to the grid-wide data pass
-  uint32_t pad2[4];
+  uint32_t defer_count;              // 256-chunk leaf tiles whose inserts K1 left to K1b
+  uint32_t insert_next;              // work-stealing cursor of K1b
+  uint32_t pad2[2];
+};
+
+struct InsertParams {
+  Geo g;
+  const Digest* prev;
+  const uint32_t* cand;
+  uint64_t nwords;
+  Slot* tab;
+  uint64_t cap;
+  uint32_t* slot_of;
+  Totals* tot;
+  uint32_t* defer;               // (tile << 3 | round) entries left for K1b
+  // tree work discovery (K1/K1t mark, K1b block 0 compacts)
+  uint32_t* dbits;               // dirty bit per stage-0 tree tile
+  uint64_t n_tiles;
+  uint32_t* wl0;                 // out: dirty stage-0 tiles
+  int S;
+  int gsz[kMaxStages];
+  uint32_t* dcnt[kMaxStages];    // out: s >= 1, dirty children per group
+  ulonglong4* trace;             // diagnostics (CKPT_TRACE)
+  uint32_t* trace_n;
 };
 
 struct LeafParams {
@@ -45,22 +68,8 @@ struct LeafParams {
   int nst;               // pipeline stages
   Digest* prev;          // persistent leaf digests Tree(leaf), 16 n bytes
   uint32_t* cand;        // candidate (non-FIXED) bit per chunk
-};
-
-struct InsertParams {
-  Geo g;
-  const Digest* prev;
-  const uint32_t* cand;
-  uint64_t nwords;
-  Slot* tab;
-  uint64_t cap;
-  uint32_t* slot_of;
-  uint32_t* wl0;
-  Totals* tot;
-  int S;                         // tree stages
-  uint32_t* dirty[kMaxStages];   // per stage: epoch mark of dirty groups
-  uint32_t* cnt[kMaxStages];     // per stage s >= 1: dirty children of each group
-  int gsz[kMaxStages];
+  int insert_warp;       // 1: K1's insert warp performs the record inserts (k > 0)
+  InsertParams ins;      // record insert state (K1's insert warp, K1b)
 };
 
 struct LevelIO {               // per-position arrays at one height (stage boundary)
@@ -77,16 +86,17 @@ struct StageParams {
   LevelIO in;                  // s >= 1: input arrays (written by stage s-1)
   Digest* tdig;                // per group: digests of internal nodes (2^gsz entries)
   unsigned long long* tsrc;    // per group: sources of SHIFT nodes (2 * 2^gsz entries)
-  uint32_t* cnt;               // s >= 1: dirty children per group (K1b)
-  uint32_t* done2;             // s >= 1: finished children per group, phase 2
-  uint32_t* done3;             //                                      phase 3
+  uint32_t* dirty;             // epoch mark of this stage's dirty groups (written in phase 2)
+  uint32_t* arr2;              // s >= 1: arrivals of dirty children, phase 2
+  uint32_t* arr3;              //                                     phase 3
+  const uint32_t* dcnt;        // s >= 1: dirty children per group (K1b)
 };
 
 struct TreeParams {
   Geo g;
   int S;
   uint64_t n_tiles;
-  const uint32_t* wl0;         // stage-0 worklist (dirty tiles)
+  const uint32_t* wl0;         // dirty stage-0 tiles (K1b)
   const uint32_t* cand;
   const uint32_t* slot_of;
   const Digest* prev;
@@ -109,7 +119,7 @@ struct CompactParams {
   const uint4* scratch;
   unsigned long long* blocksum;  // 3 per reduce block
   uint4* toff;                   // per tile {F_off, S_off, data_off lo, data_off hi}
-  const uint32_t* wl0;
+  const uint32_t* wl0;           // dirty stage-0 tiles
   Totals* tot;
   ulonglong2* big;               // deferred big FIRST regions: {data offset, source offset}
   unsigned long long* big_len;   //                              byte length
@@ -140,7 +150,7 @@ cudaError_t leaf_setup_attributes();
 cudaError_t tree_setup_attributes();
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
-cudaError_t launch_insert(const InsertParams& p, cudaStream_t st);
+cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st);
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st);
