@@ -282,22 +282,26 @@ def run_ours(args):
     for k in range(Wm):
         diffs.append(ck.checkpoint(bufs[k], stream=stream))
         if k == 0:
-            ck0 = ck.phase_times()
+            ck0 = ck.phase_times(0)
     n = (B + C - 1) // C
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     k1_ms, phase = [], []
     barrier(ws)
     torch.cuda.synchronize()
+    raw = []
     with ClockSampler(local) as clk:
         ev0.record(stream)
         for k in range(Wm, Wm + K):
-            d = ck.checkpoint(bufs[k], stream=stream)
-            diffs.append(d)
-            pt = ck.phase_times()
-            phase.append(pt)
-            k1_ms.append(pt["leaf_hash"])
+            raw.append(ck.checkpoint(bufs[k], nbytes=B, stream=stream, raw=True))
         ev1.record(stream)
         stream.synchronize()
+    # per-phase device times of the timed checkpoints (CUDA events recorded by the library
+    # on `stream` during the timed region; queried only now)
+    for k in range(Wm, Wm + K):
+        pt = ck.phase_times(k)
+        phase.append(pt)
+        k1_ms.append(pt["leaf_hash"])
+    diffs.extend(r.as_dict() for r in raw)
     torch.cuda.synchronize()
     barrier(ws)
     ms_local = ev0.elapsed_time(ev1)

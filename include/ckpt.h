@@ -137,6 +137,9 @@ CKPT_API int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_
  * synchronisation, [9] bookkeeping after it.  n <= 10 values are written. */
 CKPT_API int ckpt_set_profiling(ckpt_handle h, int enable);
 CKPT_API int ckpt_phase_times(ckpt_handle h, float* times, int n);
+/* Same for checkpoint `id` (device times kept for the latest 256 profiled checkpoints; the
+ * event queries happen here, never inside ckpt_checkpoint). Errors: CKPT_ERANGE. */
+CKPT_API int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n);
 
 /* Release all device memory of the handle (record, leaf digests, every diff). */
 CKPT_API int ckpt_destroy(ckpt_handle h);

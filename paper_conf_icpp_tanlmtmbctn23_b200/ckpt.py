@@ -21,7 +21,7 @@ CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_EC
 ABI_FUNCTIONS = [
     "ckpt_create", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
     "ckpt_checkpoint_host", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
-    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_destroy", "ckpt_strerror",
+    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_destroy", "ckpt_strerror",
 ]
 
 
@@ -82,6 +82,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_record_dump": ([vp, vp, vp, vp, u64, P(u64)], i32),
             "ckpt_set_profiling": ([vp, i32], i32),
             "ckpt_phase_times": ([vp, P(ctypes.c_float), i32], i32),
+            "ckpt_phase_times_of": ([vp, u32, P(ctypes.c_float), i32], i32),
             "ckpt_destroy": ([vp], i32),
             "ckpt_strerror": ([i32], ctypes.c_char_p),
         }
@@ -219,12 +220,20 @@ class Checkpointer:
     def set_profiling(self, on: bool = True) -> None:
         lib().ckpt_set_profiling(self._h, 1 if on else 0)
 
-    def phase_times(self) -> dict:
+    PHASES = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total",
+              "host_pre", "host_enqueue", "host_sync_wait", "host_post"]
+
+    def phase_times(self, cid: int | None = None) -> dict:
+        """Per-phase device times (ms) of checkpoint cid (default: the latest), measured with
+        CUDA events on the caller's stream when profiling is on; host times for the latest."""
         t = (ctypes.c_float * 10)()
-        lib().ckpt_phase_times(self._h, t, 10)
-        names = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total",
-                 "host_pre", "host_enqueue", "host_sync_wait", "host_post"]
-        return {names[i]: t[i] for i in range(10)}
+        if cid is None:
+            lib().ckpt_phase_times(self._h, t, 10)
+        else:
+            rc = lib().ckpt_phase_times_of(self._h, cid, t, 10)
+            if rc != CKPT_OK:
+                raise CkptError(rc, "ckpt_phase_times_of")
+        return {self.PHASES[i]: t[i] for i in range(10)}
 
     def close(self) -> None:
         if getattr(self, "_h", None):

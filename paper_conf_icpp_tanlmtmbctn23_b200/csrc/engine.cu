@@ -84,8 +84,12 @@ struct ckpt_ctx {
   uint64_t staging_size = 0;
   cudaStream_t internal = nullptr;
   bool prof = false;
-  cudaEvent_t ev[6] = {};
-  float times[12] = {};
+  // per-checkpoint event sets (ring), queried lazily so the call itself never waits on them
+  static constexpr int kEvRing = 256;
+  cudaEvent_t evr[kEvRing][6] = {};
+  int64_t ev_id[kEvRing] = {};
+  cudaEvent_t* ev = nullptr;     // event set of the current call
+  float times[12] = {};          // host times of the latest call ([6..9])
   PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   std::vector<void*> allocs;   // per-geometry allocations
   // diagnostics: CKPT_TRACE=<file prefix> records per-group tree timings of each call
@@ -347,7 +351,10 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
   }
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaMallocHost(&h->tot_host, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  for (int i = 0; i < 6; ++i) cudaEventCreate(&h->ev[i]);
+  for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
+    h->ev_id[r] = -1;
+    for (int i = 0; i < 6; ++i) cudaEventCreate(&h->evr[r][i]);
+  }
   *out = h;
   return CKPT_OK;
 }
@@ -361,7 +368,8 @@ int ckpt_destroy(ckpt_handle h) {
   if (h->tab) cudaFree(h->tab);
   if (h->tot_host) cudaFreeHost(h->tot_host);
   if (h->staging) cudaFree(h->staging);
-  for (int i = 0; i < 6; ++i) if (h->ev[i]) cudaEventDestroy(h->ev[i]);
+  for (int r = 0; r < ckpt_ctx::kEvRing; ++r)
+    for (int i = 0; i < 6; ++i) if (h->evr[r][i]) cudaEventDestroy(h->evr[r][i]);
   if (h->internal) cudaStreamDestroy(h->internal);
   cudaGetLastError();
   delete h;
@@ -380,10 +388,30 @@ int ckpt_set_profiling(ckpt_handle h, int enable) {
   return CKPT_OK;
 }
 
+int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
+  if (!h || !times) return CKPT_EINVAL;
+  if (id >= h->diffs.size()) return CKPT_ERANGE;
+  const int r = (int)(id % ckpt_ctx::kEvRing);
+  float t[10] = {};
+  if (h->ev_id[r] == (int64_t)id) {
+    cudaEvent_t* e = h->evr[r];
+    for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], e[i], e[i + 1]);   // K1, K1b, phase 2, phase 3, compaction
+    cudaEventElapsedTime(&t[5], e[0], e[5]);
+    cudaGetLastError();
+  }
+  if (id + 1 == h->diffs.size())
+    for (int i = 6; i < 10; ++i) t[i] = h->times[i];
+  for (int i = 0; i < n && i < 10; ++i) times[i] = t[i];
+  return CKPT_OK;
+}
+
 int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
-  for (int i = 0; i < n && i < 12; ++i) times[i] = h->times[i];
-  return CKPT_OK;
+  if (h->diffs.empty()) {
+    for (int i = 0; i < n && i < 10; ++i) times[i] = 0.f;
+    return CKPT_OK;
+  }
+  return ckpt_phase_times_of(h, (uint32_t)(h->diffs.size() - 1), times, n);
 }
 
 int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
@@ -466,6 +494,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     if (r != CKPT_OK) { h->poisoned = true; return r; }
   }
 
+  h->ev = h->evr[k % ckpt_ctx::kEvRing];
+  h->ev_id[k % ckpt_ctx::kEvRing] = h->prof ? (int64_t)k : -1;
   const auto t_pre = clk::now();
   CK(cudaMemsetAsync(h->ctr, 0, h->ctr_bytes, st));
   if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
@@ -535,11 +565,6 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     char path[512];
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
     if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), nt, f); fclose(f); }
-  }
-  if (h->prof) {
-    for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&h->times[i], h->ev[i], h->ev[i + 1]);
-    cudaEventElapsedTime(&h->times[5], h->ev[0], h->ev[5]);
-    // times: [0] K1 [1] K1b [2] phase 2 [3] phase 3 [4] compaction [5] total
   }
   h->live += t.n_first + t.p2_inserts;
   DiffRec rec;

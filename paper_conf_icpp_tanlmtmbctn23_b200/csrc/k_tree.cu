@@ -558,6 +558,7 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     }
   }
 
+  if (p.trace && lane == 0) ws.tp[3] = gtimer();
   // ---- group root (single position at level gsz: lane 0 bit 0)
   const uint32_t rF = __shfl_sync(0xffffffffu, F, 0) & 1u;
   const uint32_t rS = __shfl_sync(0xffffffffu, S, 0) & 1u;
@@ -585,6 +586,7 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
   }
   __syncwarp();
 
+  if (p.trace && lane == 0) ws.tp[4] = gtimer();
   // ---- stage-0 compaction of this tile's regions (leaf order; FIRST list then SHIFT list)
   if (PHASE == 3 && c.leaf) {
     const uint32_t wF = ws.stF[lane], wS = ws.stS[lane];
@@ -701,9 +703,10 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
     unsigned long long t0 = p.trace ? gtimer() : 0;
     process_group<PHASE>(c, ws, ins, coll, lc);
     if (p.trace && lane == 0) {
-      const uint32_t i = atomicAdd(p.trace_n, 2u);
+      const uint32_t i = atomicAdd(p.trace_n, 3u);
       p.trace[i] = make_ulonglong4(t0, gtimer(), (unsigned long long)c.G, PHASE);
       p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 10 + PHASE);
+      p.trace[i + 2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 20 + PHASE);
     }
     return c;
   };

@@ -23,3 +23,11 @@ for f in sorted(glob.glob(sys.argv[1] + ".*.bin"))[-1:]:
         g = a[idx - 1].astype(np.int64); q = a[idx].astype(np.int64)
         print(f"phase{ph} per-tile median us: input {np.median(q[:,0]-g[:,0])/1e3:.2f}  pass1 {np.median(q[:,1]-q[:,0])/1e3:.2f}  "
               f"pass2 {np.median(q[:,2]-q[:,1])/1e3:.2f}  pass3+root+compaction {np.median(g[:,1]-q[:,2])/1e3:.2f}")
+
+for f in sorted(glob.glob(sys.argv[1] + ".*.bin"))[-1:]:
+    a = np.fromfile(f, dtype=np.uint64).reshape(-1, 4).astype(np.int64)
+    for ph in (2, 3):
+        idx = np.nonzero(a[:, 3] == 20 + ph)[0]
+        if len(idx) == 0: continue
+        g = a[idx - 2]; q1 = a[idx - 1]; q2 = a[idx]
+        print(f"phase{ph} tail split median us: pass3/labels {np.median(q2[:,0]-q1[:,2])/1e3:.2f} root {np.median(q2[:,1]-q2[:,0])/1e3:.2f} compaction {np.median(g[:,1]-q2[:,1])/1e3:.2f}")
