@@ -516,12 +516,13 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
   if (p.trace && lane == 0) ws.tp[2] = gtimer();
 
   if (PHASE == 2) {
-    // the FIRST label chain up to the group root
+    // the FIRST label chain up to the group root (stops once no FIRST node is left)
     for (int lv = 1; lv <= gsz; ++lv) {
       const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
       uint32_t l, r;
       lr(F, Nc, l, r);
       F = (l & r & valid_word(Np) & (lv == 1 ? ~leafm1 : 0xFFFFFFFFu)) | (lv == 1 ? lF1 : 0u);
+      if (!__any_sync(0xffffffffu, F != 0)) break;
     }
   } else {
     // ---- pass 3: Alg.1 l.33-46 with the lookup results; emission of "roots" (R8)
@@ -555,6 +556,13 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
       F = bothF | (lv == 1 ? lF1 : 0u);
       X = bothX | (lv == 1 ? lX1 : 0u);
       S = hitS | (lv == 1 ? lS1 : 0u);
+      if (lv < gsz && !__any_sync(0xffffffffu, (F | S) != 0)) {
+        // no FIRST/SHIFT node left: the levels above hold only FIXED and DONE nodes and
+        // emit nothing; the root is FIXED iff every node of this level is FIXED
+        const bool allX = __all_sync(0xffffffffu, X == valid_word(Np));
+        X = (lane == 0 && allX) ? 1u : 0u;
+        break;
+      }
     }
   }
 
