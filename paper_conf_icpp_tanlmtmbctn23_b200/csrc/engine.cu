@@ -182,6 +182,9 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     const size_t dbits_off = bytes;
     bytes += ((n_tiles + 31) / 32) * sizeof(uint32_t);
     bytes = (bytes + 255) & ~size_t(255);
+    const size_t bsum_off = bytes;
+    bytes += (3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3) * sizeof(unsigned long long);
+    bytes = (bytes + 255) & ~size_t(255);
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
@@ -191,6 +194,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     h->ctr_bytes = bytes;
     h->tot = reinterpret_cast<Totals*>(h->ctr);
     h->dbits = reinterpret_cast<uint32_t*>(h->ctr + dbits_off);
+    h->blocksum = reinterpret_cast<unsigned long long*>(h->ctr + bsum_off);
     for (int s = 1; s < h->S; ++s) {
       h->arr2[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
       h->arr3[s] = h->arr2[s] + h->ngroups[s];
@@ -203,7 +207,6 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->lmask, n_tiles * 192);   // k_tree.cu kLmWords
   AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
   AL(h->toff, n_tiles);
-  AL(h->blocksum, 3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3);
   AL(h->big, B / (1 << 20) + 2);
   AL(h->big_len, B / (1 << 20) + 2);
 #undef AL
@@ -518,6 +521,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
+  tp.blocksum = h->blocksum;
   tp.trace = h->trace; tp.trace_n = h->trace_n;
   tp.dbg = h->dbg;
 
@@ -547,6 +551,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.toff = h->toff; cp.wl0 = h->wl0; cp.tot = h->tot;
   cp.big = h->big; cp.big_len = h->big_len;
   cp.out = out; cp.buf = buf;
+  cp.trace = h->trace; cp.trace_n = h->trace_n;
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
   CK(cudaMemcpyAsync(h->tot_host, h->tot, sizeof(Totals), cudaMemcpyDeviceToHost, st));

@@ -4,8 +4,8 @@
 // difference directly on the GPU memory ... pre-calculates offsets in the consolidated
 // difference and assigns GPU threads to parallelize the data transfers", with "a
 // team of threads to copy each chunk" so accesses coalesce.
-//   KR reduce_kernel : per 1024 stage-0 tiles, sums of (#FIRST regions, #SHIFT regions,
-//                      FIRST bytes) over tiles dirty in this checkpoint.
+//   (the per-1024-tile sums of #FIRST regions, #SHIFT regions and FIRST bytes are
+//    accumulated by the phase-3 kernel as it writes the tile counts)
 //   KO offsets_kernel: prefix over earlier blocks + block scan -> per-tile offsets;
 //                      the last block writes the 64-B header, the zero pad and totals.
 //   KG gather_kernel : one CTA per dirty tile writes its FIRST entries (u32 node) and
@@ -161,6 +161,8 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
   const uint64_t nwarps = (uint64_t)gridDim.x * kGW;
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   for (uint64_t w = (uint64_t)blockIdx.x * kGW + wid; w < count; w += nwarps) {
+    unsigned long long tg0 = 0, tg1 = 0, tg2 = 0;
+    if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg0));
     const uint64_t T = __ldcg(p.wl0 + w);
     const uint4 cnt = p.tilecnt[T];
     if (cnt.w != g.epoch) continue;
@@ -169,6 +171,7 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
     const uint4 off = p.toff[T];
     const unsigned long long doff = (unsigned long long)off.z | ((unsigned long long)off.w << 32);
     const uint4* recs = p.scratch + ((uint64_t)T << g.t0);
+    if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg1));
     // SHIFT entries (R13): u32 node, u32 src node, u32 src ckpt
     for (uint32_t i = lane; i < nS; i += 32) {
       const uint4 r = recs[nF + i];
@@ -212,15 +215,17 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
       carry += __shfl_sync(0xffffffffu, incl, 31);
       __syncwarp();
       const uint32_t nreg = (nF - b0) < 32 ? (nF - b0) : 32;
-      // stream copy of the inline bytes: unit x covers [16x, 16x+16)
+      // stream copy of the inline bytes: unit x covers [16x, 16x+16); 8 independent units
+      // per lane per iteration (4 KB per warp) so a typical tile needs one round trip
       const unsigned long long nunits = (btot + 15) / 16;
-      for (unsigned long long x0 = 0; x0 < nunits; x0 += 128) {
-        uint4 v[4];
-        uint8_t* d[4];
-        unsigned long long rem[4];
-        const uint8_t* sp[4];
+      constexpr int kU = 8;
+      for (unsigned long long x0 = 0; x0 < nunits; x0 += 32 * kU) {
+        uint4 v[kU];
+        uint8_t* d[kU];
+        unsigned long long rem[kU];
+        const uint8_t* sp[kU];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < kU; ++u) {
           const unsigned long long x = x0 + u * 32 + lane;
           rem[u] = 0;
           if (x < nunits) {
@@ -229,24 +234,27 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
 #pragma unroll
             for (int step = 16; step > 0; step >>= 1)
               if (r + step < (int)nreg && gw.off[r + step] <= o) r += step;
-            // skip zero-length (deferred big) regions that share this offset
-            while (r + 1 < (int)nreg && gw.off[r + 1] <= o) ++r;
+            while (r + 1 < (int)nreg && gw.off[r + 1] <= o) ++r;   // skip deferred (zero-length) regions
             const unsigned long long rel = o - gw.off[r];
             sp[u] = p.buf + gw.src[r] + rel;
             d[u] = dat + gw.dst[r] + rel;
-            rem[u] = gw.off[r + 1 <= (int)nreg ? r + 1 : nreg] - o;
-            if (r + 1 >= (int)nreg) rem[u] = btot - o;
+            rem[u] = (r + 1 < (int)nreg ? gw.off[r + 1] : btot) - o;
             if (rem[u] >= 16) v[u] = __ldg(reinterpret_cast<const uint4*>(sp[u]));
           }
         }
 #pragma unroll
-        for (int u = 0; u < 4; ++u) {
+        for (int u = 0; u < kU; ++u) {
           if (rem[u] >= 16) *reinterpret_cast<uint4*>(d[u]) = v[u];
           else
             for (unsigned long long b = 0; b < rem[u]; ++b) d[u][b] = sp[u][b];
         }
       }
       __syncwarp();
+    }
+    if (p.trace && lane == 0) {
+      asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg2));
+      const uint32_t i = atomicAdd(p.trace_n, 1u);
+      p.trace[i] = make_ulonglong4(tg0, tg1, tg2, 77);
     }
   }
 }
@@ -274,8 +282,8 @@ __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
 
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st) {
   const unsigned nblk = (unsigned)((p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock);
-  cudaError_t e = launch_pdl(reduce_kernel, nblk, kCT, 0, st, p);
-  if (e == cudaSuccess) e = launch_pdl(offsets_kernel, nblk, kCT, 0, st, p);
+  // per-block sums were accumulated by the phase-3 kernel (k_tree.cu), so no reduce pass
+  cudaError_t e = launch_pdl(offsets_kernel, nblk, kCT, 0, st, p);
   if (e != cudaSuccess) return e;
   uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
   if (grid > (uint64_t)num_sms * 8) grid = (uint64_t)num_sms * 8;

@@ -343,6 +343,10 @@ __device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, 
   p.scratch[tile << p.g.t0] = make_uint4(node, (uint32_t)(src & 0xffffffffu), (uint32_t)(src >> 32),
                                          first ? L_FIRST : L_SHIFT);
   p.tilecnt[tile] = make_uint4(first ? 1u : 0u, first ? 0u : 1u, bytes, p.g.epoch);
+  // the tile had no region of its own (it lies inside this one): add the region to its block sum
+  unsigned long long* bs = p.blocksum + 3 * (tile / kTilesPerBlock);
+  atomicAdd(bs + (first ? 0 : 1), 1ull);
+  if (first) atomicAdd(bs + 2, (unsigned long long)bytes);
 }
 
 // Process one group through its gsz levels. PHASE 2 or 3.
@@ -644,7 +648,13 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
-    if (lane == 0) p.tilecnt[c.G] = make_uint4(nFt, nSt, bytes, g.epoch);
+    if (lane == 0) {
+      p.tilecnt[c.G] = make_uint4(nFt, nSt, bytes, g.epoch);
+      unsigned long long* bs = p.blocksum + 3 * (c.G / kTilesPerBlock);
+      if (nFt) atomicAdd(bs, (unsigned long long)nFt);
+      if (nSt) atomicAdd(bs + 1, (unsigned long long)nSt);
+      if (bytes) atomicAdd(bs + 2, (unsigned long long)bytes);
+    }
     __syncwarp();
   }
 }

@@ -104,7 +104,8 @@ struct TreeParams {
   uint64_t cap;
   uint4* scratch;              // per tile: up to 2^t0 region records {node, src_node, src_ckpt, kind}
   uint4* tilecnt;              // per tile: {nF, nS, data_bytes, epoch}
-  uint32_t* lmask;             // per tile: resolved leaf masks (phase 2 -> phase 3), 128 words
+  uint32_t* lmask;             // per tile: resolved leaf masks (phase 2 -> phase 3)
+  unsigned long long* blocksum;  // per 1024 tiles: (#FIRST, #SHIFT, FIRST bytes), zeroed per call
   Totals* tot;
   int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
   ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
@@ -125,6 +126,8 @@ struct CompactParams {
   unsigned long long* big_len;   //                              byte length
   uint8_t* out;                  // diff destination (device arena)
   const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
+  ulonglong4* trace;             // diagnostics (CKPT_TRACE)
+  uint32_t* trace_n;
 };
 
 // Launch with programmatic stream serialization (PDL): the kernel may be scheduled while
