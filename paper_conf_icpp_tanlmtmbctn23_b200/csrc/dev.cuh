@@ -229,6 +229,18 @@ __device__ __forceinline__ unsigned long long table_lookup(const Slot* tab, uint
   }
 }
 
+// Lookup continuing at slot s (the caller already checked the home slot).
+__device__ __forceinline__ unsigned long long table_lookup_from(const Slot* tab, uint64_t cap, const Digest& d, uint64_t s) {
+  for (;;) {
+    const Slot* p = tab + s;
+    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p));
+    const unsigned long long val = __ldcg(&p->val);
+    if (kv.x == d.lo && kv.y == d.hi) return val;
+    if (kv.x == kEmpty && kv.y == kEmpty) return kEmpty;
+    if (++s == cap) s = 0;
+  }
+}
+
 __device__ __forceinline__ unsigned long long pack_entry(uint32_t ckpt, uint32_t node) {
   return ((unsigned long long)ckpt << 32) | node;
 }

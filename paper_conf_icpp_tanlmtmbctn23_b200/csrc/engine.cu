@@ -62,6 +62,8 @@ struct ckpt_ctx {
   uint32_t* arr2[kMaxStages] = {};
   uint32_t* arr3[kMaxStages] = {};
   uint32_t* dcnt[kMaxStages] = {};
+  uint32_t* gm2[kMaxStages] = {};
+  uint32_t* gm3[kMaxStages] = {};
   uint32_t* wl0 = nullptr;
   uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
   uint8_t* ctr = nullptr;        // Totals + per-stage counters, zeroed by one memset per call
@@ -188,7 +190,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
-      bytes += 3 * h->ngroups[s] * sizeof(uint32_t);
+      bytes += (3 + 128) * h->ngroups[s] * sizeof(uint32_t);
     }
     AL(h->ctr, bytes);
     h->ctr_bytes = bytes;
@@ -199,6 +201,8 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
       h->arr2[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
       h->arr3[s] = h->arr2[s] + h->ngroups[s];
       h->dcnt[s] = h->arr3[s] + h->ngroups[s];
+      h->gm2[s] = h->dcnt[s] + h->ngroups[s];
+      h->gm3[s] = h->gm2[s] + 32 * h->ngroups[s];
     }
   }
   AL(h->scratch, n_tiles << h->t0);
@@ -537,6 +541,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.arr2 = h->arr2[s];
     sp.arr3 = h->arr3[s];
     sp.dcnt = h->dcnt[s];
+    sp.gm2 = h->gm2[s];
+    sp.gm3 = h->gm3[s];
   }
   CK(launch_tree(tp, 2, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[3], st));

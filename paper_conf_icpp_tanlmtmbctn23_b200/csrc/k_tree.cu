@@ -149,6 +149,38 @@ __device__ __forceinline__ void for_each_bit_balanced(WarpSmem& ws, uint32_t m, 
   __syncwarp();
 }
 
+// Batched form: lane takes items j = base + 32 t + lane (t < K) of the balanced order, so
+// it can issue the memory operations of K items before waiting on any of them.
+constexpr int kB = 4;
+struct Batch {
+  uint32_t total;
+};
+__device__ __forceinline__ uint32_t batch_begin(WarpSmem& ws, uint32_t m) {
+  const int lane = threadIdx.x & 31;
+  if (!__any_sync(0xffffffffu, m != 0)) return 0;
+  const uint32_t cnt = __popc(m);
+  uint32_t incl = cnt;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+  ws.pw[lane] = m;
+  ws.px[lane] = incl - cnt;
+  __syncwarp();
+  return total;
+}
+// item j (< total) -> (word, bit)
+__device__ __forceinline__ void batch_item(const WarpSmem& ws, uint32_t j, uint32_t& w, uint32_t& b) {
+  int lo = 0;
+#pragma unroll
+  for (int step = 16; step > 0; step >>= 1)
+    if (lo + step < 32 && ws.px[lo + step] <= j) lo += step;
+  w = (uint32_t)lo;
+  b = __fns(ws.pw[lo], 0, (int)(j - ws.px[lo]) + 1);
+}
+
 // ---- natural order -> bit-reversed order for a level of N = 2^n positions.
 // n == 10: 32-ballot transpose (lane w first fetches natural word rev5(w)); smaller
 // levels: scatter through shared memory (small groups only).
@@ -285,19 +317,41 @@ __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint6
   ws.hitS[lane] = 0;
   __syncwarp();
   const uint32_t k = p.g.k;
-  for_each_bit_balanced(ws, cand, [&](uint32_t w, uint32_t b, uint32_t pos) {
-    const uint64_t ch = chunk0 + pos;
-    const uint32_t slot = __ldg(p.slot_of + ch);
-    const unsigned long long val = __ldcg(&p.tab[slot].val);
-    if (val == pack_entry(k, node_of_chunk(p.g, ch))) {
-      atomicOr(&ws.hitF[w], 1u << b);
-      ++lc.f;
-    } else {
-      atomicOr(&ws.hitS[w], 1u << b);
-      c.tsrc[src_base + rev_n(pos0 + pos, nrev)] = val;
-      if ((uint32_t)(val >> 32) == k) ++lc.s; else ++lc.t;
+  const uint32_t total = batch_begin(ws, cand);
+  for (uint32_t base = 0; base < total; base += 32 * kB) {
+    uint64_t ch[kB];
+    uint32_t iw[kB], ib[kB], slot[kB];
+    unsigned long long val[kB];
+#pragma unroll
+    for (int t = 0; t < kB; ++t) {
+      const uint32_t j = base + 32 * t + lane;
+      ch[t] = ~0ull;
+      if (j < total) {
+        batch_item(ws, j, iw[t], ib[t]);
+        ch[t] = chunk0 + iw[t] * 32 + ib[t];
+      }
     }
-  });
+#pragma unroll
+    for (int t = 0; t < kB; ++t)
+      if (ch[t] != ~0ull) slot[t] = __ldg(p.slot_of + ch[t]);
+#pragma unroll
+    for (int t = 0; t < kB; ++t)
+      if (ch[t] != ~0ull) val[t] = __ldcg(&p.tab[slot[t]].val);
+#pragma unroll
+    for (int t = 0; t < kB; ++t) {
+      if (ch[t] == ~0ull) continue;
+      const uint32_t pos = iw[t] * 32 + ib[t];
+      if (val[t] == pack_entry(k, node_of_chunk(p.g, ch[t]))) {
+        atomicOr(&ws.hitF[iw[t]], 1u << ib[t]);
+        ++lc.f;
+      } else {
+        atomicOr(&ws.hitS[iw[t]], 1u << ib[t]);
+        c.tsrc[src_base + rev_n(pos0 + pos, nrev)] = val[t];
+        if ((uint32_t)(val[t] >> 32) == k) ++lc.s; else ++lc.t;
+      }
+    }
+  }
+  __syncwarp();
   F = ws.hitF[lane];
   S = ws.hitS[lane];
   X = valid & ~cand;
@@ -315,6 +369,20 @@ __device__ __forceinline__ bool insert_new(Slot* tab, uint64_t cap, const Digest
       return true;
     }
     if (olo == d.lo && ohi == d.hi) return false;   // already recorded: a collision (R14)
+    if (++s == cap) s = 0;
+  }
+}
+
+__device__ __forceinline__ bool insert_new_from(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed,
+                                                uint64_t s) {
+  for (;;) {
+    unsigned long long olo, ohi;
+    cas128(tab + s, kEmpty, kEmpty, d.lo, d.hi, olo, ohi);
+    if (olo == kEmpty && ohi == kEmpty) {
+      tab[s].val = packed;
+      return true;
+    }
+    if (olo == d.lo && ohi == d.hi) return false;
     if (++s == cap) s = 0;
   }
 }
@@ -416,39 +484,20 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     }
     lX1 = leafm1 & ~(lF1 | lS1);
   } else {
-    // 32 positions per lane (natural order): dirty marks and labels as vector loads
+    // the children ORed their root labels into this group's masks (bit-reversed order);
+    // positions with no bit are FIXED (clean children)
     const StageParams& sp = p.st[c.s];
-    const uint64_t j0 = (c.G << gsz) + (uint64_t)lane * 32;
-    const uint8_t* labs = PHASE == 2 ? sp.in.lab2 : sp.in.lab3;
-    uint32_t nF = 0, nS = 0, nX = 0;
-    if (P0 >= 32) {
-      if ((uint64_t)lane * 32 < P0) {
-        uint4 dv[8], lv2[2];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) dv[i] = __ldcg(reinterpret_cast<const uint4*>(sp.dirty_in + j0) + i);
-#pragma unroll
-        for (int i = 0; i < 2; ++i) lv2[i] = __ldcg(reinterpret_cast<const uint4*>(labs + j0) + i);
-        const uint32_t* dw = reinterpret_cast<const uint32_t*>(dv);
-        const uint8_t* lb = reinterpret_cast<const uint8_t*>(lv2);
-#pragma unroll
-        for (int b = 0; b < 32; ++b) {
-          const uint8_t L = (dw[b] == g.epoch) ? lb[b] : (uint8_t)L_FIXED;
-          nF |= (uint32_t)(L == L_FIRST) << b;
-          nS |= (uint32_t)(L == L_SHIFT) << b;
-          nX |= (uint32_t)(L == L_FIXED) << b;
-        }
-      }
+    if (PHASE == 2) {
+      F = __ldcg(sp.gm2 + c.G * 32 + lane);
+      S = 0;
+      X = valid_word(P0) & ~F;
     } else {
-      // fewer than 32 positions: lane b loads position b, ballots build lane 0's words
-      const uint64_t jb = (c.G << gsz) + lane;
-      uint8_t L = L_ABSENT;
-      if ((uint64_t)lane < P0) L = (__ldcg(sp.dirty_in + jb) == g.epoch) ? __ldcg(labs + jb) : (uint8_t)L_FIXED;
-      const uint32_t bf = __ballot_sync(0xffffffffu, L == L_FIRST);
-      const uint32_t bs = __ballot_sync(0xffffffffu, L == L_SHIFT);
-      const uint32_t bx = __ballot_sync(0xffffffffu, L == L_FIXED);
-      if (lane == 0) { nF = bf; nS = bs; nX = bx; }
+      const uint32_t* gm = sp.gm3 + c.G * 96;
+      F = __ldcg(gm + lane);
+      S = __ldcg(gm + 32 + lane);
+      const uint32_t D = __ldcg(gm + 64 + lane);
+      X = valid_word(P0) & ~(F | S | D);
     }
-    to_rev3(ws, gsz, nF, nS, nX, F, S, X);
   }
   __syncwarp();
   if (p.trace && lane == 0) ws.tp[0] = gtimer();
@@ -456,7 +505,7 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
   // ---- pass 1: digests bottom-up, no record traffic (see file header)
   ws.W[lane] = 0;
   __syncwarp();
-  {
+  if (__any_sync(0xffffffffu, ((PHASE == 2 ? F : S) | (PHASE == 2 ? lF1 : lS1)) != 0)) {
     uint32_t P = PHASE == 2 ? F : S;
     for (int lv = 1; lv <= gsz; ++lv) {
       const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
@@ -498,25 +547,76 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
   // ---- pass 2: record operations for all pass-1 nodes at once
   ws.H[lane] = 0;
   __syncwarp();
-  for_each_bit_balanced(ws, ws.W[lane], [&](uint32_t w, uint32_t b, uint32_t) {
-    int lv;
-    uint32_t r;
-    lay_decode(w, b, lv, r);
-    const Digest d = dig_load(ws, c.tdig, ws.WP[w] + __popc(ws.W[w] & ((1u << b) - 1u)));
-    if (PHASE == 2) {
-      // Alg.1 l.29: Map[Tree(node)] <- (node, chkptID)
-      const uint64_t gpos = (c.G << (gsz - lv)) + rev_n(r, gsz - lv);
-      if (insert_new(p.tab, p.cap, d, pack_entry(g.k, node_id(g, c.Lin + lv, gpos)))) ++ins_cnt;
-      else ++coll_cnt;   // R14: a FIRST-FIRST digest already in the record = 128-bit collision
-    } else {
-      // Alg.1 l.39: Tree(node) in Map ?
-      const unsigned long long v = table_lookup(p.tab, p.cap, d);
-      if (v != kEmpty) {
-        atomicOr(&ws.H[w], 1u << b);
-        c.tsrc[P0 + lvl_off(P0, lv) + r] = v;
+  {
+    constexpr int kB2 = 2;
+    const uint32_t total = batch_begin(ws, ws.W[lane]);
+    for (uint32_t base = 0; base < total; base += 32 * kB2) {
+      uint32_t iw[kB2], ib[kB2];
+      int lvs[kB2];
+      uint32_t rs[kB2];
+      Digest d[kB2];
+      uint64_t sl[kB2];
+      unsigned long long olo[kB2], ohi[kB2], oval[kB2];
+      bool has[kB2];
+#pragma unroll
+      for (int t = 0; t < kB2; ++t) {
+        const uint32_t j = base + 32 * t + lane;
+        has[t] = j < total;
+        if (has[t]) {
+          batch_item(ws, j, iw[t], ib[t]);
+          lay_decode(iw[t], ib[t], lvs[t], rs[t]);
+          d[t] = dig_load(ws, c.tdig, ws.WP[iw[t]] + __popc(ws.W[iw[t]] & ((1u << ib[t]) - 1u)));
+          sl[t] = slot_home(d[t].lo, p.cap);
+        }
+      }
+      // first probe of every item in flight at once
+#pragma unroll
+      for (int t = 0; t < kB2; ++t) {
+        if (!has[t]) continue;
+        if (PHASE == 2) {
+          cas128(p.tab + sl[t], kEmpty, kEmpty, d[t].lo, d[t].hi, olo[t], ohi[t]);   // Alg.1 l.29 (new key)
+        } else {
+          const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p.tab + sl[t]));  // Alg.1 l.39
+          olo[t] = kv.x;
+          ohi[t] = kv.y;
+          oval[t] = __ldcg(&p.tab[sl[t]].val);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < kB2; ++t) {
+        if (!has[t]) continue;
+        const int lv = lvs[t];
+        const uint32_t r = rs[t];
+        if (PHASE == 2) {
+          const uint64_t gpos = (c.G << (gsz - lv)) + rev_n(r, gsz - lv);
+          const unsigned long long packed = pack_entry(g.k, node_id(g, c.Lin + lv, gpos));
+          bool ok;
+          if (olo[t] == kEmpty && ohi[t] == kEmpty) {
+            p.tab[sl[t]].val = packed;
+            ok = true;
+          } else if (olo[t] == d[t].lo && ohi[t] == d[t].hi) {
+            ok = false;
+          } else {
+            uint64_t s2 = sl[t] + 1 == p.cap ? 0 : sl[t] + 1;
+            (void)s2;
+            ok = insert_new_from(p.tab, p.cap, d[t], packed, s2);
+          }
+          if (ok) ++ins_cnt;
+          else ++coll_cnt;   // R14: a FIRST-FIRST digest already in the record = 128-bit collision
+        } else {
+          unsigned long long v;
+          if (olo[t] == d[t].lo && ohi[t] == d[t].hi) v = oval[t];
+          else if (olo[t] == kEmpty && ohi[t] == kEmpty) v = kEmpty;
+          else v = table_lookup_from(p.tab, p.cap, d[t], sl[t] + 1 == p.cap ? 0 : sl[t] + 1);
+          if (v != kEmpty) {
+            atomicOr(&ws.H[iw[t]], 1u << ib[t]);
+            c.tsrc[P0 + lvl_off(P0, lv) + r] = v;
+          }
+        }
       }
     }
-  });
+    __syncwarp();
+  }
   if (p.trace && lane == 0) ws.tp[2] = gtimer();
 
   if (PHASE == 2) {
@@ -581,19 +681,23 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
       emit_region(c, ws, gsz, 0, rF != 0, rS ? child_src(c, gsz, 0) : 0ull);   // R10
   } else if (lane == 0) {
     const StageParams& nx = p.st[c.s + 1];
+    const uint32_t qn = (uint32_t)(c.G & ((1ull << nx.gsz) - 1));   // natural position in the parent group
+    const uint32_t rr = rev_n(qn, nx.gsz);
+    const uint64_t Pg = c.G >> nx.gsz;
     if (PHASE == 2) {
-      nx.in.lab2[c.G] = rF ? L_FIRST : L_FIXED;
       if (rF) {
         const Digest d = child_digest(c, ws, gsz, 0);
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
+        atomicOr(nx.gm2 + Pg * 32 + (rr >> 5), 1u << (rr & 31));
       }
     } else {
-      nx.in.lab3[c.G] = rF ? L_FIRST : (rS ? L_SHIFT : (rX ? L_FIXED : L_DONE));
       if (rS) {
         const Digest d = child_digest(c, ws, gsz, 0);
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
         nx.in.src[c.G] = child_src(c, gsz, 0);
       }
+      const int which = rF ? 0 : (rS ? 1 : (rX ? -1 : 2));
+      if (which >= 0) atomicOr(nx.gm3 + Pg * 96 + which * 32 + (rr >> 5), 1u << (rr & 31));
     }
   }
   __syncwarp();
@@ -663,7 +767,7 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
 
 // ================================================================= kernel
 template <int PHASE>
-__global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constant__ TreeParams p) {
+__global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_constant__ TreeParams p) {
   extern __shared__ __align__(16) uint8_t tree_smem[];
   WarpSmem* sm = reinterpret_cast<WarpSmem*>(tree_smem);
   __shared__ unsigned long long s_cnt[4];
@@ -701,8 +805,10 @@ __global__ void __launch_bounds__(kTreeThreads) tree_kernel(const __grid_constan
       process_group<PHASE>(c, ws, ins, coll, lc);
       if (PHASE == 2 && lane == 0) up.dirty[P] = p.g.epoch;
       if (p.trace && lane == 0) {
-        const uint32_t i = atomicAdd(p.trace_n, 1u);
+        const uint32_t i = atomicAdd(p.trace_n, 3u);
         p.trace[i] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
+        p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 40 + PHASE);
+        p.trace[i + 2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 50 + PHASE);
       }
     }
   };

@@ -90,6 +90,8 @@ struct StageParams {
   uint32_t* arr2;              // s >= 1: arrivals of dirty children, phase 2
   uint32_t* arr3;              //                                     phase 3
   const uint32_t* dcnt;        // s >= 1: dirty children per group (K1b)
+  uint32_t* gm2;               // s >= 1: per group, 32 words: FIRST children (bit-reversed), phase 2
+  uint32_t* gm3;               // s >= 1: per group, 96 words: FIRST / SHIFT / DONE children, phase 3
 };
 
 struct TreeParams {
