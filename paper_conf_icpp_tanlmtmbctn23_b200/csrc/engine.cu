@@ -348,7 +348,9 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
     return CKPT_ECUDA;
   }
   h->encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-  if (leaf_setup_attributes() != cudaSuccess || tree_setup_attributes() != cudaSuccess) {
+  if (leaf_setup_attributes() != cudaSuccess || tree_setup_attributes() != cudaSuccess ||
+      preload_leaf() != cudaSuccess || preload_tree() != cudaSuccess || preload_compact() != cudaSuccess ||
+      preload_restore() != cudaSuccess) {
     delete h;
     return CKPT_ECUDA;
   }

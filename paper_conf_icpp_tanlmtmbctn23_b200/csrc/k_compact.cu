@@ -292,4 +292,17 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
   return e;
 }
 
+
+// Load this file's kernels now (CUDA lazy module loading would otherwise stall the first
+// launch of each kernel inside the first checkpoint).
+cudaError_t preload_compact() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, offsets_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gather_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, data_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_kernel);
+  return e;
+}
+
 }  // namespace ckpt

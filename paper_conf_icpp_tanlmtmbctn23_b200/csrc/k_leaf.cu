@@ -467,4 +467,18 @@ cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, 
   return cudaGetLastError();
 }
 
+
+// Load this file's kernels now (CUDA lazy module loading would otherwise stall the first
+// launch of each kernel inside the first checkpoint).
+cudaError_t preload_leaf() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<1>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_tail_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, insert_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, rehash_kernel);
+  return e;
+}
+
 }  // namespace ckpt

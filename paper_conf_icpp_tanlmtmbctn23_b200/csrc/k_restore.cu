@@ -206,4 +206,19 @@ cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff*
   return cudaGetLastError();
 }
 
+
+// Load this file's kernels now (CUDA lazy module loading would otherwise stall the first
+// launch of each kernel inside the first checkpoint).
+cudaError_t preload_restore() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_block_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_add_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_first_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_stream_kernel<true>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_stream_kernel<false>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_shift_kernel);
+  return e;
+}
+
 }  // namespace ckpt

@@ -886,4 +886,15 @@ cudaError_t tree_setup_attributes() {
 
 size_t tree_lmask_words() { return kLmWords; }
 
+
+// Load this file's kernels now (CUDA lazy module loading would otherwise stall the first
+// launch of each kernel inside the first checkpoint).
+cudaError_t preload_tree() {
+  cudaFuncAttributes a;
+  cudaError_t e = cudaSuccess;
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, tree_kernel<2>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, tree_kernel<3>);
+  return e;
+}
+
 }  // namespace ckpt

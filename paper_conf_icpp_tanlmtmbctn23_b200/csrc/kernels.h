@@ -153,6 +153,10 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned 
 // ---- launchers (return cudaGetLastError())
 cudaError_t leaf_setup_attributes();
 cudaError_t tree_setup_attributes();
+cudaError_t preload_leaf();
+cudaError_t preload_tree();
+cudaError_t preload_compact();
+cudaError_t preload_restore();
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
 cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st);

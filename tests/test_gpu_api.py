@@ -115,3 +115,23 @@ def test_full_size_config2_properties(oracle_mod):
         ck.restore(k, out)
         assert torch.equal(out, bufs[k]), k
     ck.close()
+
+
+def test_phase_times_ring():
+    """ckpt_phase_times_of: per-checkpoint device phase times (CUDA events), queried after
+    the calls; the per-phase times add up to at most the whole-call time."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer, CkptError
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    ck = Checkpointer(128)
+    ck.set_profiling(True)
+    bufs = list(W.lineage(2, 1 << 24, 128, 4, p=0.01))
+    for b in bufs:
+        ck.checkpoint(torch.from_numpy(b).cuda(), nbytes=b.size)
+    for k in range(len(bufs)):
+        t = ck.phase_times(k)
+        parts = sum(t[x] for x in ("leaf_hash", "insert", "phase2", "phase3", "compact"))
+        assert all(t[x] >= 0 for x in t)
+        assert 0 < parts <= t["total"] * 1.001 + 1e-3, (k, t)
+    with pytest.raises(CkptError):
+        ck.phase_times(len(bufs))
+    ck.close()

@@ -146,3 +146,16 @@ def test_determinism_two_runs():
         outs.append([ck.diff_to_host(k) for k in range(len(bufs))])
         ck.close()
     assert outs[0] == outs[1]
+
+
+@pytest.mark.parametrize("dbg", [128, 256, 384])
+def test_alternate_engine_modes(oracle_mod, monkeypatch, dbg):
+    """Engine variants selected by CKPT_DBG at ckpt_create must stay bit-exact:
+    128 = record inserts issued by K1's insert warp instead of the K1b pass,
+    256 = record table sized to half the leaves (long probe chains, frequent growth)."""
+    monkeypatch.setenv("CKPT_DBG", str(dbg))
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    bufs = list(W.lineage(2, (1 << 23) + 48, 128, 5, p=0.05))
+    run_parity(oracle_mod, bufs, 128)
+    bufs = dup_lineage(77, 5000 * 64 - 7, 64, K=4, alphabet=5)
+    run_parity(oracle_mod, bufs, 64)
