@@ -66,8 +66,11 @@ struct ckpt_ctx {
   uint32_t* gm3[kMaxStages] = {};
   uint32_t* wl0 = nullptr;
   uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
-  uint8_t* ctr = nullptr;        // Totals + per-stage counters, zeroed by one memset per call
+  // Totals + per-stage counters, double-buffered: call k uses ctr2[k & 1] and its last
+  // kernel zeroes ctr2[(k + 1) & 1] for the next call, so no memset precedes K1.
+  uint8_t* ctr2[2] = {};
   size_t ctr_bytes = 0;
+  size_t ctr_dbits_off = 0, ctr_bsum_off = 0, ctr_stage_off[kMaxStages] = {};
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
@@ -77,7 +80,7 @@ struct ckpt_ctx {
   ulonglong2* big = nullptr;
   unsigned long long* big_len = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
-  Totals* tot_host = nullptr;   // pinned
+  Totals* tot_host = nullptr;   // pinned + mapped: written by the offsets kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
   DiffArena arena;
@@ -192,18 +195,14 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
       off[s] = bytes;
       bytes += (3 + 128) * h->ngroups[s] * sizeof(uint32_t);
     }
-    AL(h->ctr, bytes);
+    AL(h->ctr2[0], bytes);
+    AL(h->ctr2[1], bytes);
+    if (cudaMemset(h->ctr2[0], 0, bytes) != cudaSuccess || cudaMemset(h->ctr2[1], 0, bytes) != cudaSuccess)
+      return CKPT_ECUDA;
     h->ctr_bytes = bytes;
-    h->tot = reinterpret_cast<Totals*>(h->ctr);
-    h->dbits = reinterpret_cast<uint32_t*>(h->ctr + dbits_off);
-    h->blocksum = reinterpret_cast<unsigned long long*>(h->ctr + bsum_off);
-    for (int s = 1; s < h->S; ++s) {
-      h->arr2[s] = reinterpret_cast<uint32_t*>(h->ctr + off[s]);
-      h->arr3[s] = h->arr2[s] + h->ngroups[s];
-      h->dcnt[s] = h->arr3[s] + h->ngroups[s];
-      h->gm2[s] = h->dcnt[s] + h->ngroups[s];
-      h->gm3[s] = h->gm2[s] + 32 * h->ngroups[s];
-    }
+    h->ctr_dbits_off = dbits_off;
+    h->ctr_bsum_off = bsum_off;
+    for (int s = 1; s < h->S; ++s) h->ctr_stage_off[s] = off[s];
   }
   AL(h->scratch, n_tiles << h->t0);
   AL(h->tilecnt, n_tiles);
@@ -359,7 +358,7 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
     return CKPT_ECUDA;
   }
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  if (cudaMallocHost(&h->tot_host, sizeof(Totals)) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  if (cudaHostAlloc(&h->tot_host, sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
     h->ev_id[r] = -1;
     for (int i = 0; i < 6; ++i) cudaEventCreate(&h->evr[r][i]);
@@ -423,6 +422,21 @@ int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   return ckpt_phase_times_of(h, (uint32_t)(h->diffs.size() - 1), times, n);
 }
 
+// Point the per-call counter views at ctr2[parity].
+static void select_ctr(ckpt_ctx* h, int parity) {
+  uint8_t* c = h->ctr2[parity];
+  h->tot = reinterpret_cast<Totals*>(c);
+  h->dbits = reinterpret_cast<uint32_t*>(c + h->ctr_dbits_off);
+  h->blocksum = reinterpret_cast<unsigned long long*>(c + h->ctr_bsum_off);
+  for (int s = 1; s < h->S; ++s) {
+    h->arr2[s] = reinterpret_cast<uint32_t*>(c + h->ctr_stage_off[s]);
+    h->arr3[s] = h->arr2[s] + h->ngroups[s];
+    h->dcnt[s] = h->arr3[s] + h->ngroups[s];
+    h->gm2[s] = h->dcnt[s] + h->ngroups[s];
+    h->gm3[s] = h->gm2[s] + 32 * h->ngroups[s];
+  }
+}
+
 int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
   using clk = std::chrono::steady_clock;
   const auto t_entry = clk::now();
@@ -451,6 +465,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   const Geo g = make_geo(h, k);
   const uint8_t* buf = static_cast<const uint8_t*>(dev_ptr);
+  select_ctr(h, (int)(k & 1));
 
   // ---- record-insert state (K1's insert warp and K1b)
   InsertParams ip;
@@ -506,7 +521,6 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   h->ev = h->evr[k % ckpt_ctx::kEvRing];
   h->ev_id[k % ckpt_ctx::kEvRing] = h->prof ? (int64_t)k : -1;
   const auto t_pre = clk::now();
-  CK(cudaMemsetAsync(h->ctr, 0, h->ctr_bytes, st));
   if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
@@ -560,14 +574,16 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.big = h->big; cp.big_len = h->big_len;
   cp.out = out; cp.buf = buf;
   cp.trace = h->trace; cp.trace_n = h->trace_n;
+  cp.tot_host = h->tot_host;
+  cp.ctr_next = reinterpret_cast<uint4*>(h->ctr2[(k + 1) & 1]);
+  cp.ctr_next_words = h->ctr_bytes / 16;
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
-  CK(cudaMemcpyAsync(h->tot_host, h->tot, sizeof(Totals), cudaMemcpyDeviceToHost, st));
   const auto t_launched = clk::now();
   CK(cudaStreamSynchronize(st));   // the one host synchronisation of the call
   const auto t_synced = clk::now();
 
-  const Totals t = *h->tot_host;
+  const Totals t = *h->tot_host;   // written by the offsets kernel (mapped host memory)
   if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
     uint32_t nt = 0, ne = 0;
     cudaMemcpy(&nt, h->trace_n, 4, cudaMemcpyDeviceToHost);

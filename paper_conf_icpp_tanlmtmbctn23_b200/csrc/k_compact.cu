@@ -128,6 +128,8 @@ __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
     *reinterpret_cast<uint32_t*>(o + 56) = 0;            // hash seed
     *reinterpret_cast<uint32_t*>(o + 60) = 0;            // reserved
     for (unsigned long long x = raw; x < meta; ++x) o[x] = 0;
+    // every counter the host reports is final here (tree kernels done, pdl_wait above)
+    *p.tot_host = *p.tot;
   }
 }
 
@@ -262,6 +264,9 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
 // KD: first-occurrence regions above kBig bytes (e.g. a fully new checkpoint is one
 // region), each spread over the whole grid with coalesced 16-byte units.
 __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
+  // the next call's counters (not touched by this call's kernels)
+  for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < p.ctr_next_words; i += (uint64_t)gridDim.x * kCT)
+    p.ctr_next[i] = make_uint4(0, 0, 0, 0);
   pdl_wait();
   const uint32_t nbig = *(volatile uint32_t*)&p.tot->big_count;
   if (nbig == 0) return;

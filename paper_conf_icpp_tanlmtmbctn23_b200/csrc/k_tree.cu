@@ -357,22 +357,6 @@ __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint6
   X = valid & ~cand;
 }
 
-// Phase-2 record insert of a FIRST-FIRST node (Alg.1 l.29): the key is new, so the CAS
-// claim of an empty slot settles it; the value is then written plainly.
-__device__ __forceinline__ bool insert_new(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed) {
-  uint64_t s = slot_home(d.lo, cap);
-  for (;;) {
-    unsigned long long olo, ohi;
-    cas128(tab + s, kEmpty, kEmpty, d.lo, d.hi, olo, ohi);
-    if (olo == kEmpty && ohi == kEmpty) {
-      tab[s].val = packed;
-      return true;
-    }
-    if (olo == d.lo && ohi == d.hi) return false;   // already recorded: a collision (R14)
-    if (++s == cap) s = 0;
-  }
-}
-
 __device__ __forceinline__ bool insert_new_from(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed,
                                                 uint64_t s) {
   for (;;) {

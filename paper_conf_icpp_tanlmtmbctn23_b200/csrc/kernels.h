@@ -130,6 +130,9 @@ struct CompactParams {
   const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
   ulonglong4* trace;             // diagnostics (CKPT_TRACE)
   uint32_t* trace_n;
+  Totals* tot_host;              // mapped pinned host copy of the final totals (no D2H op)
+  uint4* ctr_next;               // the next call's counter block, zeroed by the data kernel
+  uint64_t ctr_next_words;
 };
 
 // Launch with programmatic stream serialization (PDL): the kernel may be scheduled while
