@@ -129,17 +129,25 @@ CKPT_API int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_
                      uint64_t cap, uint64_t* count);
 
 /* Per-phase device times (ms) of the latest ckpt_checkpoint, measured with CUDA events on
- * the caller's stream when profiling is enabled (ckpt_set_profiling(h, 1)).
+ * the caller's stream when profiling is enabled: ckpt_set_profiling(h, level), level 0 = off,
+ * 1 = events around K1 and the whole call only (an event between two kernels stops the
+ * second from launching early, so level 1 is the one to time under), 2 = every phase.
  * times[0] leaf hash pass (K1), [1] record insert (K1b), [2] phase 2 (all stages),
  * [3] phase 3 (all stages), [4] compaction (offsets + gather), [5] whole call (first
- * kernel to last kernel); host wall times of the same call (always recorded): [6] entry
- * to first enqueue, [7] enqueue of the kernel sequence, [8] wait in the one stream
- * synchronisation, [9] bookkeeping after it.  n <= 10 values are written. */
+ * kernel to last kernel; [1]..[4] are 0 at level 1); host wall times of the same call
+ * (always recorded): [6] entry to first enqueue, [7] enqueue of the kernel sequence, [8]
+ * wait in the one stream synchronisation, [9] bookkeeping after it.  n <= 10 values are
+ * written.  ckpt_set_profiling errors: CKPT_EINVAL (level outside 0..2). */
 CKPT_API int ckpt_set_profiling(ckpt_handle h, int enable);
 CKPT_API int ckpt_phase_times(ckpt_handle h, float* times, int n);
 /* Same for checkpoint `id` (device times kept for the latest 256 profiled checkpoints; the
  * event queries happen here, never inside ckpt_checkpoint). Errors: CKPT_ERANGE. */
 CKPT_API int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n);
+
+/* Number of kernels this handle has enqueued so far (ckpt_checkpoint, ckpt_restore and the
+ * calls built on them), counted at the launch sites; bench.py reports the difference over
+ * its timed region. */
+CKPT_API int ckpt_kernel_launches(ckpt_handle h, uint64_t* count);
 
 /* Release all device memory of the handle (record, leaf digests, every diff). */
 CKPT_API int ckpt_destroy(ckpt_handle h);

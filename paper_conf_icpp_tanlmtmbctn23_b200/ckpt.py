@@ -21,7 +21,8 @@ CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_EC
 ABI_FUNCTIONS = [
     "ckpt_create", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
     "ckpt_checkpoint_host", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
-    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_destroy", "ckpt_strerror",
+    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
+    "ckpt_strerror",
 ]
 
 
@@ -83,6 +84,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_set_profiling": ([vp, i32], i32),
             "ckpt_phase_times": ([vp, P(ctypes.c_float), i32], i32),
             "ckpt_phase_times_of": ([vp, u32, P(ctypes.c_float), i32], i32),
+            "ckpt_kernel_launches": ([vp, P(ctypes.c_uint64)], i32),
             "ckpt_destroy": ([vp], i32),
             "ckpt_strerror": ([i32], ctypes.c_char_p),
         }
@@ -217,8 +219,14 @@ class Checkpointer:
         k = cnt.value
         return {(keys[i].tobytes(), int(nodes[i]), int(ckpts[i])) for i in range(k)}
 
-    def set_profiling(self, on: bool = True) -> None:
-        lib().ckpt_set_profiling(self._h, 1 if on else 0)
+    def set_profiling(self, level: int | bool = 2) -> None:
+        """0/False off; 1 = CUDA events around K1 and the whole call only (keeps the
+        kernels' programmatic early launch, so this is the level to time under); 2/True =
+        events around every phase."""
+        level = 2 if level is True else (0 if level is False else int(level))
+        rc = lib().ckpt_set_profiling(self._h, level)
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_set_profiling")
 
     PHASES = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total",
               "host_pre", "host_enqueue", "host_sync_wait", "host_post"]
@@ -234,6 +242,13 @@ class Checkpointer:
             if rc != CKPT_OK:
                 raise CkptError(rc, "ckpt_phase_times_of")
         return {self.PHASES[i]: t[i] for i in range(10)}
+
+    @property
+    def kernel_launches(self) -> int:
+        """Kernels this handle has enqueued so far (counted at the library's launch sites)."""
+        c = ctypes.c_uint64()
+        lib().ckpt_kernel_launches(self._h, ctypes.byref(c))
+        return c.value
 
     def close(self) -> None:
         if getattr(self, "_h", None):

@@ -88,11 +88,13 @@ struct ckpt_ctx {
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
   cudaStream_t internal = nullptr;
-  bool prof = false;
+  uint64_t launches = 0;         // kernels this handle has enqueued (all calls)
+  int prof = 0;                  // 0 off, 1 K1 + whole call, 2 every phase
   // per-checkpoint event sets (ring), queried lazily so the call itself never waits on them
   static constexpr int kEvRing = 256;
   cudaEvent_t evr[kEvRing][6] = {};
   int64_t ev_id[kEvRing] = {};
+  int ev_level[kEvRing] = {};
   cudaEvent_t* ev = nullptr;     // event set of the current call
   float times[12] = {};          // host times of the latest call ([6..9])
   PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
@@ -390,9 +392,16 @@ int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count) {
   return CKPT_OK;
 }
 
+int ckpt_kernel_launches(ckpt_handle h, uint64_t* count) {
+  if (!h || !count) return CKPT_EINVAL;
+  *count = h->launches;
+  return CKPT_OK;
+}
+
 int ckpt_set_profiling(ckpt_handle h, int enable) {
   if (!h) return CKPT_EINVAL;
-  h->prof = enable != 0;
+  if (enable < 0 || enable > 2) return CKPT_EINVAL;
+  h->prof = enable;
   return CKPT_OK;
 }
 
@@ -403,7 +412,11 @@ int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
   float t[10] = {};
   if (h->ev_id[r] == (int64_t)id) {
     cudaEvent_t* e = h->evr[r];
-    for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], e[i], e[i + 1]);   // K1, K1b, phase 2, phase 3, compaction
+    if (h->ev_level[r] >= 2) {
+      for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], e[i], e[i + 1]);   // K1, K1b, phase 2, phase 3, compaction
+    } else {
+      cudaEventElapsedTime(&t[0], e[0], e[1]);   // K1 only
+    }
     cudaEventElapsedTime(&t[5], e[0], e[5]);
     cudaGetLastError();
   }
@@ -421,6 +434,14 @@ int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   }
   return ckpt_phase_times_of(h, (uint32_t)(h->diffs.size() - 1), times, n);
 }
+
+// Adds the kernels enqueued during one API call to the handle's launch counter.
+struct LaunchCount {
+  ckpt_ctx* h;
+  uint64_t start;
+  explicit LaunchCount(ckpt_ctx* hh) : h(hh), start(g_kernel_launches) {}
+  ~LaunchCount() { h->launches += g_kernel_launches - start; }
+};
 
 // Point the per-call counter views at ctr2[parity].
 static void select_ctr(ckpt_ctx* h, int parity) {
@@ -443,6 +464,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   auto ms_since = [](clk::time_point a, clk::time_point b) { return std::chrono::duration<float, std::milli>(b - a).count(); };
   if (!h) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  LaunchCount lc(h);
   if (!dev_ptr || !diff || bytes == 0 || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if ((bytes + h->C - 1) / h->C > (1ull << 31)) return CKPT_EINVAL;
   if (h->geo_set && bytes != h->B) return CKPT_EINVAL;   // R17
@@ -520,6 +542,10 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   h->ev = h->evr[k % ckpt_ctx::kEvRing];
   h->ev_id[k % ckpt_ctx::kEvRing] = h->prof ? (int64_t)k : -1;
+  h->ev_level[k % ckpt_ctx::kEvRing] = h->prof;
+  // an event between two kernels stops the second from launching early (PDL), so level 1
+  // keeps only the events around K1 (the first kernel) and at the end of the call
+  const bool pe = h->prof >= 2;
   const auto t_pre = clk::now();
   if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
@@ -529,7 +555,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   if (h->prof) CK(cudaEventRecord(h->ev[1], st));
   // K1b: record insert + tie-break (l.6-19), dirty tiles
   CK(launch_insert(ip, h->num_sms, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[2], st));
+  if (pe) CK(cudaEventRecord(h->ev[2], st));
 
   // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11
   TreeParams tp;
@@ -561,9 +587,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.gm3 = h->gm3[s];
   }
   CK(launch_tree(tp, 2, h->num_sms, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[3], st));
+  if (pe) CK(cudaEventRecord(h->ev[3], st));
   CK(launch_tree(tp, 3, h->num_sms, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[4], st));
+  if (pe) CK(cudaEventRecord(h->ev[4], st));
 
   // ---- compaction + serialisation
   CompactParams cp;
@@ -657,6 +683,7 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
   if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
   if (id >= h->diffs.size()) return CKPT_ERANGE;
+  LaunchCount lc(h);
   cudaStream_t st = h->internal;
   const Geo g = make_geo(h, id);
   uint64_t maxF = 1, maxS = 1;

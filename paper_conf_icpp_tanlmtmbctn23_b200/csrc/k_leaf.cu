@@ -434,6 +434,7 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   if (grid > n_tiles) grid = n_tiles;
   if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else leaf_hash_kernel<0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  note_launch();
   return cudaGetLastError();
 }
 
@@ -441,6 +442,7 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
   if (p.tail_begin >= p.g.n) return cudaSuccess;
   const uint64_t cnt = p.g.n - p.tail_begin;
   leaf_tail_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, st>>>(p);
+  note_launch();
   return cudaGetLastError();
 }
 
@@ -463,7 +465,10 @@ cudaError_t leaf_setup_attributes() {
 cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st) {
   uint64_t blocks = (old_cap + 255) / 256;
   if (blocks > 148 * 16) blocks = 148 * 16;
-  if (blocks) rehash_kernel<<<(unsigned)blocks, 256, 0, st>>>(old_tab, old_cap, new_tab, new_cap);
+  if (blocks) {
+    rehash_kernel<<<(unsigned)blocks, 256, 0, st>>>(old_tab, old_cap, new_tab, new_cap);
+    note_launch();
+  }
   return cudaGetLastError();
 }
 

@@ -167,6 +167,7 @@ cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long*
   const uint64_t nb = (count + kScanBlock - 1) / kScanBlock;
   if (nb == 1) {
     scan_block_kernel<<<1, kRT, 0, st>>>(in, out, count, nullptr);
+    note_launch();
     return cudaGetLastError();
   }
   unsigned long long* bsum = reinterpret_cast<unsigned long long*>(tmp);
@@ -174,9 +175,11 @@ cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long*
   const size_t used = 2 * nb * sizeof(unsigned long long);
   if (used > tmp_bytes) return cudaErrorInvalidValue;
   scan_block_kernel<<<(unsigned)nb, kRT, 0, st>>>(in, out, count, bsum);
+  note_launch();
   cudaError_t e = scan_u64_exclusive(bsum, boff, nb, boff + nb, tmp_bytes - used, st);
   if (e != cudaSuccess) return e;
   scan_add_kernel<<<(unsigned)((count + 255) / 256), 256, 0, st>>>(out, count, boff);
+  note_launch();
   return cudaGetLastError();
 }
 
@@ -184,6 +187,7 @@ cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long lo
                                   size_t scan_tmp_bytes, cudaStream_t st) {
   if (d.nF == 0) return cudaSuccess;
   prepare_first_kernel<<<(unsigned)((d.nF + 255) / 256), 256, 0, st>>>(g, d, tmp_len);
+  note_launch();
   return scan_u64_exclusive(tmp_len, d.Foff, d.nF, scan_tmp, scan_tmp_bytes, st);
 }
 
@@ -191,6 +195,7 @@ cudaError_t restore_copy_first(const Geo& g, const RestoreDiff& d, uint8_t* out,
   if (d.nF == 0) return cudaSuccess;
   copy_stream_kernel<true><<<num_sms * 8, kRT, 0, st>>>(g, d, out, d.Foff, nullptr, nullptr, nullptr, d.nF,
                                                        d.data_bytes);
+  note_launch();
   return cudaGetLastError();
 }
 
@@ -200,9 +205,11 @@ cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff*
                           cudaStream_t st) {
   if (d.nS == 0) return cudaSuccess;
   prepare_shift_kernel<<<(unsigned)((d.nS + 255) / 256), 256, 0, st>>>(g, d, chain_dev, t_len, t_src, t_dst, err);
+  note_launch();
   cudaError_t e = scan_u64_exclusive(t_len, t_off, d.nS, scan_tmp, scan_tmp_bytes, st);
   if (e != cudaSuccess) return e;
   copy_stream_kernel<false><<<num_sms * 8, kRT, 0, st>>>(g, d, out, t_off, t_len, t_src, t_dst, d.nS, 0);
+  note_launch();
   return cudaGetLastError();
 }
 

@@ -135,6 +135,11 @@ struct CompactParams {
   uint64_t ctr_next_words;
 };
 
+// Kernel launches issued by this thread (every launch site calls note_launch once per
+// kernel it enqueues); the engine adds the per-call difference to the handle's counter.
+inline thread_local uint64_t g_kernel_launches = 0;
+inline void note_launch() { ++g_kernel_launches; }
+
 // Launch with programmatic stream serialization (PDL): the kernel may be scheduled while
 // its predecessor drains; it must call pdl_wait() before touching the predecessor's output.
 template <typename... KArgs, typename... Args>
@@ -150,6 +155,7 @@ inline cudaError_t launch_pdl(void (*kernel)(KArgs...), unsigned grid, unsigned 
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  note_launch();
   return cudaLaunchKernelEx(&cfg, kernel, args...);
 }
 

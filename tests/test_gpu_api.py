@@ -134,4 +134,30 @@ def test_phase_times_ring():
         assert 0 < parts <= t["total"] * 1.001 + 1e-3, (k, t)
     with pytest.raises(CkptError):
         ck.phase_times(len(bufs))
+    ck.set_profiling(1)                # K1 + whole call only
+    b = W.cfg2_mutate(bufs[-1].copy(), len(bufs), W.seed_of(2), 0.01)
+    ck.checkpoint(torch.from_numpy(b).cuda(), nbytes=b.size)
+    t = ck.phase_times()
+    assert 0 < t["leaf_hash"] <= t["total"] and t["insert"] == t["phase2"] == t["phase3"] == t["compact"] == 0
+    with pytest.raises(CkptError):
+        ck.set_profiling(3)
+    ck.close()
+
+
+def test_kernel_launch_counter():
+    """ckpt_kernel_launches counts what the library enqueues: a steady checkpoint of a
+    2^23-chunk buffer is K1, K1b, phase 2, phase 3, offsets, gather, data = 7 kernels
+    (plus K1t only when B is not a multiple of 256 C)."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    ck = Checkpointer(128)
+    buf = torch.zeros(1 << 30, dtype=torch.uint8, device="cuda")
+    assert ck.kernel_launches == 0
+    ck.checkpoint(buf)
+    a = ck.kernel_launches
+    ck.checkpoint(buf)
+    assert ck.kernel_launches - a == 7
+    out = torch.empty_like(buf)
+    b = ck.kernel_launches
+    ck.restore(1, out)
+    assert ck.kernel_launches > b and torch.equal(out, buf)
     ck.close()
