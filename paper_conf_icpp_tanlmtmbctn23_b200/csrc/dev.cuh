@@ -128,6 +128,15 @@ __device__ __forceinline__ void chunk_range(const Geo& g, int L, uint64_t j, uin
   hi = chunk_of_vslot(g, (j + 1) << L);
 }
 
+// A stage-0 tree tile is FULL when every one of its leaves is a candidate (non-FIXED):
+// only then can its root be FIRST or SHIFT (Alg.1: a parent is FIRST / SHIFT only if
+// both children are). tcc = candidate leaves counted by K1/K1t.
+__device__ __forceinline__ bool tile_full(const Geo& g, const uint32_t* tcc, uint64_t T) {
+  uint64_t lo, hi;
+  chunk_range(g, g.t0, T, lo, hi);
+  return (uint64_t)__ldcg(tcc + T) == hi - lo;
+}
+
 __device__ __forceinline__ uint64_t range_bytes(const Geo& g, uint64_t lo, uint64_t hi) {
   uint64_t e = hi * (uint64_t)g.C;
   if (e > g.B) e = g.B;

@@ -55,7 +55,6 @@ struct ckpt_ctx {
   uint32_t* cand = nullptr;
   uint64_t nwords = 0;
   uint32_t* slot_of = nullptr;
-  uint32_t* dirty[kMaxStages] = {};
   LevelIO lvl[kMaxStages] = {};
   Digest* tdig[kMaxStages] = {};
   unsigned long long* tsrc[kMaxStages] = {};
@@ -66,11 +65,12 @@ struct ckpt_ctx {
   uint32_t* gm3[kMaxStages] = {};
   uint32_t* wl0 = nullptr;
   uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
+  uint32_t* tcc = nullptr;       // candidate leaves per stage-0 tree tile (inside ctr)
   // Totals + per-stage counters, double-buffered: call k uses ctr2[k & 1] and its last
   // kernel zeroes ctr2[(k + 1) & 1] for the next call, so no memset precedes K1.
   uint8_t* ctr2[2] = {};
   size_t ctr_bytes = 0;
-  size_t ctr_dbits_off = 0, ctr_bsum_off = 0, ctr_stage_off[kMaxStages] = {};
+  size_t ctr_dbits_off = 0, ctr_tcc_off = 0, ctr_bsum_off = 0, ctr_stage_off[kMaxStages] = {};
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
@@ -170,12 +170,8 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->cand, h->nwords + 32);
   AL(h->slot_of, n);
   for (int s = 0; s < h->S; ++s) {
-    AL(h->dirty[s], h->ngroups[s]);
-    if (cudaMemset(h->dirty[s], 0, h->ngroups[s] * 4) != cudaSuccess) return CKPT_ECUDA;
     if (s >= 1) {
       const uint64_t P = 1ull << (h->h - h->Lin[s]);
-      AL(h->lvl[s].lab2, P);
-      AL(h->lvl[s].lab3, P);
       AL(h->lvl[s].dig, P);
       AL(h->lvl[s].src, P);
     }
@@ -189,13 +185,16 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     const size_t dbits_off = bytes;
     bytes += ((n_tiles + 31) / 32) * sizeof(uint32_t);
     bytes = (bytes + 255) & ~size_t(255);
+    const size_t tcc_off = bytes;
+    bytes += n_tiles * sizeof(uint32_t);
+    bytes = (bytes + 255) & ~size_t(255);
     const size_t bsum_off = bytes;
     bytes += (3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3) * sizeof(unsigned long long);
     bytes = (bytes + 255) & ~size_t(255);
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
-      bytes += (3 + 128) * h->ngroups[s] * sizeof(uint32_t);
+      bytes += (3 + 32 + 64) * h->ngroups[s] * sizeof(uint32_t);   // arr2 arr3 dcnt, gm2, gm3
     }
     AL(h->ctr2[0], bytes);
     AL(h->ctr2[1], bytes);
@@ -203,6 +202,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
       return CKPT_ECUDA;
     h->ctr_bytes = bytes;
     h->ctr_dbits_off = dbits_off;
+    h->ctr_tcc_off = tcc_off;
     h->ctr_bsum_off = bsum_off;
     for (int s = 1; s < h->S; ++s) h->ctr_stage_off[s] = off[s];
   }
@@ -217,7 +217,8 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
   if (h->trace_path) {
-    if (dalloc(h, &h->trace, 24 * n_tiles + n / 16 + 64) != cudaSuccess || dalloc(h, &h->trace_n, 4) != cudaSuccess)
+    if (dalloc(h, &h->trace, (uint64_t)kTraceLanes * kTraceLaneCap) != cudaSuccess ||
+        dalloc(h, &h->trace_n, 8 * kTraceLanes) != cudaSuccess)
       return CKPT_ENOMEM;
   }
   bool reserved = false;
@@ -448,6 +449,7 @@ static void select_ctr(ckpt_ctx* h, int parity) {
   uint8_t* c = h->ctr2[parity];
   h->tot = reinterpret_cast<Totals*>(c);
   h->dbits = reinterpret_cast<uint32_t*>(c + h->ctr_dbits_off);
+  h->tcc = reinterpret_cast<uint32_t*>(c + h->ctr_tcc_off);
   h->blocksum = reinterpret_cast<unsigned long long*>(c + h->ctr_bsum_off);
   for (int s = 1; s < h->S; ++s) {
     h->arr2[s] = reinterpret_cast<uint32_t*>(c + h->ctr_stage_off[s]);
@@ -497,6 +499,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   ip.tot = h->tot;
   ip.defer = h->defer;
   ip.dbits = h->dbits;
+  ip.tcc = h->tcc;
   ip.n_tiles = h->ngroups[0];
   ip.wl0 = h->wl0;
   ip.S = h->S;
@@ -547,7 +550,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   // keeps only the events around K1 (the first kernel) and at the end of the call
   const bool pe = h->prof >= 2;
   const auto t_pre = clk::now();
-  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 16, st));
+  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 32 * kTraceLanes, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
   CK(launch_leaf_tail(lp, st));
@@ -564,6 +567,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.S = h->S;
   tp.n_tiles = h->ngroups[0];
   tp.wl0 = h->wl0;
+  tp.tcc = h->tcc;
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
@@ -575,11 +579,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     StageParams& sp = tp.st[s];
     sp.Lin = h->Lin[s];
     sp.gsz = h->gsz[s];
-    sp.dirty_in = s >= 1 ? h->dirty[s - 1] : nullptr;
     sp.in = s >= 1 ? h->lvl[s] : LevelIO{};
     sp.tdig = h->tdig[s];
     sp.tsrc = h->tsrc[s];
-    sp.dirty = h->dirty[s];
     sp.arr2 = h->arr2[s];
     sp.arr3 = h->arr3[s];
     sp.dcnt = h->dcnt[s];
@@ -611,15 +613,18 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   const Totals t = *h->tot_host;   // written by the offsets kernel (mapped host memory)
   if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
-    uint32_t nt = 0, ne = 0;
-    cudaMemcpy(&nt, h->trace_n, 4, cudaMemcpyDeviceToHost);
-    cudaMemcpy(&ne, h->trace_n + 1, 4, cudaMemcpyDeviceToHost);
-    (void)ne;
-    std::vector<ulonglong4> tr(nt);
-    cudaMemcpy(tr.data(), h->trace, nt * sizeof(ulonglong4), cudaMemcpyDeviceToHost);
+    std::vector<uint32_t> cnt(8 * kTraceLanes);
+    cudaMemcpy(cnt.data(), h->trace_n, cnt.size() * 4, cudaMemcpyDeviceToHost);
+    std::vector<ulonglong4> tr;
+    for (uint32_t l = 0; l < kTraceLanes; ++l) {
+      const uint32_t nl = std::min<uint32_t>(cnt[8 * l], kTraceLaneCap);
+      const size_t o = tr.size();
+      tr.resize(o + nl);
+      cudaMemcpy(tr.data() + o, h->trace + (size_t)l * kTraceLaneCap, nl * sizeof(ulonglong4), cudaMemcpyDeviceToHost);
+    }
     char path[512];
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
-    if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), nt, f); fclose(f); }
+    if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), f); fclose(f); }
   }
   h->live += t.n_first + t.p2_inserts;
   DiffRec rec;

@@ -37,32 +37,13 @@ __device__ __forceinline__ void block_sum3(unsigned long long& a, unsigned long 
 constexpr int kCT = 256;
 constexpr int kPer = kTilesPerBlock / kCT;
 
-__global__ void __launch_bounds__(kCT) reduce_kernel(CompactParams p) {
-  __shared__ unsigned long long sh[3 * (kCT / 32)];
-  pdl_launch_dependents();
-  pdl_wait();
-  unsigned long long a = 0, b = 0, c = 0;
-  const uint64_t t0 = (uint64_t)blockIdx.x * kTilesPerBlock + threadIdx.x * kPer;
-  for (int i = 0; i < kPer; ++i) {
-    const uint64_t T = t0 + i;
-    if (T < p.n_tiles) {
-      const uint4 v = p.tilecnt[T];
-      if (v.w == p.g.epoch) { a += v.x; b += v.y; c += v.z; }
-    }
-  }
-  block_sum3(a, b, c, sh);
-  if (threadIdx.x == 0) {
-    p.blocksum[3 * blockIdx.x] = a;
-    p.blocksum[3 * blockIdx.x + 1] = b;
-    p.blocksum[3 * blockIdx.x + 2] = c;
-  }
-}
-
 __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
   __shared__ unsigned long long sh[3 * (kCT / 32)];
   __shared__ unsigned long long wx[kCT / 32], wy[kCT / 32], wz[kCT / 32];
+  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   pdl_launch_dependents();
   pdl_wait();
+  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   // prefix of earlier blocks
   unsigned long long a = 0, b = 0, c = 0;
   for (uint32_t i = threadIdx.x; i < blockIdx.x; i += kCT) {
@@ -131,6 +112,7 @@ __global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
     // every counter the host reports is final here (tree kernels done, pdl_wait above)
     *p.tot_host = *p.tot;
   }
+  trace_block(p.trace, p.trace_n, bt0, bt1, 4);
 }
 
 // KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata entries
@@ -153,8 +135,10 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   GatherWarp& gw = gsm[wid];
   const Geo& g = p.g;
+  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   pdl_launch_dependents();
   pdl_wait();
+  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   const unsigned long long nF_tot = p.tot->nF;
   uint8_t* const ent_f = p.out + 64;
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
@@ -255,21 +239,27 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
     }
     if (p.trace && lane == 0) {
       asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg2));
-      const uint32_t i = atomicAdd(p.trace_n, 1u);
-      p.trace[i] = make_ulonglong4(tg0, tg1, tg2, 77);
+      if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 1)) *r = make_ulonglong4(tg0, tg1, tg2, 77);
     }
   }
+  __syncthreads();
+  trace_block(p.trace, p.trace_n, bt0, bt1, 5);
 }
 
 // KD: first-occurrence regions above kBig bytes (e.g. a fully new checkpoint is one
 // region), each spread over the whole grid with coalesced 16-byte units.
 __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
+  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   // the next call's counters (not touched by this call's kernels)
   for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < p.ctr_next_words; i += (uint64_t)gridDim.x * kCT)
     p.ctr_next[i] = make_uint4(0, 0, 0, 0);
   pdl_wait();
+  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   const uint32_t nbig = *(volatile uint32_t*)&p.tot->big_count;
-  if (nbig == 0) return;
+  if (nbig == 0) {
+    trace_block(p.trace, p.trace_n, bt0, bt1, 6);
+    return;
+  }
   uint8_t* const dat = p.out + p.tot->meta_bytes;
   const unsigned long long stride = (unsigned long long)gridDim.x * kCT * 16;
   for (uint32_t b = 0; b < nbig; ++b) {
@@ -283,6 +273,7 @@ __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
     if (blockIdx.x == 0 && threadIdx.x == 0)
       for (unsigned long long o = full; o < len; ++o) d[o] = s[o];
   }
+  trace_block(p.trace, p.trace_n, bt0, bt1, 6);
 }
 
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st) {
@@ -306,7 +297,6 @@ cudaError_t preload_compact() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, offsets_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gather_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, data_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, reduce_kernel);
   return e;
 }
 

@@ -91,12 +91,34 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
 
 // Mark the stage-0 tree tile(s) holding 256-chunk leaf tile `tile` dirty (fire-and-forget;
 // a tree tile marked without candidates is processed as all-FIXED, which is harmless).
-__device__ __forceinline__ void mark_tree_dirty(const InsertParams& p, uint32_t tile) {
+// bits [a, b) of a 256-bit word array
+__device__ __forceinline__ uint32_t popc_range(const uint32_t* w, uint32_t a, uint32_t b) {
+  uint32_t n = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const uint32_t lo = 32u * i, hi = lo + 32u;
+    const uint32_t x = a > lo ? a : lo, y = b < hi ? b : hi;
+    if (x < y) n += __popc(w[i] & (((y - lo) == 32 ? 0xFFFFFFFFu : ((1u << (y - lo)) - 1u)) & ~((1u << (x - lo)) - 1u)));
+  }
+  return n;
+}
+
+// A 256-chunk leaf tile with candidates: mark the stage-0 tree tile(s) it overlaps dirty and
+// add its candidates to their counts (a leaf tile can straddle two tree tiles where the
+// leaves sit at height 1, R3).
+__device__ __forceinline__ void mark_tree_dirty(const InsertParams& p, uint32_t tile, const uint32_t* w) {
   const uint64_t c0 = (uint64_t)tile * 256;
   uint64_t c1 = c0 + 255;
   if (c1 >= p.g.n) c1 = p.g.n - 1;
   const uint64_t t0 = vpos_of_chunk(p.g, c0) >> p.g.t0, t1 = vpos_of_chunk(p.g, c1) >> p.g.t0;
-  for (uint64_t t = t0; t <= t1; ++t) atomicOr(p.dbits + (t >> 5), 1u << (t & 31));
+  for (uint64_t t = t0; t <= t1; ++t) {
+    atomicOr(p.dbits + (t >> 5), 1u << (t & 31));
+    uint64_t lo, hi;
+    chunk_range(p.g, p.g.t0, t, lo, hi);
+    const uint64_t a = lo > c0 ? lo : c0, b = hi < c1 + 1 ? hi : c1 + 1;
+    const uint32_t cnt = a < b ? popc_range(w, (uint32_t)(a - c0), (uint32_t)(b - c0)) : 0u;
+    if (cnt) atomicAdd(p.tcc + t, cnt);
+  }
 }
 
 // Defer a tile's inserts to K1b as one entry (tile << 3 | round) per 32 candidates, so
@@ -135,6 +157,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
   uint64_t* const bars = reinterpret_cast<uint64_t*>(prevbuf + nst * kLeafThreads);
   K1Ring& ring = *reinterpret_cast<K1Ring*>(bars + 8);
 
+  const unsigned long long bt0 = p.ins.trace ? gtime_ns() : 0;
   const int tid = threadIdx.x;
   const uint32_t n_tiles = (uint32_t)(p.n_main / kLeafThreads);
   const int segs = p.segs;
@@ -241,7 +264,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
 #pragma unroll
         for (int i = 0; i < 8; ++i) { w[i] = ring.stage_words[ntile_done & 1][i]; any |= w[i]; pc += __popc(w[i]); }
         if (any) {
-          mark_tree_dirty(p.ins, tile);
+          mark_tree_dirty(p.ins, tile, w);
           const uint32_t t = ring.tail;
           if (p.insert_warp && t - ring.head < (uint32_t)kRing) {
 #pragma unroll
@@ -264,6 +287,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
     __threadfence_block();
     ring.done = 1;
   }
+  trace_block(p.ins.trace, p.ins.trace_n, bt0, bt0, 0);
 }
 
 // ------------------------------------------------------------------ K1t
@@ -302,13 +326,17 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
     }
     cand = leaf_is_candidate(p.g, d, pd);
   }
+  __shared__ uint32_t s_w[8];
   const unsigned mask = __ballot_sync(0xffffffffu, cand);
-  if ((threadIdx.x & 31) == 0 && c < p.g.n) p.cand[c >> 5] = mask;
+  if ((threadIdx.x & 31) == 0) {
+    s_w[threadIdx.x >> 5] = mask;
+    if (c < p.g.n) p.cand[c >> 5] = mask;
+  }
   if (cand) reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
   const int pc = __syncthreads_count(cand);
   if (pc && threadIdx.x == 0) {
     const uint32_t tile = (uint32_t)((p.tail_begin >> 8) + blockIdx.x);
-    mark_tree_dirty(p.ins, tile);
+    mark_tree_dirty(p.ins, tile, s_w);
     defer_tile(p.ins, tile, (uint32_t)pc);
   }
 }
@@ -357,30 +385,35 @@ __device__ void build_tree_work(const InsertParams& p) {
     for (int t = 1; t < s; ++t) nchild >>= p.gsz[t];
     const uint64_t ngroups = nchild >> p.gsz[s];
     const uint32_t per = 1u << p.gsz[s];
-    for (uint64_t G = tid; G < ngroups; G += blockDim.x) {
+    // FULL children per group, one warp per group: only a full child can have a FIRST or
+    // SHIFT root, so only full children climb to their parent in the tree kernels
+    for (uint64_t G = wid; G < ngroups; G += blockDim.x >> 5) {
       uint32_t cnt = 0;
       if (s == 1) {
-        const uint64_t b0 = G * per;
-        for (uint64_t b = b0; b < b0 + per;) {
-          if ((b & 31) == 0 && b + 32 <= b0 + per) { cnt += __popc(__ldcg(p.dbits + (b >> 5))); b += 32; }
-          else { cnt += (__ldcg(p.dbits + (b >> 5)) >> (b & 31)) & 1u; ++b; }
-        }
+        for (uint64_t T = G * per + lane; T < (G + 1) * per; T += 32) cnt += tile_full(p.g, p.tcc, T);
       } else {
-        for (uint64_t ch = G * per; ch < (G + 1) * per; ++ch) cnt += p.dcnt[s - 1][ch] != 0;
+        const uint32_t full = 1u << p.gsz[s - 1];
+        for (uint64_t ch = G * per + lane; ch < (G + 1) * per; ch += 32) cnt += __ldcg(p.dcnt[s - 1] + ch) == full;
       }
-      p.dcnt[s][G] = cnt;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+      if (lane == 0) p.dcnt[s][G] = cnt;
     }
     __syncthreads();
   }
 }
 
 __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
+  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   pdl_launch_dependents();
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   __shared__ uint32_t s_word[8][32], s_excl[8][32];
   pdl_wait();
+  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   if (blockIdx.x == 0) {
     build_tree_work(p);
+    __syncthreads();
+    trace_block(p.trace, p.trace_n, bt0, bt1, 11);
     return;
   }
   unsigned long long tk0 = 0;
@@ -400,12 +433,13 @@ __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
     if (p.trace) {
       asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t3));
       if (lane == 0) {
-        const uint32_t i = atomicAdd(p.trace_n, 1u);
-        p.trace[i] = make_ulonglong4(tk0, t1, t2, t3);
+        if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 1)) *r = make_ulonglong4(tk0, t1, t2, t3);
       }
     }
   }
   if (lane == 0 && ncand) atomicAdd(&p.tot->n_cand, ncand);
+  __syncthreads();
+  trace_block(p.trace, p.trace_n, bt0, bt1, 1);
 }
 
 // ------------------------------------------------------------------ rehash

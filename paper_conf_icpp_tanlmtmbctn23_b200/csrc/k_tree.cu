@@ -261,6 +261,7 @@ struct Ctx {
   bool leaf;         // stage 0
   Digest* tdig;      // this group's spilled digests (P0 entries)
   unsigned long long* tsrc;   // this group's sources (2 P0 entries, bit-reversed indices)
+  bool pub;          // the group published a FIRST/SHIFT root to its parent (needs a release)
 };
 
 // digest of the node at (lv, rev index r) of the current group: leaves / inputs from
@@ -403,7 +404,7 @@ __device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, 
 
 // Process one group through its gsz levels. PHASE 2 or 3.
 template <int PHASE>
-__device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt, unsigned long long& coll_cnt,
+__device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt, unsigned long long& coll_cnt,
                               LeafCount& lc) {
   const TreeParams& p = *c.p;
   const Geo& g = p.g;
@@ -468,24 +469,32 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     }
     lX1 = leafm1 & ~(lF1 | lS1);
   } else {
-    // the children ORed their root labels into this group's masks (bit-reversed order);
-    // positions with no bit are FIXED (clean children)
+    // the children ORed their FIRST / SHIFT root labels into this group's masks
+    // (bit-reversed order). Every other child is FIXED or DONE; the two behave alike from
+    // here up (neither is emitted, and a parent with a FIRST/SHIFT child and a FIXED or
+    // DONE child is DONE either way), so both are carried as X.
     const StageParams& sp = p.st[c.s];
     if (PHASE == 2) {
       F = __ldcg(sp.gm2 + c.G * 32 + lane);
       S = 0;
-      X = valid_word(P0) & ~F;
     } else {
-      const uint32_t* gm = sp.gm3 + c.G * 96;
+      const uint32_t* gm = sp.gm3 + c.G * 64;
       F = __ldcg(gm + lane);
       S = __ldcg(gm + 32 + lane);
-      const uint32_t D = __ldcg(gm + 64 + lane);
-      X = valid_word(P0) & ~(F | S | D);
     }
+    X = valid_word(P0) & ~(F | S);
   }
   __syncwarp();
   if (p.trace && lane == 0) ws.tp[0] = gtimer();
 
+  // An upper group none of whose children has a FIRST or SHIFT root (the steady state:
+  // updates are far smaller than a tile) hashes, inserts and emits nothing; its root is
+  // FIXED iff every child is, else DONE.
+  const bool trivial = !c.leaf && !__any_sync(0xffffffffu, (F | S) != 0);
+  if (trivial) {
+    const bool allX = __all_sync(0xffffffffu, X == valid_word(P0));
+    X = (lane == 0 && allX) ? 1u : 0u;
+  } else {
   // ---- pass 1: digests bottom-up, no record traffic (see file header)
   ws.W[lane] = 0;
   __syncwarp();
@@ -654,12 +663,13 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
     }
   }
 
+  }   // !trivial
   if (p.trace && lane == 0) ws.tp[3] = gtimer();
   // ---- group root (single position at level gsz: lane 0 bit 0)
   const uint32_t rF = __shfl_sync(0xffffffffu, F, 0) & 1u;
   const uint32_t rS = __shfl_sync(0xffffffffu, S, 0) & 1u;
-  const uint32_t rX = __shfl_sync(0xffffffffu, X, 0) & 1u;
   const bool last = (c.s == p.S - 1);
+  c.pub = !last && (rF || (PHASE == 3 && rS));
   if (last) {
     if (PHASE == 3 && lane == 0 && (rF | rS))
       emit_region(c, ws, gsz, 0, rF != 0, rS ? child_src(c, gsz, 0) : 0ull);   // R10
@@ -680,8 +690,7 @@ __device__ void process_group(const Ctx& c, WarpSmem& ws, unsigned long long& in
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
         nx.in.src[c.G] = child_src(c, gsz, 0);
       }
-      const int which = rF ? 0 : (rS ? 1 : (rX ? -1 : 2));
-      if (which >= 0) atomicOr(nx.gm3 + Pg * 96 + which * 32 + (rr >> 5), 1u << (rr & 31));
+      if (rF | rS) atomicOr(nx.gm3 + Pg * 64 + (rF ? 0 : 32) + (rr >> 5), 1u << (rr & 31));
     }
   }
   __syncwarp();
@@ -758,24 +767,33 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   LeafCount lc{0, 0, 0};
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   WarpSmem& ws = sm[wid];
+  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   pdl_launch_dependents();
   if (threadIdx.x < 4) s_cnt[threadIdx.x] = 0;
   __syncthreads();
   pdl_wait();
+  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   unsigned long long ins = 0, coll = 0;
 
-  // Climb from (stage s, group G) after it is finished: arrive at the parent; the warp of
-  // the last arrival processes the parent (phase 2: when any child was dirty; phase 3:
-  // the parent's dirty-children count was recorded by phase 2).
+  // Climb from (stage s, group G) after it is finished. Only a FULL group (every leaf below
+  // it a candidate) can have a FIRST or SHIFT root, and a parent has work only through
+  // such children, so only full groups arrive at their parent; the warp of the last full
+  // arrival (K1b counted them) processes the parent. In the steady state no tile is full
+  // and nothing climbs.
   auto climb = [&](Ctx& c) {
     while (c.s < p.S - 1) {
+      const bool full = c.s == 0 ? tile_full(p.g, p.tcc, c.G) : __ldcg(p.st[c.s].dcnt + c.G) == (1u << c.gsz);
+      if (!full) return;
       const StageParams& up = p.st[c.s + 1];
       const uint64_t P = c.G >> up.gsz;
+      const uint32_t target = __ldcg(up.dcnt + P);
       uint32_t old = 0;
-      __threadfence();
+      // release: only a group that published a root label / digest to the parent has
+      // writes the parent's processor reads (nothing else it wrote is read in this kernel)
+      if (c.pub) __threadfence();
       if (lane == 0) old = atomicAdd((PHASE == 2 ? up.arr2 : up.arr3) + P, 1u);
       old = __shfl_sync(0xffffffffu, old, 0);
-      if (old + 1 != __ldcg(up.dcnt + P)) return;   // not the last dirty child
+      if (old + 1 != target) return;   // not the last full child
       __threadfence();
       c.s += 1;
       c.G = P;
@@ -787,12 +805,12 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
       c.tsrc = up.tsrc + ((P << c.gsz) << 1);
       unsigned long long t0 = p.trace ? gtimer() : 0;
       process_group<PHASE>(c, ws, ins, coll, lc);
-      if (PHASE == 2 && lane == 0) up.dirty[P] = p.g.epoch;
       if (p.trace && lane == 0) {
-        const uint32_t i = atomicAdd(p.trace_n, 3u);
-        p.trace[i] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
-        p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 40 + PHASE);
-        p.trace[i + 2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 50 + PHASE);
+        if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 3)) {
+          r[0] = make_ulonglong4(t0, gtimer(), ((unsigned long long)c.s << 32) | c.G, PHASE);
+          r[1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 40 + PHASE);
+          r[2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 50 + PHASE);
+        }
       }
     }
   };
@@ -811,10 +829,11 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
     unsigned long long t0 = p.trace ? gtimer() : 0;
     process_group<PHASE>(c, ws, ins, coll, lc);
     if (p.trace && lane == 0) {
-      const uint32_t i = atomicAdd(p.trace_n, 3u);
-      p.trace[i] = make_ulonglong4(t0, gtimer(), (unsigned long long)c.G, PHASE);
-      p.trace[i + 1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 10 + PHASE);
-      p.trace[i + 2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 20 + PHASE);
+      if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 3)) {
+        r[0] = make_ulonglong4(t0, gtimer(), (unsigned long long)c.G, PHASE);
+        r[1] = make_ulonglong4(ws.tp[0], ws.tp[1], ws.tp[2], 10 + PHASE);
+        r[2] = make_ulonglong4(ws.tp[3], ws.tp[4], 0, 20 + PHASE);
+      }
     }
     return c;
   };
@@ -825,23 +844,35 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   for (uint64_t w = (uint64_t)blockIdx.x * kWarps + wid; w < count; w += nwarps) {
     const uint64_t T = __ldcg(p.wl0 + w);
     Ctx c = run_tile(T);
-    if (PHASE == 2 && lane == 0) p.st[0].dirty[T] = p.g.epoch;
     climb(c);
   }
-  if (ins) atomicAdd(&s_cnt[3], ins);
-  if (PHASE == 2 && coll) atomicAdd(&p.tot->collisions, coll);
+  const unsigned long long ta = p.trace ? gtime_ns() : 0;
   if (PHASE == 2) {
-    if (lc.f) atomicAdd(&s_cnt[0], (unsigned long long)lc.f);
-    if (lc.s) atomicAdd(&s_cnt[1], (unsigned long long)lc.s);
-    if (lc.t) atomicAdd(&s_cnt[2], (unsigned long long)lc.t);
+    // warp sums first: 64-bit shared atomics are CAS loops, 256 contending threads serialise
+    unsigned long long v[5] = {ins, coll, lc.f, lc.s, lc.t};
+#pragma unroll
+    for (int i = 0; i < 5; ++i)
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_xor_sync(0xffffffffu, v[i], o);
+    if (lane == 0) {
+      if (v[0]) atomicAdd(&s_cnt[3], v[0]);
+      if (v[1]) atomicAdd(&p.tot->collisions, v[1]);
+      if (v[2]) atomicAdd(&s_cnt[0], v[2]);
+      if (v[3]) atomicAdd(&s_cnt[1], v[3]);
+      if (v[4]) atomicAdd(&s_cnt[2], v[4]);
+    }
   }
   __syncthreads();
+  const unsigned long long tb = p.trace ? gtime_ns() : 0;
   if (threadIdx.x == 0 && PHASE == 2) {
     if (s_cnt[3]) atomicAdd(&p.tot->p2_inserts, s_cnt[3]);
     if (s_cnt[0]) atomicAdd(&p.tot->n_first, s_cnt[0]);
     if (s_cnt[1]) atomicAdd(&p.tot->n_spatial, s_cnt[1]);
     if (s_cnt[2]) atomicAdd(&p.tot->n_temporal, s_cnt[2]);
   }
+  if (p.trace && threadIdx.x == 0)
+    if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 1)) *r = make_ulonglong4(ta, tb, gtime_ns(), 90 + PHASE);
+  trace_block(p.trace, p.trace_n, bt0, bt1, PHASE);
 }
 
 static int g_tree_blocks_per_sm[2] = {0, 0};

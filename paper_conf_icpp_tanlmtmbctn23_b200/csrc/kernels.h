@@ -48,11 +48,12 @@ struct InsertParams {
   uint32_t* defer;               // (tile << 3 | round) entries left for K1b
   // tree work discovery (K1/K1t mark, K1b block 0 compacts)
   uint32_t* dbits;               // dirty bit per stage-0 tree tile
+  uint32_t* tcc;                 // candidate leaves per stage-0 tree tile (full-tile test)
   uint64_t n_tiles;
   uint32_t* wl0;                 // out: dirty stage-0 tiles
   int S;
   int gsz[kMaxStages];
-  uint32_t* dcnt[kMaxStages];    // out: s >= 1, dirty children per group
+  uint32_t* dcnt[kMaxStages];    // out: s >= 1, FULL children per group (the climb target)
   ulonglong4* trace;             // diagnostics (CKPT_TRACE)
   uint32_t* trace_n;
 };
@@ -73,8 +74,6 @@ struct LeafParams {
 };
 
 struct LevelIO {               // per-position arrays at one height (stage boundary)
-  uint8_t* lab2;               // phase-2 label (FIRST or not)
-  uint8_t* lab3;               // phase-3 label (FIRST / FIXED / SHIFT / DONE)
   Digest* dig;                 // digest of FIRST (phase 2) or SHIFT (phase 3) positions
   unsigned long long* src;     // packed (ckpt<<32|node) source of SHIFT positions
 };
@@ -82,16 +81,14 @@ struct LevelIO {               // per-position arrays at one height (stage bound
 struct StageParams {
   int Lin;                     // input height
   int gsz;                     // log2 positions per group (levels processed)
-  const uint32_t* dirty_in;    // s >= 1: dirty marks of stage s-1 (per input position)
   LevelIO in;                  // s >= 1: input arrays (written by stage s-1)
   Digest* tdig;                // per group: digests of internal nodes (2^gsz entries)
   unsigned long long* tsrc;    // per group: sources of SHIFT nodes (2 * 2^gsz entries)
-  uint32_t* dirty;             // epoch mark of this stage's dirty groups (written in phase 2)
   uint32_t* arr2;              // s >= 1: arrivals of dirty children, phase 2
   uint32_t* arr3;              //                                     phase 3
-  const uint32_t* dcnt;        // s >= 1: dirty children per group (K1b)
+  const uint32_t* dcnt;        // s >= 1: full children per group (K1b)
   uint32_t* gm2;               // s >= 1: per group, 32 words: FIRST children (bit-reversed), phase 2
-  uint32_t* gm3;               // s >= 1: per group, 96 words: FIRST / SHIFT / DONE children, phase 3
+  uint32_t* gm3;               // s >= 1: per group, 64 words: FIRST / SHIFT children, phase 3
 };
 
 struct TreeParams {
@@ -99,6 +96,7 @@ struct TreeParams {
   int S;
   uint64_t n_tiles;
   const uint32_t* wl0;         // dirty stage-0 tiles (K1b)
+  const uint32_t* tcc;         // candidate leaves per stage-0 tile (K1/K1t)
   const uint32_t* cand;
   const uint32_t* slot_of;
   const Digest* prev;
@@ -134,6 +132,9 @@ struct CompactParams {
   uint4* ctr_next;               // the next call's counter block, zeroed by the data kernel
   uint64_t ctr_next_words;
 };
+
+// CKPT_TRACE diagnostics buffer: kTraceLanes regions of kTraceLaneCap 32-B records.
+constexpr uint32_t kTraceLanes = 64, kTraceLaneCap = 16384;
 
 // Kernel launches issued by this thread (every launch site calls note_launch once per
 // kernel it enqueues); the engine adds the per-call difference to the handle's counter.

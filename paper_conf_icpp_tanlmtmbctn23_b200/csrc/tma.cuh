@@ -83,4 +83,27 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap* map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
 }
 
+__device__ __forceinline__ unsigned long long gtime_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Diagnostics (CKPT_TRACE): records are appended to one of kTraceLanes regions (lane =
+// block index mod kTraceLanes, one counter per lane 32 B apart) so tracing adds no single
+// hot atomic to the kernels it measures. Returns nullptr when the lane is full.
+__device__ __forceinline__ ulonglong4* trace_alloc(ulonglong4* tr, uint32_t* tn, uint32_t nrec) {
+  const uint32_t l = blockIdx.x & (kTraceLanes - 1);
+  const uint32_t i = atomicAdd(tn + 8 * l, nrec);
+  return i + nrec <= kTraceLaneCap ? tr + (size_t)l * kTraceLaneCap + i : nullptr;
+}
+
+// one record per block {entry, after griddepcontrol.wait, exit, 100 + kernel code}
+__device__ __forceinline__ void trace_block(ulonglong4* tr, uint32_t* tn, unsigned long long t0, unsigned long long t1,
+                                            uint32_t code) {
+  if (tr && threadIdx.x == 0) {
+    if (ulonglong4* r = trace_alloc(tr, tn, 1)) *r = make_ulonglong4(t0, t1, gtime_ns(), 100 + code);
+  }
+}
+
 }  // namespace ckpt
