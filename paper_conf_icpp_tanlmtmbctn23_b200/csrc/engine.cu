@@ -70,13 +70,13 @@ struct ckpt_ctx {
   // kernel zeroes ctr2[(k + 1) & 1] for the next call, so no memset precedes K1.
   uint8_t* ctr2[2] = {};
   size_t ctr_bytes = 0;
-  size_t ctr_dbits_off = 0, ctr_tcc_off = 0, ctr_bsum_off = 0, ctr_stage_off[kMaxStages] = {};
+  size_t ctr_dbits_off = 0, ctr_tcc_off = 0, ctr_bsum_off = 0, ctr_gsum_off = 0, ctr_stage_off[kMaxStages] = {};
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
   uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b
-  uint4* toff = nullptr;
   unsigned long long* blocksum = nullptr;
+  unsigned long long* gsum = nullptr;
   ulonglong2* big = nullptr;
   unsigned long long* big_len = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
@@ -191,6 +191,9 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     const size_t bsum_off = bytes;
     bytes += (3 * ((n_tiles + kTilesPerBlock - 1) / kTilesPerBlock) + 3) * sizeof(unsigned long long);
     bytes = (bytes + 255) & ~size_t(255);
+    const size_t gsum_off = bytes;
+    bytes += 3 * ((n_tiles + 31) / 32) * sizeof(unsigned long long);
+    bytes = (bytes + 255) & ~size_t(255);
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
@@ -204,6 +207,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     h->ctr_dbits_off = dbits_off;
     h->ctr_tcc_off = tcc_off;
     h->ctr_bsum_off = bsum_off;
+    h->ctr_gsum_off = gsum_off;
     for (int s = 1; s < h->S; ++s) h->ctr_stage_off[s] = off[s];
   }
   AL(h->scratch, n_tiles << h->t0);
@@ -211,7 +215,6 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->wl0, n_tiles);
   AL(h->lmask, n_tiles * 192);   // k_tree.cu kLmWords
   AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
-  AL(h->toff, n_tiles);
   AL(h->big, B / (1 << 20) + 2);
   AL(h->big_len, B / (1 << 20) + 2);
 #undef AL
@@ -451,6 +454,7 @@ static void select_ctr(ckpt_ctx* h, int parity) {
   h->dbits = reinterpret_cast<uint32_t*>(c + h->ctr_dbits_off);
   h->tcc = reinterpret_cast<uint32_t*>(c + h->ctr_tcc_off);
   h->blocksum = reinterpret_cast<unsigned long long*>(c + h->ctr_bsum_off);
+  h->gsum = reinterpret_cast<unsigned long long*>(c + h->ctr_gsum_off);
   for (int s = 1; s < h->S; ++s) {
     h->arr2[s] = reinterpret_cast<uint32_t*>(c + h->ctr_stage_off[s]);
     h->arr3[s] = h->arr2[s] + h->ngroups[s];
@@ -572,6 +576,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
   tp.blocksum = h->blocksum;
+  tp.gsum = h->gsum;
   tp.trace = h->trace; tp.trace_n = h->trace_n;
   tp.dbg = h->dbg;
 
@@ -598,7 +603,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.g = g;
   cp.n_tiles = h->ngroups[0];
   cp.tilecnt = h->tilecnt; cp.scratch = h->scratch; cp.blocksum = h->blocksum;
-  cp.toff = h->toff; cp.wl0 = h->wl0; cp.tot = h->tot;
+  cp.gsum = h->gsum; cp.wl0 = h->wl0; cp.tot = h->tot;
   cp.big = h->big; cp.big_len = h->big_len;
   cp.out = out; cp.buf = buf;
   cp.trace = h->trace; cp.trace_n = h->trace_n;

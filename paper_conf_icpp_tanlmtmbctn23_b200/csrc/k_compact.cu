@@ -4,13 +4,14 @@
 // difference directly on the GPU memory ... pre-calculates offsets in the consolidated
 // difference and assigns GPU threads to parallelize the data transfers", with "a
 // team of threads to copy each chunk" so accesses coalesce.
-//   (the per-1024-tile sums of #FIRST regions, #SHIFT regions and FIRST bytes are
-//    accumulated by the phase-3 kernel as it writes the tile counts)
-//   KO offsets_kernel: prefix over earlier blocks + block scan -> per-tile offsets;
-//                      the last block writes the 64-B header, the zero pad and totals.
-//   KG gather_kernel : one CTA per dirty tile writes its FIRST entries (u32 node) and
-//                      SHIFT entries (u32 node, src node, src ckpt) (R13)
-//                      and the global data offset of each FIRST region.
+//   (the phase-3 kernel writes every dirty tile's counts {#FIRST regions, #SHIFT regions,
+//    FIRST bytes} and adds them to per-32-tile and per-1024-tile sums)
+//   KG gather_kernel : one warp per dirty tile. Its offsets in the three sections are the
+//                      exclusive prefix of the counts, summed directly from <= 2048 block
+//                      sums, <= 31 group sums and <= 31 tile counts (one round of loads);
+//                      it writes its FIRST entries (u32 node) and SHIFT entries (u32 node,
+//                      src node, src ckpt) (R13) and copies its FIRST bytes.
+//                      Block 0 writes the 64-B header, the zero pad and the totals.
 //   KD data_kernel   : copies the FIRST chunks into the data section, warp per 8-KiB
 //                      segment, coalesced 16-byte loads/stores (balanced even when one
 //                      region is the whole buffer).
@@ -19,101 +20,17 @@
 
 namespace ckpt {
 
-__device__ __forceinline__ void block_sum3(unsigned long long& a, unsigned long long& b, unsigned long long& c,
-                                           unsigned long long* sh /* 3 * nwarps */) {
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+__device__ __forceinline__ void warp_sum3(unsigned long long& a, unsigned long long& b, unsigned long long& c) {
+#pragma unroll
   for (int o = 16; o > 0; o >>= 1) {
     a += __shfl_xor_sync(0xffffffffu, a, o);
     b += __shfl_xor_sync(0xffffffffu, b, o);
     c += __shfl_xor_sync(0xffffffffu, c, o);
   }
-  if (lane == 0) { sh[wid] = a; sh[nw + wid] = b; sh[2 * nw + wid] = c; }
-  __syncthreads();
-  a = b = c = 0;
-  for (int i = 0; i < nw; ++i) { a += sh[i]; b += sh[nw + i]; c += sh[2 * nw + i]; }
-  __syncthreads();
 }
+
 
 constexpr int kCT = 256;
-constexpr int kPer = kTilesPerBlock / kCT;
-
-__global__ void __launch_bounds__(kCT) offsets_kernel(CompactParams p) {
-  __shared__ unsigned long long sh[3 * (kCT / 32)];
-  __shared__ unsigned long long wx[kCT / 32], wy[kCT / 32], wz[kCT / 32];
-  const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
-  pdl_launch_dependents();
-  pdl_wait();
-  const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
-  // prefix of earlier blocks
-  unsigned long long a = 0, b = 0, c = 0;
-  for (uint32_t i = threadIdx.x; i < blockIdx.x; i += kCT) {
-    a += p.blocksum[3 * i];
-    b += p.blocksum[3 * i + 1];
-    c += p.blocksum[3 * i + 2];
-  }
-  block_sum3(a, b, c, sh);
-  const unsigned long long pa = a, pb = b, pc = c;
-  // per-thread values
-  const uint64_t t0 = (uint64_t)blockIdx.x * kTilesPerBlock + threadIdx.x * kPer;
-  uint4 v[kPer];
-  unsigned long long ma = 0, mb = 0, mc = 0;
-  for (int i = 0; i < kPer; ++i) {
-    const uint64_t T = t0 + i;
-    v[i] = make_uint4(0, 0, 0, 0);
-    if (T < p.n_tiles) {
-      const uint4 x = p.tilecnt[T];
-      if (x.w == p.g.epoch) v[i] = x;
-    }
-    ma += v[i].x; mb += v[i].y; mc += v[i].z;
-  }
-  // block exclusive scan (warp shuffles + warp totals)
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  unsigned long long ia = ma, ib = mb, ic = mc;
-  for (int o = 1; o < 32; o <<= 1) {
-    const unsigned long long ua = __shfl_up_sync(0xffffffffu, ia, o);
-    const unsigned long long ub = __shfl_up_sync(0xffffffffu, ib, o);
-    const unsigned long long uc = __shfl_up_sync(0xffffffffu, ic, o);
-    if (lane >= o) { ia += ua; ib += ub; ic += uc; }
-  }
-  if (lane == 31) { wx[wid] = ia; wy[wid] = ib; wz[wid] = ic; }
-  __syncthreads();
-  unsigned long long oa = pa, ob = pb, oc = pc, ta = pa, tb = pb, tc = pc;
-  for (int i = 0; i < kCT / 32; ++i) {
-    if (i < wid) { oa += wx[i]; ob += wy[i]; oc += wz[i]; }
-    ta += wx[i]; tb += wy[i]; tc += wz[i];
-  }
-  oa += ia - ma; ob += ib - mb; oc += ic - mc;
-  for (int i = 0; i < kPer; ++i) {
-    const uint64_t T = t0 + i;
-    if (T < p.n_tiles && (v[i].x | v[i].y))
-      p.toff[T] = make_uint4((uint32_t)oa, (uint32_t)ob, (uint32_t)(oc & 0xffffffffu), (uint32_t)(oc >> 32));
-    oa += v[i].x; ob += v[i].y; oc += v[i].z;
-  }
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
-    // totals and the 64-byte header (R13)
-    const unsigned long long nF = ta, nS = tb, data = tc;
-    const unsigned long long raw = 64 + 4 * nF + 12 * nS;
-    const unsigned long long meta = (raw + 15) & ~15ull;
-    p.tot->nF = nF; p.tot->nS = nS; p.tot->data_bytes = data; p.tot->meta_bytes = meta;
-    uint8_t* o = p.out;
-    *reinterpret_cast<uint32_t*>(o + 0) = 0x44504B43u;   // 'CKPD'
-    *reinterpret_cast<uint16_t*>(o + 4) = 1;             // version
-    *reinterpret_cast<uint16_t*>(o + 6) = 0;             // flags
-    *reinterpret_cast<uint32_t*>(o + 8) = p.g.k;
-    *reinterpret_cast<uint32_t*>(o + 12) = p.g.C;
-    *reinterpret_cast<unsigned long long*>(o + 16) = p.g.B;
-    *reinterpret_cast<unsigned long long*>(o + 24) = p.g.n;
-    *reinterpret_cast<unsigned long long*>(o + 32) = nF;
-    *reinterpret_cast<unsigned long long*>(o + 40) = nS;
-    *reinterpret_cast<unsigned long long*>(o + 48) = data;
-    *reinterpret_cast<uint32_t*>(o + 56) = 0;            // hash seed
-    *reinterpret_cast<uint32_t*>(o + 60) = 0;            // reserved
-    for (unsigned long long x = raw; x < meta; ++x) o[x] = 0;
-    // every counter the host reports is final here (tree kernels done, pdl_wait above)
-    *p.tot_host = *p.tot;
-  }
-  trace_block(p.trace, p.trace_n, bt0, bt1, 4);
-}
 
 // KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata entries
 // and copies its FIRST bytes: the tile's FIRST regions are taken 32 at a time (lane i ->
@@ -139,10 +56,40 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
   pdl_launch_dependents();
   pdl_wait();
   const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
-  const unsigned long long nF_tot = p.tot->nF;
+  // totals = sum of the per-1024-tile block sums (every warp; 8 values at 1 GiB, C = 128)
+  const uint64_t nblk = (p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock;
+  unsigned long long nF_tot = 0, nS_tot = 0, data_tot = 0;
+  for (uint64_t i = lane; i < nblk; i += 32) {
+    nF_tot += __ldcg(p.blocksum + 3 * i);
+    nS_tot += __ldcg(p.blocksum + 3 * i + 1);
+    data_tot += __ldcg(p.blocksum + 3 * i + 2);
+  }
+  warp_sum3(nF_tot, nS_tot, data_tot);
+  const unsigned long long raw = 64 + 4 * nF_tot + 12 * nS_tot;
+  const unsigned long long meta = (raw + 15) & ~15ull;
+  if (blockIdx.x == 0 && wid == 0 && lane == 0) {
+    // totals and the 64-byte header (R13)
+    p.tot->nF = nF_tot; p.tot->nS = nS_tot; p.tot->data_bytes = data_tot; p.tot->meta_bytes = meta;
+    uint8_t* o = p.out;
+    *reinterpret_cast<uint32_t*>(o + 0) = 0x44504B43u;   // 'CKPD'
+    *reinterpret_cast<uint16_t*>(o + 4) = 1;             // version
+    *reinterpret_cast<uint16_t*>(o + 6) = 0;             // flags
+    *reinterpret_cast<uint32_t*>(o + 8) = g.k;
+    *reinterpret_cast<uint32_t*>(o + 12) = g.C;
+    *reinterpret_cast<unsigned long long*>(o + 16) = g.B;
+    *reinterpret_cast<unsigned long long*>(o + 24) = g.n;
+    *reinterpret_cast<unsigned long long*>(o + 32) = nF_tot;
+    *reinterpret_cast<unsigned long long*>(o + 40) = nS_tot;
+    *reinterpret_cast<unsigned long long*>(o + 48) = data_tot;
+    *reinterpret_cast<uint32_t*>(o + 56) = 0;            // hash seed
+    *reinterpret_cast<uint32_t*>(o + 60) = 0;            // reserved
+    for (unsigned long long x = raw; x < meta; ++x) o[x] = 0;
+    // every counter the host reports is final here (tree kernels done, pdl_wait above)
+    *p.tot_host = *p.tot;
+  }
   uint8_t* const ent_f = p.out + 64;
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
-  uint8_t* const dat = p.out + p.tot->meta_bytes;
+  uint8_t* const dat = p.out + meta;
 
   const uint64_t nwarps = (uint64_t)gridDim.x * kGW;
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
@@ -150,12 +97,35 @@ __global__ void __launch_bounds__(kCT) gather_kernel(CompactParams p) {
     unsigned long long tg0 = 0, tg1 = 0, tg2 = 0;
     if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg0));
     const uint64_t T = __ldcg(p.wl0 + w);
-    const uint4 cnt = p.tilecnt[T];
+    const uint4 cnt = __ldcg(p.tilecnt + T);
+    // exclusive prefix of tile T: earlier 1024-tile blocks, earlier 32-tile groups of its
+    // block, earlier tiles of its group (stale tile counts carry an older epoch)
+    unsigned long long pF = 0, pS = 0, pD = 0;
+    {
+      const uint64_t B0 = T / kTilesPerBlock, G0 = T / 32;
+      for (uint64_t i = lane; i < B0; i += 32) {
+        pF += __ldcg(p.blocksum + 3 * i);
+        pS += __ldcg(p.blocksum + 3 * i + 1);
+        pD += __ldcg(p.blocksum + 3 * i + 2);
+      }
+      const uint64_t gq = B0 * (kTilesPerBlock / 32) + lane;
+      if (gq < G0) {
+        pF += __ldcg(p.gsum + 3 * gq);
+        pS += __ldcg(p.gsum + 3 * gq + 1);
+        pD += __ldcg(p.gsum + 3 * gq + 2);
+      }
+      const uint64_t tq = G0 * 32 + lane;
+      if (tq < T) {
+        const uint4 x = __ldcg(p.tilecnt + tq);
+        if (x.w == g.epoch) { pF += x.x; pS += x.y; pD += x.z; }
+      }
+      warp_sum3(pF, pS, pD);
+    }
     if (cnt.w != g.epoch) continue;
     const uint32_t nF = cnt.x, nS = cnt.y;
     if (nF + nS == 0) continue;
-    const uint4 off = p.toff[T];
-    const unsigned long long doff = (unsigned long long)off.z | ((unsigned long long)off.w << 32);
+    const uint4 off = make_uint4((uint32_t)pF, (uint32_t)pS, 0u, 0u);
+    const unsigned long long doff = pD;
     const uint4* recs = p.scratch + ((uint64_t)T << g.t0);
     if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tg1));
     // SHIFT entries (R13): u32 node, u32 src node, u32 src ckpt
@@ -277,13 +247,10 @@ __global__ void __launch_bounds__(kCT) data_kernel(CompactParams p) {
 }
 
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st) {
-  const unsigned nblk = (unsigned)((p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock);
-  // per-block sums were accumulated by the phase-3 kernel (k_tree.cu), so no reduce pass
-  cudaError_t e = launch_pdl(offsets_kernel, nblk, kCT, 0, st, p);
-  if (e != cudaSuccess) return e;
+  // the tile offsets are prefix sums the gather warps compute themselves (see above)
   uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
   if (grid > (uint64_t)num_sms * 8) grid = (uint64_t)num_sms * 8;
-  e = launch_pdl(gather_kernel, (unsigned)grid, kCT, 0, st, p);
+  cudaError_t e = launch_pdl(gather_kernel, (unsigned)grid, kCT, 0, st, p);
   if (e == cudaSuccess) e = launch_pdl(data_kernel, (unsigned)(num_sms * 4), kCT, 0, st, p);
   return e;
 }
@@ -294,7 +261,6 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
 cudaError_t preload_compact() {
   cudaFuncAttributes a;
   cudaError_t e = cudaSuccess;
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, offsets_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gather_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, data_kernel);
   return e;

@@ -396,10 +396,16 @@ __device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, 
   p.scratch[tile << p.g.t0] = make_uint4(node, (uint32_t)(src & 0xffffffffu), (uint32_t)(src >> 32),
                                          first ? L_FIRST : L_SHIFT);
   p.tilecnt[tile] = make_uint4(first ? 1u : 0u, first ? 0u : 1u, bytes, p.g.epoch);
-  // the tile had no region of its own (it lies inside this one): add the region to its block sum
+  // the tile had no region of its own (it lies inside this one): add the region to the
+  // sums of its 1024-tile block and 32-tile group (the gather kernel's prefix inputs)
   unsigned long long* bs = p.blocksum + 3 * (tile / kTilesPerBlock);
+  unsigned long long* gs = p.gsum + 3 * (tile / 32);
   atomicAdd(bs + (first ? 0 : 1), 1ull);
-  if (first) atomicAdd(bs + 2, (unsigned long long)bytes);
+  atomicAdd(gs + (first ? 0 : 1), 1ull);
+  if (first) {
+    atomicAdd(bs + 2, (unsigned long long)bytes);
+    atomicAdd(gs + 2, (unsigned long long)bytes);
+  }
 }
 
 // Process one group through its gsz levels. PHASE 2 or 3.
@@ -748,9 +754,10 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
     if (lane == 0) {
       p.tilecnt[c.G] = make_uint4(nFt, nSt, bytes, g.epoch);
       unsigned long long* bs = p.blocksum + 3 * (c.G / kTilesPerBlock);
-      if (nFt) atomicAdd(bs, (unsigned long long)nFt);
-      if (nSt) atomicAdd(bs + 1, (unsigned long long)nSt);
-      if (bytes) atomicAdd(bs + 2, (unsigned long long)bytes);
+      unsigned long long* gs = p.gsum + 3 * (c.G / 32);
+      if (nFt) { atomicAdd(bs, (unsigned long long)nFt); atomicAdd(gs, (unsigned long long)nFt); }
+      if (nSt) { atomicAdd(bs + 1, (unsigned long long)nSt); atomicAdd(gs + 1, (unsigned long long)nSt); }
+      if (bytes) { atomicAdd(bs + 2, (unsigned long long)bytes); atomicAdd(gs + 2, (unsigned long long)bytes); }
     }
     __syncwarp();
   }

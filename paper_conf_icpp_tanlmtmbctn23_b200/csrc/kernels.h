@@ -106,6 +106,7 @@ struct TreeParams {
   uint4* tilecnt;              // per tile: {nF, nS, data_bytes, epoch}
   uint32_t* lmask;             // per tile: resolved leaf masks (phase 2 -> phase 3)
   unsigned long long* blocksum;  // per 1024 tiles: (#FIRST, #SHIFT, FIRST bytes), zeroed per call
+  unsigned long long* gsum;      // per 32 tiles: the same sums
   Totals* tot;
   int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
   ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
@@ -118,8 +119,8 @@ struct CompactParams {
   uint64_t n_tiles;
   const uint4* tilecnt;
   const uint4* scratch;
-  unsigned long long* blocksum;  // 3 per reduce block
-  uint4* toff;                   // per tile {F_off, S_off, data_off lo, data_off hi}
+  const unsigned long long* blocksum;  // per 1024 tiles: (#FIRST, #SHIFT, FIRST bytes) (phase 3)
+  const unsigned long long* gsum;      // per 32 tiles: the same sums (phase 3)
   const uint32_t* wl0;           // dirty stage-0 tiles
   Totals* tot;
   ulonglong2* big;               // deferred big FIRST regions: {data offset, source offset}
