@@ -77,8 +77,6 @@ struct ckpt_ctx {
   uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b
   unsigned long long* blocksum = nullptr;
   unsigned long long* gsum = nullptr;
-  ulonglong2* big = nullptr;
-  unsigned long long* big_len = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
   Totals* tot_host = nullptr;   // pinned + mapped: written by the offsets kernel
   Slot* tab = nullptr;
@@ -213,10 +211,8 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->scratch, n_tiles << h->t0);
   AL(h->tilecnt, n_tiles);
   AL(h->wl0, n_tiles);
-  AL(h->lmask, n_tiles * 192);   // k_tree.cu kLmWords
+  AL(h->lmask, n_tiles * kLmWords);
   AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
-  AL(h->big, B / (1 << 20) + 2);
-  AL(h->big_len, B / (1 << 20) + 2);
 #undef AL
   if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
   if (h->trace_path) {
@@ -571,6 +567,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.S = h->S;
   tp.n_tiles = h->ngroups[0];
   tp.wl0 = h->wl0;
+  tp.buf = buf;
   tp.tcc = h->tcc;
   tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
@@ -604,10 +601,11 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.n_tiles = h->ngroups[0];
   cp.tilecnt = h->tilecnt; cp.scratch = h->scratch; cp.blocksum = h->blocksum;
   cp.gsum = h->gsum; cp.wl0 = h->wl0; cp.tot = h->tot;
-  cp.big = h->big; cp.big_len = h->big_len;
+  cp.lmask = h->lmask;
   cp.out = out; cp.buf = buf;
   cp.trace = h->trace; cp.trace_n = h->trace_n;
   cp.tot_host = h->tot_host;
+  cp.dbg = h->dbg;
   cp.ctr_next = reinterpret_cast<uint4*>(h->ctr2[(k + 1) & 1]);
   cp.ctr_next_words = h->ctr_bytes / 16;
   CK(launch_compact(cp, h->num_sms, st));

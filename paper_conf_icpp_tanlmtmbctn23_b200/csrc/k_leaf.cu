@@ -254,7 +254,13 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
         st_evict_last_u32(p.cand + (c >> 5), mask, pol_keep);
         ring.stage_words[ntile_done & 1][tid >> 5] = mask;
       }
-      if (cand) st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
+      if (cand) {
+        st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
+        // a candidate's bytes may be copied into the diff by the gather kernel: keep the
+        // lines that TMA just brought in (evict_first) resident past the rest of the stream
+        const uint8_t* cp = p.buf + c * (uint64_t)p.g.C;
+        for (uint32_t o = 0; o < p.g.C; o += 128) l2_keep_line(cp + o);
+      }
     }
     asm volatile("bar.sync 1, %0;" ::"n"(kLeafThreads) : "memory");   // every hashing thread is done with stage st
     if (tid == 0) {

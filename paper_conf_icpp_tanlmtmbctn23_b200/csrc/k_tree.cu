@@ -38,7 +38,6 @@ namespace {
 
 constexpr int kWarps = kTreeThreads / 32;
 constexpr int kDigCap = 256;   // on-chip digests per warp (4 KB); dense groups spill to global
-constexpr int kLmWords = 192;  // per tile: F0 S0 X0 F1 S1 leaf1 (rev order), 32 words each
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -387,25 +386,29 @@ __device__ __forceinline__ void emit_region(const Ctx& c, WarpSmem& ws, int lv, 
   const uint64_t gpos = (c.G << (c.gsz - lv)) + q;
   const uint32_t node = node_id(p.g, Lc, gpos);
   const uint64_t tile = (gpos << Lc) >> p.g.t0;
-  uint32_t bytes = 0;
-  if (first) {
-    uint64_t lo, hi;
-    chunk_range(p.g, Lc, gpos, lo, hi);
-    bytes = (uint32_t)range_bytes(p.g, lo, hi);
-  }
   p.scratch[tile << p.g.t0] = make_uint4(node, (uint32_t)(src & 0xffffffffu), (uint32_t)(src >> 32),
                                          first ? L_FIRST : L_SHIFT);
-  p.tilecnt[tile] = make_uint4(first ? 1u : 0u, first ? 0u : 1u, bytes, p.g.epoch);
+  // region counts of the region's first tile (its FIRST bytes were counted by phase 2)
+  reinterpret_cast<uint2*>(p.tilecnt + tile)[0] = make_uint2(first ? 1u : 0u, first ? 0u : 1u);
   // the tile had no region of its own (it lies inside this one): add the region to the
   // sums of its 1024-tile block and 32-tile group (the gather kernel's prefix inputs)
   unsigned long long* bs = p.blocksum + 3 * (tile / kTilesPerBlock);
   unsigned long long* gs = p.gsum + 3 * (tile / 32);
   atomicAdd(bs + (first ? 0 : 1), 1ull);
   atomicAdd(gs + (first ? 0 : 1), 1ull);
-  if (first) {
-    atomicAdd(bs + 2, (unsigned long long)bytes);
-    atomicAdd(gs + 2, (unsigned long long)bytes);
-  }
+}
+
+// Natural-order bit words (lane i = bits 32i..32i+31) shifted up by s bits across the warp.
+__device__ __forceinline__ uint32_t shift_up_bits(uint32_t w, uint32_t s) {
+  const int lane = threadIdx.x & 31;
+  const int q = (int)(s >> 5);
+  const uint32_t r = s & 31;
+  const uint32_t cur = __shfl_sync(0xffffffffu, w, (lane - q) & 31);
+  const uint32_t prv = __shfl_sync(0xffffffffu, w, (lane - q - 1) & 31);
+  uint32_t o = 0;
+  if (lane >= q) o = cur << r;
+  if (lane >= q + 1 && r) o |= prv >> (32 - r);
+  return o;
 }
 
 // Process one group through its gsz levels. PHASE 2 or 3.
@@ -432,6 +435,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
     if (PHASE == 2) {
       uint32_t nF, nS, nX;
       resolve_leaves(c, ws, base, npos0, 0, 0, gsz, nF, nS, nX, lc);
+      uint32_t fchunks = nF;   // the tile's FIRST chunks, chunk order (height-0 chunks first)
       to_rev3(ws, gsz, nF, nS, nX, F, S, X);
       lm[lane] = F;
       lm[32 + lane] = S;
@@ -460,6 +464,29 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
         lm[96 + lane] = lF1;
         lm[128 + lane] = lS1;
         lm[160 + lane] = leafm1;
+        fchunks |= shift_up_bits(tF, (uint32_t)npos0);   // height-1 chunks follow at offset npos0
+      }
+      // The data section is the FIRST chunks in chunk order (every FIRST leaf lies in exactly
+      // one FIRST region and those regions hold only FIRST leaves), so the gather kernel
+      // needs just this mask and the tile's FIRST bytes (the last chunk may be short).
+      lm[kLmFirstChunks + lane] = fchunks;
+      uint32_t nfc = __popc(fchunks);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) nfc += __shfl_xor_sync(0xffffffffu, nfc, o);
+      uint64_t lo, hi;
+      chunk_range(g, g.t0, c.G, lo, hi);
+      unsigned long long fb = (unsigned long long)nfc * g.C;
+      if (hi == g.n) {   // the tile holds the buffer's last chunk, possibly short
+        const uint32_t b = (uint32_t)(g.n - 1 - lo);
+        const uint32_t wlast = __shfl_sync(0xffffffffu, fchunks, (int)(b >> 5));
+        if ((wlast >> (b & 31)) & 1u) fb -= (unsigned long long)g.n * g.C - g.B;
+      }
+      if (lane == 0) {
+        reinterpret_cast<uint2*>(p.tilecnt + c.G)[1] = make_uint2((uint32_t)fb, g.epoch);
+        if (fb) {
+          atomicAdd(p.blocksum + 3 * (c.G / kTilesPerBlock) + 2, fb);
+          atomicAdd(p.gsum + 3 * (c.G / 32) + 2, fb);
+        }
       }
     } else {
       F = __ldcg(lm + lane);
@@ -713,16 +740,13 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
     }
     const uint32_t nFt = __shfl_sync(0xffffffffu, iF, 31), nSt = __shfl_sync(0xffffffffu, iS, 31);
     uint32_t rf = iF - __popc(wF), rs = nFt + iS - __popc(wS);
-    uint32_t bytes = 0;
     uint4* out = p.scratch + (c.G << g.t0);
     for (uint32_t m = wF; m; m &= m - 1) {
       const uint32_t slot = lane * 32 + (__ffs(m) - 1);
       const int lv = ws.lvl[slot];
       const uint64_t gpos = (c.G << (gsz - lv)) + (slot >> lv);
-      uint64_t lo, hi;
-      chunk_range(g, lv, gpos, lo, hi);
-      bytes += (uint32_t)range_bytes(g, lo, hi);
       out[rf++] = make_uint4(node_id(g, lv, gpos), 0u, 0u, L_FIRST);
+
     }
     for (uint32_t m = wS; m;) {   // batches of 4: issue the source loads first
       uint32_t slots[4];
@@ -749,15 +773,12 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
         }
       }
     }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) bytes += __shfl_xor_sync(0xffffffffu, bytes, o);
     if (lane == 0) {
-      p.tilecnt[c.G] = make_uint4(nFt, nSt, bytes, g.epoch);
+      reinterpret_cast<uint2*>(p.tilecnt + c.G)[0] = make_uint2(nFt, nSt);   // bytes: phase 2
       unsigned long long* bs = p.blocksum + 3 * (c.G / kTilesPerBlock);
       unsigned long long* gs = p.gsum + 3 * (c.G / 32);
       if (nFt) { atomicAdd(bs, (unsigned long long)nFt); atomicAdd(gs, (unsigned long long)nFt); }
       if (nSt) { atomicAdd(bs + 1, (unsigned long long)nSt); atomicAdd(gs + 1, (unsigned long long)nSt); }
-      if (bytes) { atomicAdd(bs + 2, (unsigned long long)bytes); atomicAdd(gs + 2, (unsigned long long)bytes); }
     }
     __syncwarp();
   }
@@ -906,7 +927,7 @@ cudaError_t tree_setup_attributes() {
   return e;
 }
 
-size_t tree_lmask_words() { return kLmWords; }
+size_t tree_lmask_words() { return (size_t)kLmWords; }
 
 
 // Load this file's kernels now (CUDA lazy module loading would otherwise stall the first

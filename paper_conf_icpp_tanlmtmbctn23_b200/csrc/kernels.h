@@ -30,7 +30,7 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   uint32_t wl_count[kMaxStages];
   uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
   uint32_t gather_next;              // work-stealing cursor of the gather kernel
-  uint32_t big_count;                // FIRST regions deferred to the grid-wide data pass
+  uint32_t unused0;
   uint32_t defer_count;              // 256-chunk leaf tiles whose inserts K1 left to K1b
   uint32_t insert_next;              // work-stealing cursor of K1b
   uint32_t pad2[2];
@@ -96,6 +96,7 @@ struct TreeParams {
   int S;
   uint64_t n_tiles;
   const uint32_t* wl0;         // dirty stage-0 tiles (K1b)
+  const uint8_t* buf;          // checkpoint buffer (phase 3 prefetches FIRST bytes into L2)
   const uint32_t* tcc;         // candidate leaves per stage-0 tile (K1/K1t)
   const uint32_t* cand;
   const uint32_t* slot_of;
@@ -123,16 +124,22 @@ struct CompactParams {
   const unsigned long long* gsum;      // per 32 tiles: the same sums (phase 3)
   const uint32_t* wl0;           // dirty stage-0 tiles
   Totals* tot;
-  ulonglong2* big;               // deferred big FIRST regions: {data offset, source offset}
-  unsigned long long* big_len;   //                              byte length
+  const uint32_t* lmask;         // per tile (phase 2): FIRST-chunk mask at kLmFirstChunks
   uint8_t* out;                  // diff destination (device arena)
   const uint8_t* buf;            // checkpoint buffer (source of first-occurrence data)
   ulonglong4* trace;             // diagnostics (CKPT_TRACE)
   uint32_t* trace_n;
   Totals* tot_host;              // mapped pinned host copy of the final totals (no D2H op)
+  int dbg;                       // diagnostics only (CKPT_DBG bits; 0 in production)
   uint4* ctr_next;               // the next call's counter block, zeroed by the data kernel
   uint64_t ctr_next_words;
 };
+
+// Per stage-0 tile, written by phase 2: the resolved leaf masks for phase 3 (F0 S0 X0 F1 S1
+// leaf1, bit-reversed, 32 words each) and the tile's FIRST chunks in chunk order (32
+// words, bit i = chunk lo + i) for the gather kernel.
+constexpr int kLmWords = 224;
+constexpr int kLmFirstChunks = 192;
 
 // CKPT_TRACE diagnostics buffer: kTraceLanes regions of kTraceLaneCap 32-B records.
 constexpr uint32_t kTraceLanes = 64, kTraceLaneCap = 16384;

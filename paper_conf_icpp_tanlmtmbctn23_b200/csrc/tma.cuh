@@ -67,6 +67,17 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
                : "memory");
 }
 
+// Raise the L2 eviction priority of the 128-B line at p (e.g. from the stream's evict_first)
+// to evict_normal; a no-op if the line is no longer resident.
+__device__ __forceinline__ void l2_keep_line(const void* p) {
+  asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(p) : "memory");
+}
+
+// L2 prefetch of a contiguous global range (16-B aligned, size a multiple of 16).
+__device__ __forceinline__ void prefetch_l2_bulk(const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
+}
+
 __device__ __forceinline__ void st_evict_last_v2(void* p, uint64_t a, uint64_t b, uint64_t pol) {
   asm volatile("st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %3;" ::"l"(p), "l"(a), "l"(b), "l"(pol) : "memory");
 }
