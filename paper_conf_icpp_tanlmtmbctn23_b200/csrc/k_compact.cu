@@ -41,13 +41,25 @@ constexpr int kCT = 256;
 // would serialise those requests.
 constexpr int kGW = kCT / 32;
 
+constexpr int kStageUnits = 768;   // 12 KB of 16-byte units staged per warp and round
+
 struct GatherWarp {
   uint32_t pre[32];   // FIRST chunks in the mask words before word i
   uint32_t fw[32];    // the tile's FIRST-chunk mask words
+  uint4 stage[kStageUnits];
 };
 
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, uint32_t src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_u32(smem)), "l"(gmem), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+}
+
 __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
-  __shared__ GatherWarp gsm[kGW];
+  extern __shared__ __align__(16) uint8_t gather_smem[];
+  GatherWarp* gsm = reinterpret_cast<GatherWarp*>(gather_smem);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   GatherWarp& gw = gsm[wid];
   const Geo& g = p.g;
@@ -103,8 +115,14 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   for (; w < count; w += nwarps) {
     unsigned long long tg0 = 0, tg1 = 0, tg2 = 0;
     if (p.trace) tg0 = gtime_ns();
+    // one round of loads: counts, FIRST-chunk mask, the first 64 region records, prefix sums
     const uint4 cnt = __ldg(p.tilecnt + T);
     const uint32_t fw = __ldg(p.lmask + T * kLmWords + kLmFirstChunks + lane);
+    const uint4* recs = p.scratch + (T << g.t0);
+    const uint32_t tcap = 1u << g.t0;   // records per tile
+    uint4 rec0 = make_uint4(0, 0, 0, 0), rec1 = make_uint4(0, 0, 0, 0);
+    if ((uint32_t)lane < tcap) rec0 = __ldg(recs + lane);
+    if ((uint32_t)lane + 32 < tcap) rec1 = __ldg(recs + 32 + lane);
     // exclusive prefix of tile T: earlier 1024-tile blocks, earlier 32-tile groups of its
     // block, earlier tiles of its group (stale tile counts carry an older epoch)
     unsigned long long pF = 0, pS = 0, pD = 0;
@@ -129,8 +147,10 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     }
     const uint64_t Tcur = T;
     if (w + nwarps < count) T = __ldg(p.wl0 + w + nwarps);   // next tile, early
-    warp_sum3(pF, pS, pD);
-    if (cnt.w != g.epoch) continue;
+    if (cnt.w != g.epoch) {
+      warp_sum3(pF, pS, pD);
+      continue;
+    }
     const uint32_t nF = cnt.x, nS = cnt.y;
     if (p.trace) tg1 = gtime_ns();
     // ranks of the FIRST chunks (chunk order)
@@ -147,49 +167,52 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     __syncwarp();
     uint64_t lo, hi;
     chunk_range(g, g.t0, Tcur, lo, hi);
-    // the FIRST bytes: unit x of the tile's stream = unit (x mod U) of its (x / U)-th chunk
+    // the FIRST bytes: unit x of the tile's stream = unit (x mod U) of its (x / U)-th chunk,
+    // source found from the mask alone; up to kStageUnits units go global -> shared with
+    // cp.async in one round trip, then shared -> the data section at tile offset + 16 x.
+    // The buffer's last chunk may be short: its last unit is zero-filled past B (the store
+    // may then write up to 15 bytes past the data section, inside the arena's slack) and
+    // units entirely past B are skipped.
     const uint32_t nunits = nch * U;
-    constexpr int kU = 8;
-    for (uint32_t x0 = 0; x0 < nunits; x0 += 32 * kU) {
-      uint4 v[kU];
-      const uint8_t* sp[kU];
-      uint8_t* dp[kU];
-      uint32_t nb[kU];
+    auto unit_src = [&](uint32_t x) -> unsigned long long {
+      const uint32_t k = x / U, sub = x - k * U;
+      int i = 0;   // last word with pre <= k (words without FIRST chunks are skipped)
 #pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        const uint32_t x = x0 + u * 32 + lane;
-        nb[u] = 0;
-        if (x < nunits) {
-          const uint32_t k = x / U, sub = x - k * U;
-          int i = 0;   // last word with pre <= k (words without FIRST chunks are skipped)
-#pragma unroll
-          for (int step = 16; step > 0; step >>= 1)
-            if (gw.pre[i + step] <= k) i += step;   // i + step <= 31
-          const uint32_t bit = __fns(gw.fw[i], 0, (int)(k - gw.pre[i] + 1));
-          const uint64_t ch = lo + 32u * i + bit;
-          const unsigned long long so = ch * (unsigned long long)g.C + 16u * sub;
-          sp[u] = p.buf + so;
-          dp[u] = dat + pD + (unsigned long long)k * g.C + 16u * sub;
-          // the buffer's last chunk may be short: units past B copy nothing
-          nb[u] = so >= g.B ? 0u : (g.B - so >= 16 ? 16u : (uint32_t)(g.B - so));
-          if (nb[u] == 16) v[u] = __ldg(reinterpret_cast<const uint4*>(sp[u]));
+      for (int step = 16; step > 0; step >>= 1)
+        if (gw.pre[i + step] <= k) i += step;   // i + step <= 31
+      const uint32_t bit = __fns(gw.fw[i], 0, (int)(k - gw.pre[i] + 1));
+      return (lo + 32u * i + bit) * (unsigned long long)g.C + 16u * sub;
+    };
+    bool entries_done = false;
+    for (uint32_t x0 = 0; x0 < nunits || !entries_done; x0 += kStageUnits) {
+      const uint32_t x1 = nunits - x0 < (uint32_t)kStageUnits ? nunits : x0 + kStageUnits;
+      for (uint32_t x = x0 + lane; x < x1; x += 32) {
+        const unsigned long long so = unit_src(x);
+        if (so < g.B) cp_async16(&gw.stage[x - x0], p.buf + so, g.B - so >= 16 ? 16u : (uint32_t)(g.B - so));
+      }
+      if (!entries_done) {
+        // while the first round is in flight: the tile's offsets and its region entries
+        // (R13): FIRST u32 node; SHIFT u32 node, u32 src node, u32 src ckpt
+        warp_sum3(pF, pS, pD);
+        for (uint32_t i = lane; i < nF + nS; i += 32) {
+          const uint4 r = i < 32 ? rec0 : (i < 64 ? rec1 : __ldg(recs + i));
+          if (i < nF) {
+            *reinterpret_cast<uint32_t*>(ent_f + 4ull * (pF + i)) = r.x;
+          } else {
+            uint32_t* e = reinterpret_cast<uint32_t*>(ent_s + 12ull * (pS + i - nF));
+            e[0] = r.x; e[1] = r.y; e[2] = r.z;
+          }
         }
+        entries_done = true;
       }
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        if (nb[u] == 16) *reinterpret_cast<uint4*>(dp[u]) = v[u];
-        else
-          for (uint32_t b = 0; b < nb[u]; ++b) dp[u][b] = sp[u][b];
+      cp_async_wait_all();
+      __syncwarp();
+      for (uint32_t x = x0 + lane; x < x1; x += 32) {
+        // only the tile's last FIRST chunk, in the tile holding the buffer's end, can be short
+        if (hi == g.n && x / U + 1 == nch && unit_src(x) >= g.B) continue;
+        *reinterpret_cast<uint4*>(dat + pD + 16ull * x) = gw.stage[x - x0];
       }
-    }
-    // region entries (R13): FIRST u32 node; SHIFT u32 node, u32 src node, u32 src ckpt
-    const uint4* recs = p.scratch + (Tcur << g.t0);
-    for (uint32_t i = lane; i < nF; i += 32)
-      *reinterpret_cast<uint32_t*>(ent_f + 4ull * (pF + i)) = __ldg(&recs[i].x);
-    for (uint32_t i = lane; i < nS; i += 32) {
-      const uint4 r = __ldg(recs + nF + i);
-      uint32_t* e = reinterpret_cast<uint32_t*>(ent_s + 12ull * (pS + i));
-      e[0] = r.x; e[1] = r.y; e[2] = r.z;
+      __syncwarp();
     }
     __syncwarp();
     if (p.trace && lane == 0) {
@@ -212,7 +235,7 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
   const int bps = g_gather_blocks_per_sm > 0 ? g_gather_blocks_per_sm : 2;
   uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
   if (grid > (uint64_t)num_sms * bps) grid = (uint64_t)num_sms * bps;
-  return launch_pdl(gather_kernel, (unsigned)grid, kCT, 0, st, p);
+  return launch_pdl(gather_kernel, (unsigned)grid, kCT, kGW * sizeof(GatherWarp), st, p);
 }
 
 
@@ -220,7 +243,10 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
 // launch of each kernel inside the first checkpoint).
 cudaError_t preload_compact() {
   cudaFuncAttributes a;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_gather_blocks_per_sm, gather_kernel, kCT, 0);
+  const int smem = (int)(kGW * sizeof(GatherWarp));
+  cudaError_t e = cudaFuncSetAttribute(gather_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_gather_blocks_per_sm, gather_kernel, kCT, smem);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, gather_kernel);
   return e;
 }
