@@ -355,6 +355,7 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
 // dirty children (the climb target of the tree kernels).
 __device__ void build_tree_work(const InsertParams& p) {
   __shared__ uint32_t s_ws[8], s_carry;
+  const unsigned long long tw0 = p.trace ? gtime_ns() : 0;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const uint64_t nw = (p.n_tiles + 31) / 32;
   if (tid == 0) s_carry = 0;
@@ -384,6 +385,7 @@ __device__ void build_tree_work(const InsertParams& p) {
     __syncthreads();
   }
   if (tid == 0) p.tot->wl_count[0] = s_carry;
+  const unsigned long long tw1 = p.trace ? gtime_ns() : 0;
   // dirty children per group, stage by stage
   for (int s = 1; s < p.S; ++s) {
     // groups of stage s: children are positions of stage s-1 (tiles for s == 1)
@@ -396,7 +398,30 @@ __device__ void build_tree_work(const InsertParams& p) {
     for (uint64_t G = wid; G < ngroups; G += blockDim.x >> 5) {
       uint32_t cnt = 0;
       if (s == 1) {
-        for (uint64_t T = G * per + lane; T < (G + 1) * per; T += 32) cnt += tile_full(p.g, p.tcc, T);
+        const uint32_t q = per / 32;   // tiles per lane
+        if (q >= 4) {
+          // a lane's q consecutive tile counts as 16-byte vectors, up to 8 in flight (one
+          // round trip for a 1024-tile group); only tiles with candidates need their size
+          const uint64_t T0 = G * per + (uint64_t)lane * q;
+          const uint4* src = reinterpret_cast<const uint4*>(p.tcc + T0);
+          for (uint32_t b = 0; b < q / 4; b += 8) {
+            uint4 v[8];
+#pragma unroll
+            for (int u = 0; u < 8; ++u) v[u] = b + u < q / 4 ? __ldcg(src + b + u) : make_uint4(0, 0, 0, 0);
+#pragma unroll
+            for (int u = 0; u < 8; ++u) {
+              const uint32_t c4[4] = {v[u].x, v[u].y, v[u].z, v[u].w};
+#pragma unroll
+              for (int j = 0; j < 4; ++j) {   // branch-free: a tile without candidates never matches
+                uint64_t lo, hi;
+                chunk_range(p.g, p.g.t0, T0 + 4 * (b + u) + j, lo, hi);
+                cnt += (uint64_t)c4[j] == hi - lo;
+              }
+            }
+          }
+        } else {
+          for (uint64_t T = G * per + lane; T < (G + 1) * per; T += 32) cnt += tile_full(p.g, p.tcc, T);
+        }
       } else {
         const uint32_t full = 1u << p.gsz[s - 1];
         for (uint64_t ch = G * per + lane; ch < (G + 1) * per; ch += 32) cnt += __ldcg(p.dcnt[s - 1] + ch) == full;
@@ -407,6 +432,8 @@ __device__ void build_tree_work(const InsertParams& p) {
     }
     __syncthreads();
   }
+  if (p.trace && tid == 0)
+    if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 1)) *r = make_ulonglong4(tw0, tw1, gtime_ns(), 12);
 }
 
 __global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
