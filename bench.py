@@ -25,6 +25,9 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 GiB = 1 << 30
+# BASELINE.json "metric", verbatim: value = box GB/s (all ranks); per_gpu_gbs, hbm_frac_of_measured
+# and diff_ratio carry the other parts of it
+METRIC = "checkpoint de-dup GB/s per GPU & box (1/2/4/8 B200), % HBM peak; diff size ratio"
 
 
 def parse():
@@ -239,7 +242,7 @@ def run_reference(args):
     dt = time.perf_counter() - t0
     val = K * nb / dt / 1e9
     line = {
-        "impl": "reference", "metric": "checkpoint de-dup GB/s", "value": round(val, 4), "unit": "GB/s",
+        "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s",
         "n_gpus": args.gpus, "steps": K, "warmup": Wm, "ms_per_step": round(1e3 * dt / K, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"config{args.config} GDV-like (BASELINE configs[1] recipe)", "buffer_bytes": nb,
@@ -390,7 +393,7 @@ def run_ours(args):
     if rank == 0:
         ratio = sum(B for _ in steady) / max(1, sum(d["bytes"] for d in steady))
         line = {
-            "metric": "checkpoint de-dup GB/s", "value": round(value, 3), "unit": "GB/s", "n_gpus": ws,
+            "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": ws,
             "steps": K, "warmup": Wm, "ms_per_step": round(ms / K, 4), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": {"workload": "config2: 1 GiB GDV-like buffer per GPU (73 x u32 rows), C = 128 B, "

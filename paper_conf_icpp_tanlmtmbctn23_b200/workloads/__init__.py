@@ -159,7 +159,7 @@ def cfg2_mutate(buf: np.ndarray, k: int, seed: int, p: float) -> np.ndarray:
 
 # ------------------------------------------------------------------ config 4
 class DupHeavy:
-    """Duplicate-heavy lineage (config 4), host-only (parity sizes 2^20 / 2^26).
+    """Duplicate-heavy lineage (config 4), host-side (parity sizes 2^20 / 2^26; 1 GiB for tools/sweep.py).
 
     A dictionary of 512 blocks: 75 % have length C·2^j (j in 0..8), 25 % length
     C·m + r (unaligned). The buffer is a sequence of Zipf(1.1) placements; half of the
@@ -183,23 +183,36 @@ class DupHeavy:
         ranks = np.arange(1, self.NBLK + 1, dtype=np.float64)
         pmf = ranks ** -1.1
         self.cdf = np.cumsum(pmf / pmf.sum())
-        # initial item list: long enough to cover 2B of raw length
+        # initial item list: long enough to cover 2B of raw length (draws vectorised in
+        # batches; item p uses H(seed, 5, p) and H(seed, 6, p) exactly as a scalar loop would)
         items = []
-        total, p = 0, 0
+        total, p0 = 0, 0
         while total < 2 * nbytes:
-            u = float(H(seed, 5, p)) / 2.0 ** 64
-            blk = int(min(np.searchsorted(self.cdf, u), self.NBLK - 1))
-            al = bool(self.bpow2[blk]) and (int(H(seed, 6, p)) % 2 == 0)
-            items.append(("d", blk, al))
-            total += int(self.blen[blk])
-            p += 1
+            ps = np.arange(p0, p0 + 65536, dtype=np.uint64)
+            u = H(seed, 5, ps).astype(np.float64) / 2.0 ** 64
+            blks = np.minimum(np.searchsorted(self.cdf, u), self.NBLK - 1)
+            als = self.bpow2[blks] & ((H(seed, 6, ps) % np.uint64(2)) == 0)
+            lens = self.blen[blks]
+            cum = total + np.cumsum(lens)
+            stop = int(np.searchsorted(cum, 2 * nbytes)) + 1 if cum[-1] >= 2 * nbytes else len(ps)
+            items.extend(("d", int(b), bool(a)) for b, a in zip(blks[:stop], als[:stop]))
+            total = int(cum[stop - 1])
+            p0 += 65536
         self.items = items
         self.k = 0
+        self._dict_cache = {}   # dictionary block contents (fixed per block; perf-size lineages)
 
     def _content(self, item) -> np.ndarray:
         if item[0] == "d":
             blk = item[1]
+            c = self._dict_cache.get(blk)
+            if c is not None:
+                return c
             key, ln = H(self.seed, 4, blk), int(self.blen[blk])
+            nw = (ln + 7) // 8
+            c = H(key, np.arange(nw, dtype=np.uint64)).astype("<u8").view(np.uint8)[:ln]
+            self._dict_cache[blk] = c
+            return c
         else:
             _, kk, pp, ln = item
             key = H(self.seed, 11, kk, pp)
@@ -231,15 +244,19 @@ class DupHeavy:
         if self.k > 0:
             k, s, P = self.k, self.seed, len(self.items)
             it = self.items
-            for p in range(0, P - 1, 2):
-                if int(H(s, 7, k, p)) < threshold(0.02):
-                    it[p], it[p + 1] = it[p + 1], it[p]
-            for p in range(P):
-                if int(H(s, 8, k, p)) < threshold(0.01):
+            ps = np.arange(P, dtype=np.uint64)
+            swap = np.nonzero(H(s, 7, k, ps[0:P - 1:2]) < np.uint64(threshold(0.02)))[0] * 2
+            for p in swap.tolist():
+                it[p], it[p + 1] = it[p + 1], it[p]
+            hit8 = H(s, 8, k, ps) < np.uint64(threshold(0.01))
+            hit10 = H(s, 10, k, ps) < np.uint64(threshold(0.002))
+            # sequential in p (a donor may be an item replaced earlier in this pass)
+            for p in np.nonzero(hit8 | hit10)[0].tolist():
+                if hit8[p]:
                     donor = it[int(H(s, 9, k, p)) % P]
                     if donor[0] == "d":
                         it[p] = ("d", donor[1], it[p][2] if it[p][0] == "d" else False)
-                if int(H(s, 10, k, p)) < threshold(0.002):
+                if hit10[p]:
                     it[p] = ("p", k, p, self._len(it[p]))
         self.k += 1
         return self.layout()

@@ -1,0 +1,144 @@
+#!/usr/bin/env python
+"""Measurement sweep over BASELINE.json configs 2-5 on one B200.
+
+    python tools/sweep.py [--only 2,3,4,5] [--out gpurun_out/sweep.json]
+
+Per case: one handle, one device buffer mutated in place between checkpoints (the
+generator runs outside the library's events), per-checkpoint device time from the
+library's CUDA events at profiling level 1 (events around the whole call only, PDL kept).
+Reported: checkpoint 0 separately, steady state = sum_{k>=1} B / sum_{k>=1} t_k (§8(d)),
+diff ratio with and without checkpoint 0, metadata ratio, Tree-vs-List entry
+compaction, and restore(last) == the last input (byte equality on the device).
+
+  cfg2: 1 GiB GDV-like, C = 128, K = 20, p in {0.001, 0.005, 0.01, 0.05}
+  cfg3: 4 GiB GDV-like, p = 0.01, K = 10, C in {32 ... 4096}
+  cfg4: 1 GiB duplicate-heavy (host generator, H2D before each checkpoint), C = 128, K = 50
+  cfg5: 16 GiB GDV-like on one GPU, C = 128, p = 0.01, K = 10 (bench.py --gpus N runs
+        the multi-GPU weak-scaling form at 1 GiB per rank)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+GiB = 1 << 30
+
+
+def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1):
+    import torch
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    seed = W.seed_of(cfg)
+    buf = torch.empty(B, dtype=torch.uint8, device="cuda")
+    ck = Checkpointer(C)
+    ck.set_profiling(prof)
+    diffs, ts, walls, phases = [], [], [], []
+    t_gen = 0.0
+    for k in range(K):
+        g0 = time.perf_counter()
+        with torch.cuda.stream(stream):
+            if host_gen is not None:
+                hb = torch.from_numpy(host_gen.next()).pin_memory()
+                buf.copy_(hb, non_blocking=True)
+            elif k == 0:
+                W.DeviceGen.initial(cfg, buf, B, seed, stream)
+            else:
+                W.DeviceGen.mutate(cfg, buf, B, k, C, seed, p, stream)
+        stream.synchronize()
+        t_gen += time.perf_counter() - g0
+        w0 = time.perf_counter()
+        diffs.append(ck.checkpoint(buf, stream=stream))
+        walls.append(time.perf_counter() - w0)
+        pt = ck.phase_times(k)
+        ts.append(pt["total"])
+        phases.append(pt)
+    out = torch.empty_like(buf)
+    r0 = time.perf_counter()
+    ck.restore(K - 1, out)
+    torch.cuda.synchronize()
+    rs = time.perf_counter() - r0
+    ok = bool(torch.equal(out, buf))
+    del out
+    ck.close()
+    del buf
+    torch.cuda.empty_cache()
+    st = diffs[1:]
+    t_st = ts[1:]
+    sum_b = sum(d["bytes"] for d in diffs)
+    sum_b_st = sum(d["bytes"] for d in st)
+    rec = {
+        "case": name, "config": cfg, "buffer_bytes": B, "chunk_bytes": C, "checkpoints": K, "update_rate": p,
+        "steady_gbs": round((K - 1) * B / (sum(t_st) / 1e3) / 1e9, 1),
+        "steady_ms_median": round(statistics.median(t_st), 4),
+        "steady_ms_min": round(min(t_st), 4), "steady_ms_max": round(max(t_st), 4),
+        "steady_wall_gbs": round((K - 1) * B / sum(walls[1:]) / 1e9, 1),
+        "ckpt0_ms": round(ts[0], 3), "ckpt0_gbs": round(B / (ts[0] / 1e3) / 1e9, 1),
+        "diff_ratio_all": round(K * B / max(1, sum_b), 3),
+        "diff_ratio_steady": round((K - 1) * B / max(1, sum_b_st), 2),
+        "diff_bytes_ckpt0": diffs[0]["bytes"], "diff_bytes_steady_mean": int(sum_b_st / max(1, K - 1)),
+        "meta_over_diff_steady": round(sum(d["meta_bytes"] for d in st) / max(1, sum_b_st), 4),
+        "meta_over_input_steady": round(sum(d["meta_bytes"] for d in st) / ((K - 1) * B), 6),
+        "compaction_vs_list_steady": round(sum(d["list_entries"] for d in st) /
+                                           max(1, sum(d["n_first_regions"] + d["n_shift_regions"] for d in st)), 3),
+        "leaves_steady_mean": {x: int(sum(d[x] for d in st) / max(1, K - 1))
+                               for x in ("n_first", "n_spatial", "n_temporal", "n_fixed")},
+        "regions_steady_mean": {x: int(sum(d[x] for d in st) / max(1, K - 1))
+                                for x in ("n_first_regions", "n_shift_regions")},
+        "record_size": diffs[-1]["record_size"],
+        "restore_last_s": round(rs, 4), "restore_last_gbs": round(B / rs / 1e9, 2), "restore_ok": ok,
+        "gen_s": round(t_gen, 2),
+        "profiling_level": prof,
+    }
+    if prof >= 2:   # events between every kernel (breaks PDL overlap: a breakdown, not a rate)
+        rec["phase_ms_steady_mean"] = {x: round(sum(q[x] for q in phases[1:]) / max(1, K - 1), 4)
+                                       for x in ("leaf_hash", "insert", "phase2", "phase3", "compact", "total")}
+    return rec
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--only", default="2,3,4,5")
+    ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "sweep.json"))
+    ap.add_argument("--small", action="store_true", help="quick shapes (CI / smoke of the tool)")
+    ap.add_argument("--prof", type=int, default=1, help="library profiling level (2: per-phase breakdown)")
+    ap.add_argument("--k", type=int, default=0, help="override the number of checkpoints")
+    a = ap.parse_args()
+    import torch
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    torch.cuda.set_device(0)
+    stream = torch.cuda.Stream()
+    only = {int(x) for x in a.only.split(",")}
+    s = 64 if a.small else 1
+    cases = []
+    if 2 in only:
+        for p in (0.001, 0.005, 0.01, 0.05):
+            cases.append((f"cfg2_p{p}", 2, GiB // s, 128, 20, p, None))
+    if 3 in only:
+        for C in (32, 64, 128, 256, 512, 1024, 2048, 4096):
+            cases.append((f"cfg3_C{C}", 3, 4 * GiB // s, C, 10, 0.01, None))
+    if 4 in only:
+        cases.append(("cfg4_dup_heavy", 4, GiB // s, 128, 50, 0.0, "dup"))
+    if 5 in only:
+        cases.append(("cfg5_16GiB_1gpu", 5, 16 * GiB // s, 128, 10, 0.01, None))
+    recs = []
+    os.makedirs(os.path.dirname(a.out), exist_ok=True)
+    for name, cfg, B, C, K, p, hg in cases:
+        gen = W.DupHeavy(B, C, W.seed_of(cfg)) if hg == "dup" else None
+        r = run_case(name, cfg, B, C, a.k or K, p, stream, gen, a.prof)
+        r["device"] = torch.cuda.get_device_name(0)
+        print(json.dumps(r), flush=True)
+        recs.append(r)
+        with open(a.out, "w") as f:
+            json.dump(recs, f, indent=1)
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())
