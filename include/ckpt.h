@@ -93,7 +93,10 @@ CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes,
 
 /* Rebuild checkpoint `id` into the caller's device buffer ("start from the
  * first-time occurrences, then fill the fixed duplicates and finally assemble the shifted
- * duplicates from the corresponding checkpoint ID") by replaying diffs 0..id (R16).
+ * duplicates from the corresponding checkpoint ID"). Equivalent to replaying diffs 0..id
+ * (R16), computed directly: each chunk is written once, from the newest diff <= id whose
+ * regions cover it. Per-diff restore plans are built by the first
+ * restore that needs them and cached (about 2-3x the diff's metadata in device memory).
  *   dev_ptr  device buffer of B bytes, 16-byte aligned, owned by the caller; overwritten.
  * Synchronous (runs on an internal stream of the handle).
  * Errors: CKPT_ERANGE (id >= number of checkpoints), CKPT_EINVAL, CKPT_ECUDA, CKPT_ESTATE. */

@@ -182,16 +182,24 @@ __device__ __forceinline__ void cas128(Slot* s, unsigned long long cmp_lo, unsig
 
 // Find-or-claim the slot of key d. Safe against concurrent inserters: a plain read is
 // trusted only when it shows a complete key with no all-ones half (a torn read of a
-// slot being claimed always shows one EMPTY half); otherwise the CAS decides.
+// slot being claimed always shows one EMPTY half); otherwise the CAS decides. The value
+// is read in the same round trip (both loads in flight): *val_seen is the slot's value
+// as read when the key was found by the plain read, else kEmpty.
 // Returns the slot index; *claimed = true if this call created the key.
-__device__ __forceinline__ uint64_t table_find_or_claim(Slot* tab, uint64_t cap, const Digest& d, bool* claimed) {
+__device__ __forceinline__ uint64_t table_find_or_claim(Slot* tab, uint64_t cap, const Digest& d, bool* claimed,
+                                                        unsigned long long* val_seen = nullptr) {
   uint64_t s = slot_home(d.lo, cap);
   *claimed = false;
+  if (val_seen) *val_seen = kEmpty;
   for (;;) {
     Slot* p = tab + s;
     unsigned long long lo, hi;
     ld_key_relaxed(p, lo, hi);
-    if (lo == d.lo && hi == d.hi && lo != kEmpty && hi != kEmpty) return s;
+    const unsigned long long v = val_seen ? ld_val_relaxed(p) : kEmpty;
+    if (lo == d.lo && hi == d.hi && lo != kEmpty && hi != kEmpty) {
+      if (val_seen) *val_seen = v;
+      return s;
+    }
     if (lo == kEmpty || hi == kEmpty) {
       unsigned long long olo, ohi;
       cas128(p, kEmpty, kEmpty, d.lo, d.hi, olo, ohi);
@@ -215,12 +223,21 @@ __device__ __forceinline__ uint64_t table_claim_cas(Slot* tab, uint64_t cap, con
   }
 }
 
-// Insert-or-min: Map.insert(digest, entry) of Alg.1 l.7 with the R6 tie-break.
+// Insert-or-min: Map.insert(digest, entry) of Alg.1 l.7 with the R6 tie-break. The value
+// only decreases, so a value already <= packed (an entry of an earlier checkpoint, the
+// common case for temporal duplicates) needs no atomic at all.
 __device__ __forceinline__ uint64_t table_insert_min(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed,
                                                     bool* claimed, bool cas_first = false) {
-  uint64_t s = cas_first ? table_claim_cas(tab, cap, d, claimed) : table_find_or_claim(tab, cap, d, claimed);
+  if (cas_first) {
+    const uint64_t s = table_claim_cas(tab, cap, d, claimed);
+    Slot* p = tab + s;
+    if (*claimed || ld_val_relaxed(p) > packed) atomicMin(&p->val, packed);
+    return s;
+  }
+  unsigned long long seen;
+  const uint64_t s = table_find_or_claim(tab, cap, d, claimed, &seen);
   Slot* p = tab + s;
-  if (*claimed || ld_val_relaxed(p) > packed) atomicMin(&p->val, packed);
+  if (*claimed || seen > packed) atomicMin(&p->val, packed);
   return s;
 }
 

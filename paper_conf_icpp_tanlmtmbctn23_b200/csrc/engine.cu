@@ -28,8 +28,16 @@ namespace {
 struct DiffRec {
   ckpt_diff info;
   uint8_t* ptr;
-  unsigned long long* Flo = nullptr;   // restore caches (lazy)
+  // restore plan (k_restore.cu), built lazily by the first restore that needs it
+  unsigned long long* Flo = nullptr;
   unsigned long long* Foff = nullptr;
+  unsigned long long* Slo = nullptr;
+  unsigned long long* Soff = nullptr;
+  unsigned long long* Ssrc = nullptr;
+  unsigned long long* Fseg = nullptr;
+  unsigned long long* Sseg = nullptr;
+  unsigned long long shift_bytes = 0;
+  bool planned = false;
 };
 
 constexpr double kMaxLoad = 0.8;     // reserve so that even a worst-case checkpoint stays below this
@@ -85,6 +93,15 @@ struct ckpt_ctx {
   std::vector<DiffRec> diffs;
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
+  // restore state (lazy): painter mark per chunk, plan scratch, the chain's plans on device
+  uint32_t* painted = nullptr;
+  unsigned long long* rs_len = nullptr;
+  uint64_t rs_len_cap = 0;
+  void* rs_scan = nullptr;
+  size_t rs_scan_bytes = 0;
+  int* rs_err = nullptr;
+  RestoreDiff* rs_chain = nullptr;
+  uint64_t rs_chain_cap = 0;
   cudaStream_t internal = nullptr;
   uint64_t launches = 0;         // kernels this handle has enqueued (all calls)
   int prof = 0;                  // 0 off, 1 K1 + whole call, 2 every phase
@@ -374,7 +391,11 @@ int ckpt_destroy(ckpt_handle h) {
   cudaDeviceSynchronize();
   for (void* p : h->allocs) cudaFree(p);
   h->arena.release_all();
-  for (auto& d : h->diffs) { if (d.Flo) cudaFree(d.Flo); if (d.Foff) cudaFree(d.Foff); }
+  for (auto& d : h->diffs)
+    for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg})
+      if (q) cudaFree(q);
+  for (void* q : {(void*)h->painted, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
+    if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
   if (h->tot_host) cudaFreeHost(h->tot_host);
   if (h->staging) cudaFree(h->staging);
@@ -517,9 +538,6 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   lp.prev = h->prev;
   lp.cand = h->cand;
   lp.ins = ip;
-  // K1's insert warp overlaps the inserts with the stream but lengthens K1 by about as
-  // much as it saves (measured); it stays available (CKPT_DBG bit 128) and off by default.
-  lp.insert_warp = (k > 0 && (h->dbg & 128)) ? 1 : 0;
   const uint64_t n_full = h->B / h->C;
   if (h->C % 128 == 0) {
     lp.mode3d = 1;
@@ -687,6 +705,105 @@ int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, vo
   return CKPT_OK;
 }
 
+// Restore plans of diffs 0..id (built once per diff, then cached; diffs are immutable).
+static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st) {
+  uint64_t need_len = 1;
+  bool any = false;
+  for (uint32_t c = 0; c <= id; ++c) {
+    const DiffRec& d = h->diffs[c];
+    if (d.planned) continue;
+    any = true;
+    need_len = std::max<uint64_t>(need_len, std::max(d.info.n_first_regions, d.info.n_shift_regions));
+  }
+  if (!any) return CKPT_OK;
+  auto grow = [](void** p, size_t bytes) -> bool {
+    if (*p) cudaFree(*p);
+    *p = nullptr;
+    if (cudaMalloc(p, bytes) != cudaSuccess) { cudaGetLastError(); return false; }
+    return true;
+  };
+  if (h->rs_len_cap < need_len) {
+    if (!grow(reinterpret_cast<void**>(&h->rs_len), need_len * 8)) return CKPT_ENOMEM;
+    h->rs_len_cap = need_len;
+  }
+  const size_t sb = scan_tmp_bytes_for(need_len);
+  if (h->rs_scan_bytes < sb) {
+    if (!grow(&h->rs_scan, sb)) return CKPT_ENOMEM;
+    h->rs_scan_bytes = sb;
+  }
+  if (!h->rs_err && !grow(reinterpret_cast<void**>(&h->rs_err), sizeof(int))) return CKPT_ENOMEM;
+  if (h->rs_chain_cap < h->diffs.size()) {
+    const uint64_t cap = std::max<uint64_t>(64, 2 * h->diffs.size());
+    RestoreDiff* nc = nullptr;
+    if (cudaMalloc(&nc, cap * sizeof(RestoreDiff)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
+    if (h->rs_chain) cudaFree(h->rs_chain);
+    h->rs_chain = nc;
+    h->rs_chain_cap = cap;
+  }
+  if (cudaMemsetAsync(h->rs_err, 0, sizeof(int), st) != cudaSuccess) return CKPT_ECUDA;
+  // FIRST plans first: a SHIFT plan of diff c reads the FIRST plan of its source diff c' <= c
+  std::vector<RestoreDiff> rd(id + 1, RestoreDiff{});
+  for (uint32_t c = 0; c <= id; ++c) {
+    DiffRec& d = h->diffs[c];
+    RestoreDiff& r = rd[c];
+    r.base = d.ptr;
+    r.nF = d.info.n_first_regions;
+    r.nS = d.info.n_shift_regions;
+    r.meta_bytes = d.info.meta_bytes;
+    r.data_bytes = d.info.data_bytes;
+    if (!d.planned) {
+      if ((r.nF && !d.Flo) || (r.nS && !d.Slo)) {
+        if ((r.nF && (cudaMalloc(&d.Flo, r.nF * 8) != cudaSuccess || cudaMalloc(&d.Foff, r.nF * 8) != cudaSuccess)) ||
+            (r.nS && (cudaMalloc(&d.Slo, r.nS * 8) != cudaSuccess || cudaMalloc(&d.Soff, (r.nS + 1) * 8) != cudaSuccess ||
+                      cudaMalloc(&d.Ssrc, r.nS * 8) != cudaSuccess))) {
+          cudaGetLastError();
+          return CKPT_ENOMEM;
+        }
+      }
+    }
+    r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
+    r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
+    if (!d.planned && r.nF && restore_prepare_first(g, r, h->rs_len, h->rs_scan, h->rs_scan_bytes, st) != cudaSuccess)
+      return CKPT_ECUDA;
+  }
+  if (cudaMemcpyAsync(h->rs_chain, rd.data(), rd.size() * sizeof(RestoreDiff), cudaMemcpyHostToDevice, st) != cudaSuccess)
+    return CKPT_ECUDA;
+  for (uint32_t c = 0; c <= id; ++c) {
+    DiffRec& d = h->diffs[c];
+    if (!d.planned && rd[c].nS &&
+        restore_prepare_shift(g, rd[c], h->rs_chain, h->rs_len, h->rs_err, h->rs_scan, h->rs_scan_bytes, st) != cudaSuccess)
+      return CKPT_ECUDA;
+  }
+  // SHIFT stream totals (device scalars) back to the host, then the segment maps
+  std::vector<unsigned long long> shb(id + 1, 0);
+  for (uint32_t c = 0; c <= id; ++c)
+    if (!h->diffs[c].planned && rd[c].nS &&
+        cudaMemcpyAsync(&shb[c], rd[c].Soff + rd[c].nS, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess)
+      return CKPT_ECUDA;
+  int herr = 0;
+  if (cudaMemcpyAsync(&herr, h->rs_err, sizeof(int), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+      cudaStreamSynchronize(st) != cudaSuccess)
+    return CKPT_ECUDA;
+  if (herr) return CKPT_EINVAL;   // malformed chain (a source outside any FIRST region)
+  for (uint32_t c = 0; c <= id; ++c) {
+    DiffRec& d = h->diffs[c];
+    if (d.planned) continue;
+    d.shift_bytes = shb[c];
+    rd[c].shift_bytes = shb[c];
+    if ((rd[c].nF && cudaMalloc(&d.Fseg, (restore_segments(rd[c].data_bytes) + 1) * 8) != cudaSuccess) ||
+        (rd[c].nS && cudaMalloc(&d.Sseg, (restore_segments(shb[c]) + 1) * 8) != cudaSuccess)) {
+      cudaGetLastError();
+      return CKPT_ENOMEM;
+    }
+    rd[c].Fseg = d.Fseg;
+    rd[c].Sseg = d.Sseg;
+    if (restore_segmaps(rd[c], st) != cudaSuccess) return CKPT_ECUDA;
+  }
+  if (cudaStreamSynchronize(st) != cudaSuccess) return CKPT_ECUDA;
+  for (uint32_t c = 0; c <= id; ++c) h->diffs[c].planned = true;
+  return CKPT_OK;
+}
+
 int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
   if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
@@ -694,76 +811,32 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
   LaunchCount lc(h);
   cudaStream_t st = h->internal;
   const Geo g = make_geo(h, id);
-  uint64_t maxF = 1, maxS = 1;
-  for (uint32_t c = 0; c <= id; ++c) {
-    maxF = std::max<uint64_t>(maxF, h->diffs[c].info.n_first_regions);
-    maxS = std::max<uint64_t>(maxS, h->diffs[c].info.n_shift_regions);
+  int rc = ensure_plans(h, id, g, st);
+  if (rc != CKPT_OK) {
+    if (rc == CKPT_ECUDA) h->poisoned = true;
+    return rc;
   }
-  const uint64_t maxN = std::max(maxF, maxS);
-  const size_t scan_bytes = scan_tmp_bytes_for(maxN);
-  unsigned long long *t_len = nullptr, *t_off = nullptr, *t_src = nullptr, *t_dst = nullptr;
-  void* scan_tmp = nullptr;
-  int* err = nullptr;
-  RestoreDiff* chain_dev = nullptr;
-  auto cleanup = [&]() {
-    cudaFree(t_len); cudaFree(t_off); cudaFree(t_src); cudaFree(t_dst);
-    cudaFree(scan_tmp); cudaFree(err); cudaFree(chain_dev);
-  };
-  if (cudaMalloc(&t_len, maxN * 8) != cudaSuccess || cudaMalloc(&t_off, maxN * 8) != cudaSuccess ||
-      cudaMalloc(&t_src, maxN * 8) != cudaSuccess || cudaMalloc(&t_dst, maxN * 8) != cudaSuccess ||
-      cudaMalloc(&scan_tmp, scan_bytes) != cudaSuccess || cudaMalloc(&err, sizeof(int)) != cudaSuccess ||
-      cudaMalloc(&chain_dev, sizeof(RestoreDiff) * (id + 1)) != cudaSuccess) {
-    cudaGetLastError();
-    cleanup();
-    return CKPT_ENOMEM;
+  if (!h->painted) {
+    if (cudaMalloc(&h->painted, h->n * sizeof(uint32_t)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
   }
-  std::vector<RestoreDiff> chain(id + 1);
-  int rc = CKPT_OK;
-  for (uint32_t c = 0; c <= id && rc == CKPT_OK; ++c) {
-    DiffRec& d = h->diffs[c];
-    RestoreDiff& rd = chain[c];
-    rd.base = d.ptr;
-    rd.nF = d.info.n_first_regions;
-    rd.nS = d.info.n_shift_regions;
-    rd.meta_bytes = d.info.meta_bytes;
-    rd.data_bytes = d.info.data_bytes;
-    if (!d.Flo && rd.nF) {
-      if (cudaMalloc(&d.Flo, rd.nF * 8) != cudaSuccess || cudaMalloc(&d.Foff, rd.nF * 8) != cudaSuccess) {
-        cudaGetLastError();
-        rc = CKPT_ENOMEM;
-        break;
-      }
-      rd.Flo = d.Flo;
-      rd.Foff = d.Foff;
-      if (restore_prepare_first(g, rd, t_len, scan_tmp, scan_bytes, st) != cudaSuccess) rc = CKPT_ECUDA;
-    }
-    rd.Flo = d.Flo;
-    rd.Foff = d.Foff;
-  }
-  if (rc == CKPT_OK) {
-    if (cudaMemcpyAsync(chain_dev, chain.data(), sizeof(RestoreDiff) * (id + 1), cudaMemcpyHostToDevice, st) !=
-            cudaSuccess ||
-        cudaMemsetAsync(err, 0, sizeof(int), st) != cudaSuccess || cudaMemsetAsync(dev_ptr, 0, h->B, st) != cudaSuccess)
-      rc = CKPT_ECUDA;
-  }
+  // newest diff first; a chunk is written by the newest diff whose regions cover it
+  // (diff 0 covers every chunk, so the target needs no clearing)
+  CK(cudaMemsetAsync(h->painted, 0, h->n * sizeof(uint32_t), st));
   uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
-  for (uint32_t c = 0; c <= id && rc == CKPT_OK; ++c) {
-    // first-time occurrences, then (implicitly) fixed, then shifted duplicates
-    if (restore_copy_first(g, chain[c], outp, h->num_sms, st) != cudaSuccess) rc = CKPT_ECUDA;
-    else if (restore_shift(g, chain[c], chain_dev, outp, t_len, t_off, t_src, t_dst, err, scan_tmp, scan_bytes,
-                           h->num_sms, st) != cudaSuccess)
-      rc = CKPT_ECUDA;
+  for (int64_t c = id; c >= 0; --c) {
+    const DiffRec& d = h->diffs[c];
+    RestoreDiff r;
+    r.base = d.ptr;
+    r.nF = d.info.n_first_regions;
+    r.nS = d.info.n_shift_regions;
+    r.meta_bytes = d.info.meta_bytes;
+    r.data_bytes = d.info.data_bytes;
+    r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
+    r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
+    CK(restore_paint(g, r, outp, h->painted, (uint32_t)c + 1u, h->num_sms, st));
   }
-  int herr = 0;
-  if (rc == CKPT_OK) {
-    if (cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-        cudaStreamSynchronize(st) != cudaSuccess)
-      rc = CKPT_ECUDA;
-  }
-  cleanup();
-  if (rc == CKPT_ECUDA) h->poisoned = true;
-  if (rc == CKPT_OK && herr) rc = CKPT_EINVAL;   // malformed chain (a source outside any FIRST region)
-  return rc;
+  CK(cudaStreamSynchronize(st));
+  return CKPT_OK;
 }
 
 int ckpt_leaf_digests(ckpt_handle h, void* dev_out) {

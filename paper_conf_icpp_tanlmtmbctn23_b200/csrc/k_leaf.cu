@@ -27,6 +27,7 @@ __device__ __forceinline__ bool leaf_is_candidate(const Geo& g, const Digest& d,
 }
 
 // ------------------------------------------------------------------ record insert
+constexpr uint32_t kDenseTile = 64;   // candidates per 256-chunk tile above which inserts read first
 // Map.insert(digest, (leaf, chkptID)) for the candidates of one 256-chunk leaf tile
 // (Alg.1 l.6-19), by one warp: lane i < 8 holds candidate word i. The candidates are
 // spread evenly over the lanes (prefix over popcounts, __fns), identical digests within a
@@ -78,8 +79,11 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
       uint32_t slot = 0;
       if (lane == leader) {
         bool claimed;
-        // checkpoint 0 is full of hot repeated keys (read first); later ones mostly insert new keys (CAS first)
-        slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed, p.g.k > 0);
+        // Sparse candidates after checkpoint 0 are mostly new keys (CAS first: one round trip).
+        // Checkpoint 0 and dense tiles (moved or repeated content) mostly hit existing keys:
+        // read key + value first, no atomic when the entry is older (one round trip).
+        slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed,
+                                          p.g.k > 0 && total < kDenseTile);
       }
       slot = __shfl_sync(active, slot, leader);
       st_evict_last_u32(p.slot_of + c, slot, pol);
@@ -130,20 +134,25 @@ __device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile,
 }
 
 // ------------------------------------------------------------------ K1
-// 8 hashing warps + 1 insert warp. A finished tile's 8 candidate words go through a small
-// shared-memory ring to the insert warp, which runs the record inserts while the hashing
-// warps keep streaming; when the ring is full (or at checkpoint 0, when every chunk is a
-// candidate) the tile is deferred to K1b instead, so the stream never waits on inserts.
-constexpr int kRing = 16;
+// 8 hashing (consumer) warps + 1 producer warp. The producer streams the stages with TMA
+// (full barriers, complete_tx) and re-fills a stage as soon as all 8 consumer warps have
+// released it (empty barriers, one arrive per warp): fast warps never wait for slow ones
+// at a CTA barrier, they run ahead into the next filled stage. At the end of a 256-chunk
+// tile each consumer warp leaves its candidate ballot word in the stage's slot; the
+// producer, on the stage's release, marks the tree tile(s) dirty and defers the tile's
+// inserts to K1b, so that bookkeeping is off the hashing warps' path.
 constexpr int kK1Threads = kLeafThreads + 32;
+constexpr int kMaxStagesK1 = 8;
 
-struct K1Ring {
-  uint32_t words[kRing][8];
-  uint32_t tile[kRing];
-  uint32_t stage_words[2][8];
-  uint32_t s_word[32], s_excl[32];
-  volatile uint32_t head, tail, done;
+struct K1Shared {
+  uint64_t full[kMaxStagesK1];
+  uint64_t empty[kMaxStagesK1];
+  uint32_t words[kMaxStagesK1][8];   // candidate ballot words of the tile ending in the stage
 };
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
 
 template <int MODE3D>
 __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
@@ -154,8 +163,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
   const int nst = p.nst;
   const uint32_t stage_bytes = p.stage_bytes;
   Digest* const prevbuf = reinterpret_cast<Digest*>(data + nst * stage_bytes);   // nst * 256 digests
-  uint64_t* const bars = reinterpret_cast<uint64_t*>(prevbuf + nst * kLeafThreads);
-  K1Ring& ring = *reinterpret_cast<K1Ring*>(bars + 8);
+  K1Shared& sh = *reinterpret_cast<K1Shared*>(prevbuf + nst * kLeafThreads);
 
   const unsigned long long bt0 = p.ins.trace ? gtime_ns() : 0;
   const int tid = threadIdx.x;
@@ -167,71 +175,67 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
 
   if (tid == 0) {
     prefetch_tmap(&tmap);
-    for (int s = 0; s < nst; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < nst; ++s) {
+      mbar_init(&sh.full[s], 1);
+      mbar_init(&sh.empty[s], kLeafThreads / 32);
+    }
     fence_mbar_init();
-    ring.head = 0;
-    ring.tail = 0;
-    ring.done = 0;
   }
   __syncthreads();
 
   if (tid >= kLeafThreads) {
-    // ---------------- insert warp
-    const int lane = tid & 31;
-    unsigned long long ncand = 0;
-    uint32_t head = 0;
-    for (;;) {
-      const uint32_t t = ring.tail;
-      if (head == t) {
-        if (ring.done && head == ring.tail) break;
-        __nanosleep(128);
-        continue;
+    // ---------------- producer warp (lane 0)
+    if (tid != kLeafThreads) return;
+    const uint64_t pol_stream = policy_evict_first();
+    // the tile epilogue of step i (consumed from stage i % nst): dirty marks + deferral
+    auto epilogue = [&](uint32_t i) {
+      if ((int)(i % (uint32_t)segs) != segs - 1) return;
+      const uint32_t tile = blockIdx.x + (i / (uint32_t)segs) * gridDim.x;
+      const int s = (int)(i % (uint32_t)nst);
+      uint32_t w[8], any = 0, pc = 0;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) { w[q] = sh.words[s][q]; any |= w[q]; pc += __popc(w[q]); }
+      if (any) {
+        mark_tree_dirty(p.ins, tile, w);
+        defer_tile(p.ins, tile, pc);
       }
-      __threadfence_block();
-      const uint32_t slot = head % kRing;
-      const uint32_t tile = ring.tile[slot];
-      const uint32_t word = lane < 8 ? ring.words[slot][lane] : 0u;
-      __syncwarp();
-      insert_tile(p.ins, tile, word, ring.s_word, ring.s_excl, ncand);
-      ++head;
-      __syncwarp();
-      if (lane == 0) ring.head = head;
+    };
+    for (uint32_t i = 0; i < total; ++i) {
+      const int s = (int)(i % (uint32_t)nst);
+      if (i >= (uint32_t)nst) {
+        mbar_wait(&sh.empty[s], ((i / nst) - 1) & 1u);   // all consumer warps released step i - nst
+        epilogue(i - nst);
+      }
+      const uint32_t tile = blockIdx.x + (i / (uint32_t)segs) * gridDim.x;
+      const int seg = (int)(i % (uint32_t)segs);
+      const bool with_prev = use_prev && seg == segs - 1;
+      mbar_arrive_expect_tx(&sh.full[s], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
+      if (MODE3D)
+        tma_load_3d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, seg, (int)(tile * kLeafThreads), pol_stream);
+      else
+        tma_load_2d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, (int)(tile * (stage_bytes / 128)), pol_stream);
+      if (with_prev)
+        bulk_load(prevbuf + s * kLeafThreads, p.prev + (uint64_t)tile * kLeafThreads, kLeafThreads * 16u, &sh.full[s],
+                  pol_stream);
     }
-    if (lane == 0 && ncand) atomicAdd(&p.ins.tot->n_cand, ncand);
+    const uint32_t first_tail = total > (uint32_t)nst ? total - nst : 0;
+    for (uint32_t i = first_tail; i < total; ++i) {
+      mbar_wait(&sh.empty[i % nst], (i / nst) & 1u);
+      epilogue(i);
+    }
     return;
   }
 
-  // ---------------- hashing warps (named barrier 1 over 256 threads)
-  int is_st = 0, is_seg = 0;
-  uint32_t is_tile = blockIdx.x, issued = 0;
-  const uint64_t pol_stream = policy_evict_first();
+  // ---------------- consumer (hashing) warps
   const uint64_t pol_keep = policy_evict_last();
-  auto issue_next = [&]() {
-    const bool with_prev = use_prev && is_seg == segs - 1;
-    mbar_arrive_expect_tx(&bars[is_st], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
-    if (MODE3D)
-      tma_load_3d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, is_seg, (int)(is_tile * kLeafThreads),
-                  pol_stream);
-    else
-      tma_load_2d(data + (size_t)is_st * stage_bytes, &tmap, &bars[is_st], 0, (int)(is_tile * (stage_bytes / 128)),
-                  pol_stream);
-    if (with_prev)
-      bulk_load(prevbuf + is_st * kLeafThreads, p.prev + (uint64_t)is_tile * kLeafThreads, kLeafThreads * 16u, &bars[is_st],
-                pol_stream);
-    ++issued;
-    if (++is_st == nst) is_st = 0;
-    if (++is_seg == segs) { is_seg = 0; is_tile += gridDim.x; }
-  };
-  if (tid == 0)
-    while (issued < (uint32_t)nst && issued < total) issue_next();
-
   const int units = MODE3D ? 8 : (int)(p.g.C / 16);   // 16-byte blocks of this thread per stage
   const uint32_t ubase = (uint32_t)tid * (uint32_t)units;
+  const int lane = tid & 31, wid = tid >> 5;
   uint64_t h1 = 0, h2 = 0;
   int st = 0, seg = 0;
-  uint32_t phase = 0, tile = blockIdx.x, ntile_done = 0;
+  uint32_t phase = 0, tile = blockIdx.x;
   for (uint32_t step = 0; step < total; ++step) {
-    mbar_wait(&bars[st], phase);
+    mbar_wait(&sh.full[st], phase);
     if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
     const uint8_t* sd = data + (size_t)st * stage_bytes;
 #pragma unroll 8
@@ -242,17 +246,16 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
       const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + off);
       mm::block(h1, h2, v.x, v.y);
     }
-    const bool tile_end = (seg == segs - 1);
-    if (tile_end) {
+    if (seg == segs - 1) {
       const Digest d = mm::finish(h1, h2, p.g.C);
       const uint64_t c = (uint64_t)tile * kLeafThreads + tid;
       Digest pd{0, 0};
       if (use_prev) pd = prevbuf[st * kLeafThreads + tid];
       const bool cand = leaf_is_candidate(p.g, d, pd);
       const unsigned mask = __ballot_sync(0xffffffffu, cand);
-      if ((tid & 31) == 0) {
+      if (lane == 0) {
         st_evict_last_u32(p.cand + (c >> 5), mask, pol_keep);
-        ring.stage_words[ntile_done & 1][tid >> 5] = mask;
+        sh.words[st][wid] = mask;
       }
       if (cand) {
         st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
@@ -262,36 +265,10 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
         for (uint32_t o = 0; o < p.g.C; o += 128) l2_keep_line(cp + o);
       }
     }
-    asm volatile("bar.sync 1, %0;" ::"n"(kLeafThreads) : "memory");   // every hashing thread is done with stage st
-    if (tid == 0) {
-      if (tile_end) {
-        // hand the tile's candidate words to the insert warp, or defer them to K1b
-        uint32_t w[8], any = 0, pc = 0;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) { w[i] = ring.stage_words[ntile_done & 1][i]; any |= w[i]; pc += __popc(w[i]); }
-        if (any) {
-          mark_tree_dirty(p.ins, tile, w);
-          const uint32_t t = ring.tail;
-          if (p.insert_warp && t - ring.head < (uint32_t)kRing) {
-#pragma unroll
-            for (int i = 0; i < 8; ++i) ring.words[t % kRing][i] = w[i];
-            ring.tile[t % kRing] = tile;
-            __threadfence_block();
-            ring.tail = t + 1;
-          } else {
-            defer_tile(p.ins, tile, pc);
-          }
-        }
-      }
-      if (issued < total) issue_next();
-    }
-    if (tile_end) ++ntile_done;
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&sh.empty[st]);   // this warp is done with stage st
     if (++st == nst) { st = 0; phase ^= 1u; }
     if (++seg == segs) { seg = 0; tile += gridDim.x; }
-  }
-  if (tid == 0) {
-    __threadfence_block();
-    ring.done = 1;
   }
   trace_block(p.ins.trace, p.ins.trace_n, bt0, bt0, 0);
 }
@@ -488,7 +465,7 @@ __global__ void rehash_kernel(const Slot* old_tab, uint64_t old_cap, Slot* new_t
 
 // ------------------------------------------------------------------ launchers
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes) {
-  *smem_bytes = 1008 + (size_t)p.nst * p.stage_bytes + (size_t)p.nst * kLeafThreads * 16 + 64 + sizeof(K1Ring);
+  *smem_bytes = 1008 + (size_t)p.nst * p.stage_bytes + (size_t)p.nst * kLeafThreads * 16 + sizeof(K1Shared);
   return cudaSuccess;
 }
 
@@ -513,17 +490,21 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+static int g_insert_blocks_per_sm = 0;
+
 cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st) {
   const uint64_t tiles = (p.nwords + 7) / 8;
   uint64_t blocks = (tiles + 7) / 8 + 1;   // + block 0: tree work description
-  if (blocks > (uint64_t)num_sms * 8) blocks = (uint64_t)num_sms * 8;
+  // one resident wave: the deferred work is strided statically over the warps
+  const uint64_t wave = (uint64_t)num_sms * (g_insert_blocks_per_sm > 0 ? g_insert_blocks_per_sm : 4);
+  if (blocks > wave) blocks = wave;
   if (blocks) return launch_pdl(insert_kernel, (unsigned)blocks, 256, 0, st, p);
   return cudaSuccess;
 }
 
 cudaError_t leaf_setup_attributes() {
   // the largest dynamic smem any leaf configuration asks for (C >= 128: 3 x 36 KB; C < 128: <= 96 KB)
-  const int smem = 1008 + 3 * (32768 + 4096) + 64 + (int)sizeof(K1Ring);   // the largest leaf configuration
+  const int smem = 1008 + 3 * (32768 + 4096) + (int)sizeof(K1Shared);   // the largest leaf configuration
   cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;
@@ -549,6 +530,7 @@ cudaError_t preload_leaf() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<1>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_tail_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, insert_kernel);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_insert_blocks_per_sm, insert_kernel, 256, 0);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, rehash_kernel);
   return e;
 }

@@ -1,19 +1,29 @@
-// k_restore.cu — restore scatter (reading R16).
+// k_restore.cu — restore scatter (reading R16), direct form.
 //
 // "To restore a checkpoint from the differences, it is enough to start from the
 // first-time occurrences, then fill the fixed duplicates and finally assemble the
 // shifted duplicates from the corresponding checkpoint ID (which can be a previous
-// checkpoint or the current checkpoint to be restored)". The engine replays
-// diffs 0..id into the caller's buffer; per diff c:
-//   prepare_first: FIRST region i -> (first chunk, byte length); exclusive scan of the
-//                  lengths = offsets in c's data section (kept for later diffs).
-//   copy_first   : the data section streamed to its regions, warp per 8-KiB segment.
-//   prepare_shift: SHIFT (u, v, c') -> (dst offset, length, source address) where the
-//                  source is v's bytes inside the FIRST region of diff c' holding v's
-//                  first chunk (binary search over c''s sorted region starts).
-//   copy_shift   : the virtual concatenation of the SHIFT regions, same streaming.
-// FIXED chunks are simply left as diff c-1's replay wrote them.
+// checkpoint or the current checkpoint to be restored)".
+//
+// Replaying diffs 0..id writes every chunk once per diff that touches it, and the LAST
+// such diff wins: a FIXED chunk of diff c keeps what an earlier diff wrote. So the result
+// is, per chunk, the bytes of the latest diff c <= id whose regions cover it, and every
+// chunk is covered by diff 0 (no FIXED leaf at checkpoint 0, R5). The restore therefore
+// PAINTS diffs newest first: diff c writes a chunk only if no later diff painted it
+// (painted[chunk] holds c+1 of its painter), so every output byte is written exactly once
+// and FIXED chunks cost nothing — B bytes written, B bytes read, plus one 4-byte mark per
+// chunk, instead of one full copy per diff.
+//
+// Per diff, a restore plan is built once and cached (diffs are immutable):
+//   FIRST: Flo[r] (first chunk of region r), Foff[r] (its offset in the data section)
+//   SHIFT: Slo[r] (first chunk), Soff[r] (exclusive scan of byte lengths, Soff[nS] = total),
+//          Ssrc[r] (device address of the source bytes: v's bytes inside the FIRST region of
+//          diff c' holding v's first chunk, binary search over c''s sorted region starts)
+// paint_kernel streams a diff's FIRST bytes then its SHIFT bytes in 2-KB segments, one
+// warp per segment; the regions of a segment are located once per segment (two binary
+// searches) and their offsets staged in shared memory.
 #include "kernels.h"
+#include "tma.cuh"
 
 namespace ckpt {
 
@@ -21,7 +31,6 @@ namespace {
 constexpr int kRT = 256;
 constexpr int kScanPer = 4;
 constexpr uint64_t kScanBlock = kRT * kScanPer;   // 1024 elements per scan block
-constexpr unsigned long long kSeg = 8192;
 
 __device__ __forceinline__ void node_range(const Geo& g, uint32_t node, uint64_t& lo, uint64_t& hi) {
   const int depth = 31 - __clz(node + 1);
@@ -77,58 +86,119 @@ __global__ void prepare_first_kernel(Geo g, RestoreDiff d, unsigned long long* l
   len[i] = range_bytes(g, lo, hi);
 }
 
-// stream `total` bytes laid out as consecutive regions (offsets off[0..nr), sorted) to
-// dst + dst_off(r) + (o - off[r]) from src(r) + (o - off[r]).
-template <bool FIRST>
-__global__ void __launch_bounds__(kRT) copy_stream_kernel(Geo g, RestoreDiff d, uint8_t* out,
-                                                          const unsigned long long* off, const unsigned long long* len,
-                                                          const unsigned long long* srcaddr,
-                                                          const unsigned long long* dstoff, uint64_t nr,
-                                                          unsigned long long total_known) {
-  if (nr == 0) return;
-  const unsigned long long total = FIRST ? total_known : off[nr - 1] + len[nr - 1];
+constexpr uint32_t kPaintSeg = 2048;                 // bytes per warp segment
+constexpr uint32_t kPaintUnits = kPaintSeg / 16 / 32;   // 16-B units per lane per segment (4)
+constexpr uint32_t kPaintSlots = kPaintSeg / 32 + 3;    // regions per segment (C >= 32), tail, next start
+constexpr int kPaintWarps = kRT / 32;
+
+// first index r in [0, nr) with off[r] > x, minus one (off[0] == 0 <= x)
+__device__ __forceinline__ uint64_t region_at(const unsigned long long* off, uint64_t nr, unsigned long long x) {
+  uint64_t lo = 0, hi = nr;
+  while (hi - lo > 1) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (__ldg(off + mid) <= x) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void __launch_bounds__(kRT, 4) paint_kernel(Geo g, RestoreDiff d, uint8_t* out, uint32_t* painted,
+                                                   uint32_t mark) {
+  __shared__ unsigned long long s_off[kPaintWarps][kPaintSlots + 1];
+  pdl_launch_dependents();
+  pdl_wait();   // the previous (newer) diff's marks are complete
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  unsigned long long* so = s_off[wid];
   const uint8_t* data = d.base + d.meta_bytes;
-  const int lane = threadIdx.x & 31;
-  const unsigned long long nseg = (total + kSeg - 1) / kSeg;
-  const unsigned long long wg = ((unsigned long long)blockIdx.x * kRT + threadIdx.x) >> 5;
-  const unsigned long long nw = ((unsigned long long)gridDim.x * kRT) >> 5;
-  for (unsigned long long sg = wg; sg < nseg; sg += nw) {
-    const unsigned long long s0 = sg * kSeg;
-    unsigned long long lo = 0, hi = nr;
-    while (hi - lo > 1) {
-      const unsigned long long mid = (lo + hi) >> 1;
-      if (off[mid] <= s0) lo = mid; else hi = mid;
+  const unsigned long long totF = d.data_bytes;
+  const unsigned long long totS = d.shift_bytes;
+  const uint64_t nsegF = (totF + kPaintSeg - 1) / kPaintSeg, nsegS = (totS + kPaintSeg - 1) / kPaintSeg;
+  const uint32_t U = g.C / 16;   // units per chunk
+  const uint64_t nw = ((uint64_t)gridDim.x * kRT) >> 5;
+  for (uint64_t sg = ((uint64_t)blockIdx.x * kRT + threadIdx.x) >> 5; sg < nsegF + nsegS; sg += nw) {
+    const bool first = sg < nsegF;
+    const unsigned long long* off = first ? d.Foff : d.Soff;
+    const uint64_t nr = first ? d.nF : d.nS;
+    const unsigned long long total = first ? totF : totS;
+    const unsigned long long s0 = (first ? sg : sg - nsegF) * kPaintSeg;
+    const unsigned long long s1 = s0 + kPaintSeg < total ? s0 + kPaintSeg : total;
+    // regions of the segment: from the region holding its first byte (cached segment map)
+    // to the region holding the next segment's first byte (one extra slot at most)
+    const unsigned long long* segmap = first ? d.Fseg : d.Sseg;
+    const uint64_t sl = first ? sg : sg - nsegF;
+    const uint64_t r0 = __ldg(segmap + sl), r1 = __ldg(segmap + sl + 1);
+    const uint32_t nloc = (uint32_t)(r1 - r0 + 1);   // <= kPaintSlots (regions are >= 32 B but the last)
+    for (uint32_t i = lane; i <= nloc; i += 32) so[i] = (r0 + i < nr) ? __ldg(off + r0 + i) : total;
+    __syncwarp();
+    // units of this lane: o_j = s0 + 16 (lane + 32 j). Loads are issued in batches across
+    // the 8 units (region fields, then the painter marks, then the bytes) before any store.
+    uint32_t loc[kPaintUnits];
+    unsigned long long clo[kPaintUnits], sbase[kPaintUnits];
+#pragma unroll
+    for (uint32_t j = 0; j < kPaintUnits; ++j) {
+      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
+      uint32_t lo = 0, hi = nloc;   // last local region with so[lo] <= o
+      while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (so[mid] <= o) lo = mid; else hi = mid;
+      }
+      loc[j] = o < s1 ? lo : ~0u;
     }
-    unsigned long long r = lo;
-    unsigned long long next = (r + 1 < nr) ? off[r + 1] : ~0ull;
-    const unsigned long long send = (s0 + kSeg < total) ? s0 + kSeg : total;
-    for (unsigned long long o = s0 + 16ull * lane; o < send; o += 512) {
-      while (o >= next) {
-        ++r;
-        next = (r + 1 < nr) ? off[r + 1] : ~0ull;
-      }
-      const unsigned long long rel = o - off[r];
-      const uint8_t* s;
-      uint8_t* t;
-      if (FIRST) {
-        s = data + o;
-        t = out + d.Flo[r] * (unsigned long long)g.C + rel;
+#pragma unroll
+    for (uint32_t j = 0; j < kPaintUnits; ++j) {
+      if (loc[j] == ~0u) continue;
+      const uint64_t rr = r0 + loc[j];
+      clo[j] = first ? __ldg(d.Flo + rr) : __ldg(d.Slo + rr);
+      sbase[j] = first ? 0ull : __ldg(d.Ssrc + rr);
+    }
+    uint64_t chk[kPaintUnits];
+    uint32_t mk[kPaintUnits];
+#pragma unroll
+    for (uint32_t j = 0; j < kPaintUnits; ++j) {
+      if (loc[j] == ~0u) continue;
+      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
+      const uint32_t ur = (uint32_t)((o - so[loc[j]]) >> 4);
+      chk[j] = clo[j] + ur / U;
+      mk[j] = __ldcg(painted + chk[j]);
+    }
+    uint4 v[kPaintUnits];
+    uint32_t len[kPaintUnits];
+    uint32_t setmark = 0;   // bit j: unit j starts a chunk this diff paints
+#pragma unroll
+    for (uint32_t j = 0; j < kPaintUnits; ++j) {
+      len[j] = 0;
+      if (loc[j] == ~0u || mk[j] > mark) continue;   // a newer diff painted this chunk
+      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
+      const unsigned long long rel = o - so[loc[j]];
+      const unsigned long long rem = so[loc[j] + 1] - o;
+      len[j] = rem >= 16 ? 16u : (uint32_t)rem;
+      if ((rel >> 4) % U == 0) setmark |= 1u << j;
+      const uint8_t* src = first ? data + o : reinterpret_cast<const uint8_t*>(sbase[j]) + rel;
+      if (len[j] == 16) {
+        v[j] = __ldg(reinterpret_cast<const uint4*>(src));
       } else {
-        s = reinterpret_cast<const uint8_t*>(srcaddr[r]) + rel;
-        t = out + dstoff[r] + rel;
-      }
-      const unsigned long long rem = (r + 1 < nr ? off[r + 1] : total) - o;
-      if (rem >= 16) {
-        *reinterpret_cast<uint4*>(t) = *reinterpret_cast<const uint4*>(s);
-      } else {
-        for (unsigned long long b = 0; b < rem; ++b) t[b] = s[b];
+        uint32_t w[4] = {0, 0, 0, 0};
+        for (uint32_t q = 0; q < len[j]; ++q) w[q >> 2] |= (uint32_t)src[q] << (8 * (q & 3));
+        v[j] = make_uint4(w[0], w[1], w[2], w[3]);
       }
     }
+#pragma unroll
+    for (uint32_t j = 0; j < kPaintUnits; ++j) {
+      if (!len[j]) continue;
+      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
+      uint8_t* dst = out + clo[j] * (unsigned long long)g.C + (o - so[loc[j]]);
+      if (len[j] == 16) {
+        *reinterpret_cast<uint4*>(dst) = v[j];
+      } else {
+        const uint32_t w[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
+        for (uint32_t q = 0; q < len[j]; ++q) dst[q] = (uint8_t)(w[q >> 2] >> (8 * (q & 3)));
+      }
+      if ((setmark >> j) & 1u) painted[chk[j]] = mark;
+    }
+    __syncwarp();
   }
 }
 
-__global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* chain, unsigned long long* len,
-                                     unsigned long long* srcaddr, unsigned long long* dstoff, int* err) {
+__global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* chain, unsigned long long* len, int* err) {
   const uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= d.nS) return;
   const uint8_t* e = d.base + 64 + 4 * d.nF + 12 * i;
@@ -136,17 +206,28 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
   uint64_t ulo, uhi, vlo, vhi;
   node_range(g, u, ulo, uhi);
   node_range(g, v, vlo, vhi);
+  len[i] = range_bytes(g, ulo, uhi);
+  d.Slo[i] = ulo;
   const RestoreDiff& s = chain[c2];
   // FIRST region r of diff c2 with Flo[r] <= vlo (the last such): it contains v
+  if (s.nF == 0 || !s.Flo) { atomicExch(err, 1); d.Ssrc[i] = (unsigned long long)s.base; return; }
   uint64_t lo = 0, hi = s.nF;
-  if (s.nF == 0) { atomicExch(err, 1); len[i] = 0; srcaddr[i] = 0; dstoff[i] = 0; return; }
   while (hi - lo > 1) {
     const uint64_t mid = (lo + hi) >> 1;
     if (s.Flo[mid] <= vlo) lo = mid; else hi = mid;
   }
-  len[i] = range_bytes(g, ulo, uhi);
-  dstoff[i] = ulo * (unsigned long long)g.C;
-  srcaddr[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + (vlo - s.Flo[lo]) * (unsigned long long)g.C);
+  d.Ssrc[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + (vlo - s.Flo[lo]) * (unsigned long long)g.C);
+}
+
+// segment map: region holding the first byte of each 2-KB segment; map[nseg] = nr - 1
+__global__ void segmap_kernel(const unsigned long long* off, uint64_t nr, uint64_t nseg, unsigned long long* map) {
+  const uint64_t sg = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (sg > nseg) return;
+  map[sg] = sg == nseg ? nr - 1 : region_at(off, nr, sg * (unsigned long long)kPaintSeg);
+}
+
+__global__ void write_total_kernel(unsigned long long* off, const unsigned long long* len, uint64_t n) {
+  off[n] = off[n - 1] + len[n - 1];
 }
 }  // namespace
 
@@ -191,26 +272,38 @@ cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long lo
   return scan_u64_exclusive(tmp_len, d.Foff, d.nF, scan_tmp, scan_tmp_bytes, st);
 }
 
-cudaError_t restore_copy_first(const Geo& g, const RestoreDiff& d, uint8_t* out, int num_sms, cudaStream_t st) {
-  if (d.nF == 0) return cudaSuccess;
-  copy_stream_kernel<true><<<num_sms * 8, kRT, 0, st>>>(g, d, out, d.Foff, nullptr, nullptr, nullptr, d.nF,
-                                                       d.data_bytes);
+cudaError_t restore_prepare_shift(const Geo& g, RestoreDiff& d, const RestoreDiff* chain_dev, unsigned long long* tmp_len,
+                                  int* err, void* scan_tmp, size_t scan_tmp_bytes, cudaStream_t st) {
+  if (d.nS == 0) return cudaSuccess;
+  prepare_shift_kernel<<<(unsigned)((d.nS + 255) / 256), 256, 0, st>>>(g, d, chain_dev, tmp_len, err);
+  note_launch();
+  cudaError_t e = scan_u64_exclusive(tmp_len, d.Soff, d.nS, scan_tmp, scan_tmp_bytes, st);
+  if (e != cudaSuccess) return e;
+  write_total_kernel<<<1, 1, 0, st>>>(d.Soff, tmp_len, d.nS);
   note_launch();
   return cudaGetLastError();
 }
 
-cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, uint8_t* out,
-                          unsigned long long* t_len, unsigned long long* t_off, unsigned long long* t_src,
-                          unsigned long long* t_dst, int* err, void* scan_tmp, size_t scan_tmp_bytes, int num_sms,
-                          cudaStream_t st) {
-  if (d.nS == 0) return cudaSuccess;
-  prepare_shift_kernel<<<(unsigned)((d.nS + 255) / 256), 256, 0, st>>>(g, d, chain_dev, t_len, t_src, t_dst, err);
-  note_launch();
-  cudaError_t e = scan_u64_exclusive(t_len, t_off, d.nS, scan_tmp, scan_tmp_bytes, st);
-  if (e != cudaSuccess) return e;
-  copy_stream_kernel<false><<<num_sms * 8, kRT, 0, st>>>(g, d, out, t_off, t_len, t_src, t_dst, d.nS, 0);
-  note_launch();
+cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st) {
+  if (d.nF) {
+    const uint64_t ns = (d.data_bytes + kPaintSeg - 1) / kPaintSeg;
+    segmap_kernel<<<(unsigned)((ns + 256) / 256), 256, 0, st>>>(d.Foff, d.nF, ns, d.Fseg);
+    note_launch();
+  }
+  if (d.nS) {
+    const uint64_t ns = (d.shift_bytes + kPaintSeg - 1) / kPaintSeg;
+    segmap_kernel<<<(unsigned)((ns + 256) / 256), 256, 0, st>>>(d.Soff, d.nS, ns, d.Sseg);
+    note_launch();
+  }
   return cudaGetLastError();
+}
+
+uint64_t restore_segments(uint64_t bytes) { return (bytes + kPaintSeg - 1) / kPaintSeg; }
+
+cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
+                          int num_sms, cudaStream_t st) {
+  if (d.nF == 0 && d.nS == 0) return cudaSuccess;
+  return launch_pdl(paint_kernel, (unsigned)(num_sms * 4), kRT, 0, st, g, d, out, painted, mark);
 }
 
 
@@ -222,9 +315,10 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_block_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_add_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_first_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_stream_kernel<true>);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_stream_kernel<false>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, paint_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_shift_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, write_total_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, segmap_kernel);
   return e;
 }
 

@@ -69,8 +69,7 @@ struct LeafParams {
   int nst;               // pipeline stages
   Digest* prev;          // persistent leaf digests Tree(leaf), 16 n bytes
   uint32_t* cand;        // candidate (non-FIXED) bit per chunk
-  int insert_warp;       // 1: K1's insert warp performs the record inserts (k > 0)
-  InsertParams ins;      // record insert state (K1's insert warp, K1b)
+  InsertParams ins;      // record insert state (K1's producer warp marks/defers, K1b inserts)
 };
 
 struct LevelIO {               // per-position arrays at one height (stage boundary)
@@ -184,19 +183,26 @@ cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, 
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
 
 // ---- restore (k_restore.cu)
-struct RestoreDiff {           // one diff of the chain, as the restore kernels see it
+struct RestoreDiff {           // one diff of the chain, as the restore kernels see it (cached plan)
   const uint8_t* base;         // diff bytes (device)
   uint64_t nF, nS, meta_bytes, data_bytes;
   unsigned long long* Flo;     // per FIRST region: first chunk (sorted)
   unsigned long long* Foff;    // per FIRST region: offset in the data section
+  unsigned long long* Slo;     // per SHIFT region: first chunk
+  unsigned long long* Soff;    // per SHIFT region: exclusive scan of byte lengths; [nS] = total
+  unsigned long long* Ssrc;    // per SHIFT region: device address of its source bytes
+  unsigned long long shift_bytes;  // = Soff[nS]
+  unsigned long long* Fseg;    // per 2-KB segment of the FIRST stream: region of its first byte (+1 entry)
+  unsigned long long* Sseg;    // same for the SHIFT stream
 };
 cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long long* tmp_len, void* scan_tmp,
                                   size_t scan_tmp_bytes, cudaStream_t st);
-cudaError_t restore_copy_first(const Geo& g, const RestoreDiff& d, uint8_t* out, int num_sms, cudaStream_t st);
-cudaError_t restore_shift(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, uint8_t* out,
-                          unsigned long long* t_len, unsigned long long* t_off, unsigned long long* t_src,
-                          unsigned long long* t_dst, int* err, void* scan_tmp, size_t scan_tmp_bytes, int num_sms,
-                          cudaStream_t st);
+cudaError_t restore_prepare_shift(const Geo& g, RestoreDiff& d, const RestoreDiff* chain_dev, unsigned long long* tmp_len,
+                                  int* err, void* scan_tmp, size_t scan_tmp_bytes, cudaStream_t st);
+cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st);
+uint64_t restore_segments(uint64_t bytes);
+cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
+                          int num_sms, cudaStream_t st);
 size_t scan_tmp_bytes_for(uint64_t count);
 cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long* out, uint64_t count, void* tmp,
                                size_t tmp_bytes, cudaStream_t st);

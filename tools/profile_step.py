@@ -7,13 +7,20 @@ from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
 
 B, C, p = int(os.environ.get("B", 1 << 30)), int(os.environ.get("C", 128)), float(os.environ.get("P", 0.01))
 K = int(os.environ.get("K", 10))
-seed = W.seed_of(2)
+CFG = int(os.environ.get("CFG", 2))
+seed = W.seed_of(CFG)
 st = torch.cuda.Stream()
 bufs = [torch.empty(B, dtype=torch.uint8, device="cuda") for _ in range(K)]
-with torch.cuda.stream(st):
-    W.DeviceGen.initial(2, bufs[0], B, seed, st)
-    for k in range(1, K):
-        bufs[k].copy_(bufs[k - 1]); W.DeviceGen.mutate(2, bufs[k], B, k, C, seed, p, st)
+if CFG == 4:   # duplicate-heavy: host generator
+    g = W.DupHeavy(B, C, seed)
+    for k in range(K):
+        bufs[k].copy_(torch.from_numpy(g.next()))
+else:
+    with torch.cuda.stream(st):
+        W.DeviceGen.initial(CFG, bufs[0], B, seed, st)
+        for k in range(1, K):
+            bufs[k].copy_(bufs[k - 1]); W.DeviceGen.mutate(CFG, bufs[k], B, k, C, seed, p, st)
+torch.cuda.synchronize()
 st.synchronize()
 for prof in (True, False):
     ck = Checkpointer(C)
