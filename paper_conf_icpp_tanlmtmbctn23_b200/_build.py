@@ -43,6 +43,14 @@ def build(force: bool = False, verbose: bool = False) -> list[str]:
     return out
 
 
+def build_variant(name: str, defines: list[str]) -> str:
+    """An experiment build of libckpt.so with extra -D flags (selected with CKPT_LIB)."""
+    path = lib_path(name)
+    cmd = [NVCC] + FLAGS + [f"-D{d}" for d in defines] + ["-o", path] + LIBS["libckpt.so"]
+    subprocess.check_call(cmd)
+    return path
+
+
 if __name__ == "__main__":
     import sys
     for p in build(force="-f" in sys.argv, verbose="-v" in sys.argv):

@@ -65,7 +65,8 @@ def lib() -> ctypes.CDLL:
     """Load the in-tree libckpt.so (fails loudly if it is missing)."""
     global _lib
     if _lib is None:
-        path = _build.lib_path("libckpt.so")
+        # CKPT_LIB: an alternative in-tree build of the same library (A/B experiments)
+        path = os.environ.get("CKPT_LIB") or _build.lib_path("libckpt.so")
         if not os.path.exists(path):
             raise RuntimeError(f"{path} missing: run __graft_entry__.build() (no CPU fallback exists)")
         L = ctypes.CDLL(path)

@@ -47,9 +47,21 @@ __device__ __forceinline__ uint64_t rotl(uint64_t x, int r) { return (x << r) | 
 template <uint64_t C>
 __device__ __forceinline__ uint64_t mulc(uint64_t x) {
   const uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
+#ifdef CKPT_MULC3
+  // three IMADs, the high word accumulated through two mad.lo (no separate add)
+  uint32_t wlo, whi, h;
+  asm("mul.lo.u32 %0, %3, %4;\n\t"
+      "mul.hi.u32 %1, %3, %4;\n\t"
+      "mad.lo.u32 %2, %5, %4, %1;\n\t"
+      "mad.lo.u32 %2, %3, %6, %2;"
+      : "=r"(wlo), "=r"(whi), "=r"(h)
+      : "r"(lo), "n"((uint32_t)C), "r"(hi), "n"((uint32_t)(C >> 32)));
+  return ((uint64_t)h << 32) | wlo;
+#else
   const uint64_t w = (uint64_t)lo * (uint32_t)C;
   const uint32_t h = (uint32_t)(w >> 32) + hi * (uint32_t)C + lo * (uint32_t)(C >> 32);
   return ((uint64_t)h << 32) | (uint32_t)w;
+#endif
 }
 
 __device__ __forceinline__ uint64_t fmix(uint64_t k) {

@@ -543,7 +543,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     lp.mode3d = 1;
     lp.segs = (int)(h->C / 128);
     lp.stage_bytes = 128 * kLeafThreads;
-    lp.nst = 3;
+    lp.nst = kLeafStages3d;
     lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
   } else if (h->C < 128) {
     lp.mode3d = 0;

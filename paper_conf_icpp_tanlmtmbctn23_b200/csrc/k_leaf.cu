@@ -137,16 +137,25 @@ __device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile,
 // 8 hashing (consumer) warps + 1 producer warp. The producer streams the stages with TMA
 // (full barriers, complete_tx) and re-fills a stage as soon as all 8 consumer warps have
 // released it (empty barriers, one arrive per warp): fast warps never wait for slow ones
-// at a CTA barrier, they run ahead into the next filled stage. At the end of a 256-chunk
-// tile each consumer warp leaves its candidate ballot word in the stage's slot; the
-// producer, on the stage's release, marks the tree tile(s) dirty and defers the tile's
-// inserts to K1b, so that bookkeeping is off the hashing warps' path.
+// at a CTA barrier, they run ahead into the next filled stage. Tiles are handed out
+// dynamically (first wave = blockIdx, then a global cursor, fetched one tile ahead): the
+// SMs do not stream at the same rate (measured: with a static tile stride the first CTA
+// finished 20 % before the last), so a static split leaves the tail waiting on the slowest.
+// At the end of a 256-chunk tile each consumer warp leaves its candidate ballot word in
+// the stage's slot; the producer, on the stage's release, marks the tree tile(s) dirty and
+// defers the tile's inserts to K1b, so that bookkeeping is off the hashing warps' path.
 constexpr int kK1Threads = kLeafThreads + 32;
 constexpr int kMaxStagesK1 = 8;
+#ifndef CKPT_K1_CTAS
+#define CKPT_K1_CTAS 2   // resident K1 CTAs per SM (3 stages each when C % 128 == 0)
+#endif
+constexpr uint32_t kNoTile = 0xFFFFFFFFu;
 
 struct K1Shared {
   uint64_t full[kMaxStagesK1];
   uint64_t empty[kMaxStagesK1];
+  uint32_t tile[kMaxStagesK1];       // tile streamed into the stage (kNoTile: stop)
+  uint32_t tile_end[kMaxStagesK1];   // 1 if the stage holds the tile's last segment
   uint32_t words[kMaxStagesK1][8];   // candidate ballot words of the tile ending in the stage
 };
 
@@ -155,7 +164,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 }
 
 template <int MODE3D>
-__global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
+__global__ void __launch_bounds__(kK1Threads, CKPT_K1_CTAS) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
   const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -169,8 +178,6 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
   const int tid = threadIdx.x;
   const uint32_t n_tiles = (uint32_t)(p.n_main / kLeafThreads);
   const int segs = p.segs;
-  const uint32_t my_tiles = (blockIdx.x < n_tiles) ? (n_tiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-  const uint32_t total = my_tiles * (uint32_t)segs;
   const bool use_prev = p.g.k > 0;
 
   if (tid == 0) {
@@ -187,11 +194,11 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
     // ---------------- producer warp (lane 0)
     if (tid != kLeafThreads) return;
     const uint64_t pol_stream = policy_evict_first();
-    // the tile epilogue of step i (consumed from stage i % nst): dirty marks + deferral
-    auto epilogue = [&](uint32_t i) {
-      if ((int)(i % (uint32_t)segs) != segs - 1) return;
-      const uint32_t tile = blockIdx.x + (i / (uint32_t)segs) * gridDim.x;
-      const int s = (int)(i % (uint32_t)nst);
+    uint32_t* cursor = &p.ins.tot->k1_next;
+    // the tile epilogue of the step last consumed from stage s: dirty marks + deferral
+    auto epilogue = [&](int s) {
+      if (!sh.tile_end[s]) return;
+      const uint32_t tile = sh.tile[s];
       uint32_t w[8], any = 0, pc = 0;
 #pragma unroll
       for (int q = 0; q < 8; ++q) { w[q] = sh.words[s][q]; any |= w[q]; pc += __popc(w[q]); }
@@ -200,28 +207,41 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
         defer_tile(p.ins, tile, pc);
       }
     };
-    for (uint32_t i = 0; i < total; ++i) {
+    uint32_t tile = blockIdx.x, seg = 0, i = 0;
+    uint32_t nxt = tile < n_tiles ? gridDim.x + atomicAdd(cursor, 1u) : kNoTile;   // one tile ahead
+    for (;; ++i) {
       const int s = (int)(i % (uint32_t)nst);
       if (i >= (uint32_t)nst) {
         mbar_wait(&sh.empty[s], ((i / nst) - 1) & 1u);   // all consumer warps released step i - nst
-        epilogue(i - nst);
+        epilogue(s);
       }
-      const uint32_t tile = blockIdx.x + (i / (uint32_t)segs) * gridDim.x;
-      const int seg = (int)(i % (uint32_t)segs);
-      const bool with_prev = use_prev && seg == segs - 1;
+      if (tile >= n_tiles) {   // stop marker: wakes the consumers without data
+        sh.tile[s] = kNoTile;
+        sh.tile_end[s] = 0;
+        mbar_arrive(&sh.full[s]);
+        break;
+      }
+      const bool with_prev = use_prev && (int)seg == segs - 1;
+      sh.tile[s] = tile;
+      sh.tile_end[s] = (int)seg == segs - 1;
       mbar_arrive_expect_tx(&sh.full[s], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
       if (MODE3D)
-        tma_load_3d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, seg, (int)(tile * kLeafThreads), pol_stream);
+        tma_load_3d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, (int)seg, (int)(tile * kLeafThreads), pol_stream);
       else
         tma_load_2d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, (int)(tile * (stage_bytes / 128)), pol_stream);
       if (with_prev)
         bulk_load(prevbuf + s * kLeafThreads, p.prev + (uint64_t)tile * kLeafThreads, kLeafThreads * 16u, &sh.full[s],
                   pol_stream);
+      if ((int)++seg == segs) {
+        seg = 0;
+        tile = nxt;
+        if (tile < n_tiles) nxt = gridDim.x + atomicAdd(cursor, 1u);
+      }
     }
-    const uint32_t first_tail = total > (uint32_t)nst ? total - nst : 0;
-    for (uint32_t i = first_tail; i < total; ++i) {
-      mbar_wait(&sh.empty[i % nst], (i / nst) & 1u);
-      epilogue(i);
+    // drain: the real steps after the last one handled above (i - nst + 1 .. i - 1)
+    for (uint32_t j = i + 1 > (uint32_t)nst ? i + 1 - nst : 0; j < i; ++j) {
+      mbar_wait(&sh.empty[j % nst], (j / nst) & 1u);
+      epilogue((int)(j % (uint32_t)nst));
     }
     return;
   }
@@ -233,9 +253,11 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
   const int lane = tid & 31, wid = tid >> 5;
   uint64_t h1 = 0, h2 = 0;
   int st = 0, seg = 0;
-  uint32_t phase = 0, tile = blockIdx.x;
-  for (uint32_t step = 0; step < total; ++step) {
+  uint32_t phase = 0;
+  for (;;) {
     mbar_wait(&sh.full[st], phase);
+    const uint32_t tile = sh.tile[st];
+    if (tile == kNoTile) break;
     if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
     const uint8_t* sd = data + (size_t)st * stage_bytes;
 #pragma unroll 8
@@ -244,7 +266,11 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
       const uint32_t row = u >> 3;
       const uint32_t off = (row << 7) | ((((u & 7) ^ (row & 7))) << 4);   // SWIZZLE_128B
       const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + off);
+#ifdef CKPT_K1_NOHASH   // timing experiment only: data movement without the hash
+      h1 ^= v.x; h2 ^= v.y;
+#else
       mm::block(h1, h2, v.x, v.y);
+#endif
     }
     if (seg == segs - 1) {
       const Digest d = mm::finish(h1, h2, p.g.C);
@@ -268,7 +294,7 @@ __global__ void __launch_bounds__(kK1Threads, 2) leaf_hash_kernel(const __grid_c
     __syncwarp();
     if (lane == 0) mbar_arrive(&sh.empty[st]);   // this warp is done with stage st
     if (++st == nst) { st = 0; phase ^= 1u; }
-    if (++seg == segs) { seg = 0; tile += gridDim.x; }
+    if (++seg == segs) seg = 0;
   }
   trace_block(p.ins.trace, p.ins.trace_n, bt0, bt0, 0);
 }
@@ -474,7 +500,7 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   size_t smem;
   leaf_smem_config(p, &smem);
   const uint64_t n_tiles = p.n_main / kLeafThreads;
-  uint64_t grid = (uint64_t)num_sms * 2;
+  uint64_t grid = (uint64_t)num_sms * CKPT_K1_CTAS;
   if (grid > n_tiles) grid = n_tiles;
   if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else leaf_hash_kernel<0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
@@ -504,7 +530,9 @@ cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st) {
 
 cudaError_t leaf_setup_attributes() {
   // the largest dynamic smem any leaf configuration asks for (C >= 128: 3 x 36 KB; C < 128: <= 96 KB)
-  const int smem = 1008 + 3 * (32768 + 4096) + (int)sizeof(K1Shared);   // the largest leaf configuration
+  // the largest leaf configuration: kLeafStages3d x (32 KB + 4 KB) when C % 128 == 0, <= 96 KB of stages below
+  const int stages = kLeafStages3d * (32768 + 4096) > 98304 + 8 * 4096 ? kLeafStages3d * (32768 + 4096) : 98304 + 8 * 4096;
+  const int smem = 1008 + stages + (int)sizeof(K1Shared);
   cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;

@@ -22,6 +22,11 @@ constexpr int kGroupLog = 10;   // upper stages: 1024 positions per group
 constexpr int kLeafThreads = 256;
 constexpr int kTreeThreads = 256;
 constexpr int kTilesPerBlock = 1024;  // compaction: tiles per reduce/offsets CTA
+#ifdef CKPT_K1_STAGES
+constexpr int kLeafStages3d = CKPT_K1_STAGES;   // experiment builds
+#else
+constexpr int kLeafStages3d = 3;      // K1 TMA stages of 32 KB (+ 4 KB digests) when C % 128 == 0
+#endif
 
 struct Totals {                      // per-checkpoint device counters (zeroed each call)
   unsigned long long nF, nS, data_bytes, meta_bytes;
@@ -30,7 +35,7 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   uint32_t wl_count[kMaxStages];
   uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
   uint32_t gather_next;              // work-stealing cursor of the gather kernel
-  uint32_t unused0;
+  uint32_t k1_next;                  // K1 tile cursor (tiles handed out beyond the first wave)
   uint32_t defer_count;              // 256-chunk leaf tiles whose inserts K1 left to K1b
   uint32_t insert_next;              // work-stealing cursor of K1b
   uint32_t pad2[2];
