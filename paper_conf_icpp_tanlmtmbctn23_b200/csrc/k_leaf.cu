@@ -27,7 +27,10 @@ __device__ __forceinline__ bool leaf_is_candidate(const Geo& g, const Digest& d,
 }
 
 // ------------------------------------------------------------------ record insert
-constexpr uint32_t kDenseTile = 64;   // candidates per 256-chunk tile above which inserts read first
+constexpr uint32_t kDenseTile = 64;
+#ifndef CKPT_K1B_BPS
+#define CKPT_K1B_BPS 4   // K1b launch bound: 4 resident blocks per SM (<= 64 registers)
+#endif   // candidates per 256-chunk tile above which inserts read first
 // Map.insert(digest, (leaf, chkptID)) for the candidates of one 256-chunk leaf tile
 // (Alg.1 l.6-19), by one warp: lane i < 8 holds candidate word i. The candidates are
 // spread evenly over the lanes (prefix over popcounts, __fns), identical digests within a
@@ -439,7 +442,7 @@ __device__ void build_tree_work(const InsertParams& p) {
     if (ulonglong4* r = trace_alloc(p.trace, p.trace_n, 1)) *r = make_ulonglong4(tw0, tw1, gtime_ns(), 12);
 }
 
-__global__ void __launch_bounds__(256) insert_kernel(InsertParams p) {
+__global__ void __launch_bounds__(256, CKPT_K1B_BPS) insert_kernel(InsertParams p) {
   const unsigned long long bt0 = p.trace ? gtime_ns() : 0;
   pdl_launch_dependents();
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;

@@ -12,15 +12,23 @@ B, C, p, K = int(os.environ.get("B", 1 << 30)), int(os.environ.get("C", 128)), f
 cfg = int(os.environ.get("CFG", 2))
 seed = W.seed_of(cfg)
 st = torch.cuda.Stream()
+K = int(os.environ.get("K", K))
 bufs = [torch.empty(B, dtype=torch.uint8, device="cuda") for _ in range(K)]
-with torch.cuda.stream(st):
-    W.DeviceGen.initial(cfg, bufs[0], B, seed, st)
-    for k in range(1, K):
-        bufs[k].copy_(bufs[k - 1]); W.DeviceGen.mutate(cfg, bufs[k], B, k, C, seed, p, st)
-st.synchronize()
+if cfg == 4:
+    g = W.DupHeavy(B, C, seed)
+    for k in range(K):
+        bufs[k].copy_(torch.from_numpy(g.next()))
+    torch.cuda.synchronize()
+else:
+    with torch.cuda.stream(st):
+        W.DeviceGen.initial(cfg, bufs[0], B, seed, st)
+        for k in range(1, K):
+            bufs[k].copy_(bufs[k - 1]); W.DeviceGen.mutate(cfg, bufs[k], B, k, C, seed, p, st)
+    st.synchronize()
+prof = int(os.environ.get("PROF", 1))
 res = {}
 for rep in range(2):
-    ck = Checkpointer(C); ck.set_profiling(1)
+    ck = Checkpointer(C); ck.set_profiling(prof)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for k in range(3): ck.checkpoint(bufs[k], stream=st)
     e0.record(st)
@@ -30,6 +38,9 @@ for rep in range(2):
     tot = [ck.phase_times(k)["total"] for k in range(3, K)]
     res = {"k1_ms": round(statistics.median(k1), 4), "call_ms": round(statistics.median(tot), 4),
            "loop_ms_per_step": round(e0.elapsed_time(e1) / (K - 3), 4)}
+    if prof >= 2:
+        for ph in ("insert", "phase2", "phase3", "compact"):
+            res[ph] = round(statistics.median([ck.phase_times(k)[ph] for k in range(3, K)]), 4)
     ck.close()
 print("RESULT", json.dumps(res))
 '''
