@@ -414,7 +414,9 @@ def run_ours(args):
             "roofline": {"bound": "hbm", "kernel": "leaf_hash_kernel (K1)", "achieved": round(achieved, 1),
                          "peak": peak, "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
                          "peak_kind": peak_kind,
-                         "alg_bytes_per_launch": int(sum(alg) / len(alg)), "k1_ms": round(k1_avg_ms, 4)},
+                         "alg_bytes_per_launch": int(sum(alg) / len(alg)), "k1_ms": round(k1_avg_ms, 4),
+                         "context": "K1 is a read stream: the read-only TMA ceiling measured on this box type by "
+                                    "tools/bw_probe.cu is ~6.9-7.1 TB/s (profiles/bw_probe_r1.txt), above the copy peak"},
             "phase_ms": phase_avg,
             "phase_ms_note": "per-phase split from an untimed replay with events between kernels; total_timed = timed-run first-to-last-kernel span",
             "diff_ratio": round(ratio, 2),
