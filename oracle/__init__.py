@@ -56,6 +56,8 @@ def lib() -> ctypes.CDLL:
         L.orc_mmh3.restype = None
         L.orc_create.argtypes = [ctypes.c_uint32, ctypes.c_int]
         L.orc_create.restype = ctypes.c_void_p
+        L.orc_create_mode.argtypes = [ctypes.c_uint32, ctypes.c_int, ctypes.c_int]
+        L.orc_create_mode.restype = ctypes.c_void_p
         L.orc_destroy.argtypes = [ctypes.c_void_p]
         L.orc_destroy.restype = None
         L.orc_checkpoint.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
@@ -100,15 +102,20 @@ def mmh3(data: bytes, seed: int = 0) -> bytes:
     return out.tobytes()
 
 
-class Oracle:
-    """One de-duplication lineage (one process / GPU in the paper)."""
+MODE_TREE, MODE_LIST, MODE_BASIC = 0, 1, 2   # the methods compared in P:194 (Tree = ours)
 
-    def __init__(self, chunk_bytes: int, ideal: bool = False):
-        self._h = lib().orc_create(chunk_bytes, 1 if ideal else 0)
+
+class Oracle:
+    """One de-duplication lineage (one process / GPU in the paper).
+    mode: MODE_TREE (Algorithm 1), MODE_LIST or MODE_BASIC."""
+
+    def __init__(self, chunk_bytes: int, ideal: bool = False, mode: int = MODE_TREE):
+        self._h = lib().orc_create_mode(chunk_bytes, 1 if ideal else 0, mode)
         if not self._h:
-            raise ValueError("bad chunk size")
+            raise ValueError("bad chunk size or mode")
         self.chunk_bytes = chunk_bytes
         self.ideal = ideal
+        self.mode = mode
         self.buf_bytes = None
 
     def close(self):
@@ -198,9 +205,18 @@ class Oracle:
 
 
 def parse_diff(d: bytes) -> dict:
-    """Decode the consolidated-difference byte format (reading R13)."""
+    """Decode the consolidated-difference byte format (reading R13).
+    Basic diffs (flags == 2) carry a changed-chunk bitmap instead of entry lists."""
     import struct
     magic, ver, flags, cid, C, B, n, nF, nS, data_bytes, seed, _res = struct.unpack_from("<IHHIIQQQQQII", d, 0)
+    if flags == MODE_BASIC:
+        words = (n + 31) // 32
+        bits = list(struct.unpack_from(f"<{words}I", d, 64)) if words else []
+        changed = [i for i in range(n) if (bits[i // 32] >> (i % 32)) & 1]
+        meta = (64 + 4 * words + 15) // 16 * 16
+        return dict(magic=magic, version=ver, flags=flags, id=cid, chunk_bytes=C, buf_bytes=B, n_leaves=n,
+                    changed=changed, n_changed=nF, data_bytes=data_bytes, seed=seed, meta_bytes=meta,
+                    data=d[meta:], first=[], shift=[])
     F = list(struct.unpack_from(f"<{nF}I", d, 64)) if nF else []
     S = []
     off = 64 + 4 * nF
