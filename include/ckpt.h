@@ -71,12 +71,35 @@ typedef struct {
   uint64_t phase2_inserts;  /* FIRST internal nodes inserted (Alg.1 l.29)                    */
 } ckpt_diff;
 
+/* De-duplication methods compared in the paper; the diff header's u16 `flags`
+ * field (bytes 6-7) holds the method.
+ *   CKPT_MODE_TREE   Algorithm 1 with Merkle-tree metadata compaction (ours, the default).
+ *   CKPT_MODE_LIST   "identical to our method except for the metadata compaction, which is
+ *                    omitted. Instead, a full list of all first-time occurrences and shifted
+ *                    duplicates is stored along the new chunks": the Tree format with one
+ *                    entry per non-FIXED leaf; the record holds leaves only.
+ *   CKPT_MODE_BASIC  "breaks the checkpoint into chunks, hashes the chunks, then builds a
+ *                    bitmap to indicate what chunks are new and what chunks remain
+ *                    unchanged. It saves the bitmap and the new chunks": header
+ *                    (n_first_regions = changed chunks, n_shift_regions = 0), ceil(n/32) u32
+ *                    bitmap words (bit i of word i/32 = chunk i changed since checkpoint
+ *                    k-1; all set at k = 0), zero pad to 16 B, the changed chunks in chunk
+ *                    order at their true length. No record. */
+enum { CKPT_MODE_TREE = 0, CKPT_MODE_LIST = 1, CKPT_MODE_BASIC = 2 };
+
 /* Create a handle.  P:77: fixed-size chunks of "tens or hundreds of bytes".
  *   chunk_bytes  C, a multiple of 16 with 32 <= C <= 65536 (C > 2 x 16-B digest).
  *   out          receives the handle (owned by the caller; free with ckpt_destroy).
  * Binds the handle to the current CUDA device.  Errors: CKPT_EINVAL (bad C / NULL out),
  * CKPT_ECUDA (no usable sm_100 device). */
 CKPT_API int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out);
+
+/* ckpt_create with an explicit method (CKPT_MODE_*). ckpt_create is
+ * ckpt_create_mode(chunk_bytes, CKPT_MODE_TREE, out). All other calls behave as described
+ * for every mode; the statistics of a Basic diff count changed chunks as n_first and
+ * n_first_regions (no spatial / temporal de-duplication).
+ * Errors: as ckpt_create, and CKPT_EINVAL for an unknown mode. */
+CKPT_API int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out);
 
 /* De-duplicate one checkpoint (Alg.1; serialization P:81).
  *   dev_ptr  device buffer of `bytes` bytes, 16-byte aligned, BORROWED for the call; the

@@ -18,8 +18,10 @@ from . import _build
 
 CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_ECOLLIDE = range(7)
 
+CKPT_MODE_TREE, CKPT_MODE_LIST, CKPT_MODE_BASIC = 0, 1, 2   # methods of P:194 (include/ckpt.h)
+
 ABI_FUNCTIONS = [
-    "ckpt_create", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
+    "ckpt_create", "ckpt_create_mode", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
     "ckpt_checkpoint_host", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
     "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
     "ckpt_strerror",
@@ -74,6 +76,7 @@ def lib() -> ctypes.CDLL:
         P = ctypes.POINTER
         sig = {
             "ckpt_create": ([u32, P(vp)], i32),
+            "ckpt_create_mode": ([u32, i32, P(vp)], i32),
             "ckpt_checkpoint": ([vp, vp, u64, vp, P(CkptDiff)], i32),
             "ckpt_restore": ([vp, u32, vp], i32),
             "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
@@ -135,13 +138,14 @@ def _stream_handle(stream) -> int:
 class Checkpointer:
     """One de-duplication lineage on the current CUDA device (one per process / GPU)."""
 
-    def __init__(self, chunk_bytes: int):
+    def __init__(self, chunk_bytes: int, mode: int = CKPT_MODE_TREE):
         h = ctypes.c_void_p()
-        rc = lib().ckpt_create(chunk_bytes, ctypes.byref(h))
+        rc = lib().ckpt_create_mode(chunk_bytes, mode, ctypes.byref(h))
         if rc != CKPT_OK:
-            raise CkptError(rc, "ckpt_create")
+            raise CkptError(rc, "ckpt_create_mode")
         self._h = h
         self.chunk_bytes = chunk_bytes
+        self.mode = mode
 
     # ------------------------------------------------------------------ core calls
     def checkpoint(self, buf, nbytes: int | None = None, stream=None, raw: bool = False):

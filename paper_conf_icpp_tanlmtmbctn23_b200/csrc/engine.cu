@@ -51,6 +51,7 @@ struct ckpt_ctx {
   int num_sms = 148;
   bool poisoned = false;
   uint32_t C = 0;
+  int mode = kModeTree;          // CKPT_MODE_*
   // geometry (fixed after checkpoint 0, R17)
   bool geo_set = false;
   uint64_t B = 0, n = 0, m = 0;
@@ -343,8 +344,11 @@ const char* ckpt_strerror(int status) {
   }
 }
 
-int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
+int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) { return ckpt_create_mode(chunk_bytes, CKPT_MODE_TREE, out); }
+
+int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
   if (!out || chunk_bytes < 32 || chunk_bytes > 65536 || chunk_bytes % 16) return CKPT_EINVAL;
+  if (mode != CKPT_MODE_TREE && mode != CKPT_MODE_LIST && mode != CKPT_MODE_BASIC) return CKPT_EINVAL;
   *out = nullptr;
   int dev = 0;
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
@@ -356,6 +360,7 @@ int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out) {
   h->device = dev;
   h->num_sms = prop.multiProcessorCount;
   h->C = chunk_bytes;
+  h->mode = mode;
   h->trace_path = getenv("CKPT_TRACE");
   if (const char* d = getenv("CKPT_DBG")) h->dbg = atoi(d);
   void* fn = nullptr;
@@ -502,7 +507,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     if (r != CKPT_OK) return r;
   }
   const uint32_t k = (uint32_t)h->diffs.size();
-  int r = ensure_table(h, st);
+  int r = h->mode == kModeBasic ? CKPT_OK : ensure_table(h, st);   // Basic keeps no record
   if (r != CKPT_OK) return r;
   const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
   if (!h->arena.ensure(worst)) return CKPT_ENOMEM;
@@ -529,6 +534,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     ip.dcnt[s] = h->dcnt[s];
   }
   ip.trace = h->trace; ip.trace_n = h->trace_n;
+  ip.mode = h->mode;
+  ip.blocksum = h->blocksum;
+  ip.gsum = h->gsum;
 
   // ---- leaf pass configuration
   LeafParams lp;
@@ -608,10 +616,16 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.gm2 = h->gm2[s];
     sp.gm3 = h->gm3[s];
   }
-  CK(launch_tree(tp, 2, h->num_sms, st));
-  if (pe) CK(cudaEventRecord(h->ev[3], st));
-  CK(launch_tree(tp, 3, h->num_sms, st));
-  if (pe) CK(cudaEventRecord(h->ev[4], st));
+  tp.list = h->mode == kModeList;
+  if (h->mode != kModeBasic) {   // Basic: no record, no tree
+    CK(launch_tree(tp, 2, h->num_sms, st));
+    if (pe) CK(cudaEventRecord(h->ev[3], st));
+    CK(launch_tree(tp, 3, h->num_sms, st));
+    if (pe) CK(cudaEventRecord(h->ev[4], st));
+  } else if (pe) {
+    CK(cudaEventRecord(h->ev[3], st));
+    CK(cudaEventRecord(h->ev[4], st));
+  }
 
   // ---- compaction + serialisation
   CompactParams cp;
@@ -626,6 +640,10 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.dbg = h->dbg;
   cp.ctr_next = reinterpret_cast<uint4*>(h->ctr2[(k + 1) & 1]);
   cp.ctr_next_words = h->ctr_bytes / 16;
+  cp.mode = h->mode;
+  cp.cand = h->cand;
+  cp.nwords = h->nwords;
+  cp.tcc = h->tcc;
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
   const auto t_launched = clk::now();
@@ -647,7 +665,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
     if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), f); fclose(f); }
   }
-  h->live += t.n_first + t.p2_inserts;
+  if (h->mode != kModeBasic) h->live += t.n_first + t.p2_inserts;
   DiffRec rec;
   rec.ptr = out;
   fill_diff(h, k, t, out, &rec.info);
@@ -709,12 +727,14 @@ int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, vo
 static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st) {
   uint64_t need_len = 1;
   bool any = false;
+  const bool basic = h->mode == kModeBasic;
   for (uint32_t c = 0; c <= id; ++c) {
     const DiffRec& d = h->diffs[c];
     if (d.planned) continue;
     any = true;
     need_len = std::max<uint64_t>(need_len, std::max(d.info.n_first_regions, d.info.n_shift_regions));
   }
+  if (basic) need_len = std::max<uint64_t>(need_len, 2 * h->nwords);   // word counts + their scan
   if (!any) return CKPT_OK;
   auto grow = [](void** p, size_t bytes) -> bool {
     if (*p) cudaFree(*p);
@@ -763,7 +783,9 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     }
     r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
     r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
-    if (!d.planned && r.nF && restore_prepare_first(g, r, h->rs_len, h->rs_scan, h->rs_scan_bytes, st) != cudaSuccess)
+    if (!d.planned && r.nF &&
+        (basic ? restore_prepare_basic(g, r, h->nwords, h->rs_len, h->rs_scan, h->rs_scan_bytes, st)
+               : restore_prepare_first(g, r, h->rs_len, h->rs_scan, h->rs_scan_bytes, st)) != cudaSuccess)
       return CKPT_ECUDA;
   }
   if (cudaMemcpyAsync(h->rs_chain, rd.data(), rd.size() * sizeof(RestoreDiff), cudaMemcpyHostToDevice, st) != cudaSuccess)

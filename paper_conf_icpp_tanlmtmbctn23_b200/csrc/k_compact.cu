@@ -85,15 +85,18 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     data_tot += __ldg(p.blocksum + 3 * i + 2);
   }
   warp_sum3(nF_tot, nS_tot, data_tot);
-  const unsigned long long raw = 64 + 4 * nF_tot + 12 * nS_tot;
+  const bool basic = p.mode == kModeBasic;
+  // Basic: the changed-chunk bitmap replaces the entry lists (nF_tot = changed chunks)
+  const unsigned long long raw = basic ? 64 + 4ull * p.nwords : 64 + 4 * nF_tot + 12 * nS_tot;
   const unsigned long long meta = (raw + 15) & ~15ull;
   if (blockIdx.x == 0 && wid == 0 && lane == 0) {
     // totals and the 64-byte header (R13)
     p.tot->nF = nF_tot; p.tot->nS = nS_tot; p.tot->data_bytes = data_tot; p.tot->meta_bytes = meta;
+    if (basic) p.tot->n_first = nF_tot;   // every changed chunk is stored (no record)
     uint8_t* o = p.out;
     *reinterpret_cast<uint32_t*>(o + 0) = 0x44504B43u;   // 'CKPD'
     *reinterpret_cast<uint16_t*>(o + 4) = 1;             // version
-    *reinterpret_cast<uint16_t*>(o + 6) = 0;             // flags
+    *reinterpret_cast<uint16_t*>(o + 6) = (uint16_t)p.mode;   // flags: the method
     *reinterpret_cast<uint32_t*>(o + 8) = g.k;
     *reinterpret_cast<uint32_t*>(o + 12) = g.C;
     *reinterpret_cast<unsigned long long*>(o + 16) = g.B;
@@ -107,6 +110,11 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     // every counter the host reports is final here (tree kernels done, pdl_wait above)
     *p.tot_host = *p.tot;
   }
+  if (basic) {   // the bitmap: K1's candidate words, all n bits
+    uint32_t* bm = reinterpret_cast<uint32_t*>(p.out + 64);
+    for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < p.nwords; i += (uint64_t)gridDim.x * kCT)
+      bm[i] = (i + 1 == p.nwords && (p.g.n & 31)) ? (__ldg(p.cand + i) & ((1u << (p.g.n & 31)) - 1u)) : __ldg(p.cand + i);
+  }
   uint8_t* const ent_f = p.out + 64;
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
   uint8_t* const dat = p.out + meta;
@@ -116,8 +124,25 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     unsigned long long tg0 = 0, tg1 = 0, tg2 = 0;
     if (p.trace) tg0 = gtime_ns();
     // one round of loads: counts, FIRST-chunk mask, the first 64 region records, prefix sums
-    const uint4 cnt = __ldg(p.tilecnt + T);
-    const uint32_t fw = __ldg(p.lmask + T * kLmWords + kLmFirstChunks + lane);
+    uint64_t lo, hi;
+    chunk_range(g, g.t0, T, lo, hi);
+    uint4 cnt;
+    uint32_t fw;
+    if (basic) {   // the tile's changed chunks, chunk order, straight from K1's bitmap
+      cnt = make_uint4(0, 0, 0, g.epoch);
+      const uint64_t c0 = lo + 32ull * lane;
+      fw = 0;
+      if (c0 < hi) {
+        const uint32_t sh = (uint32_t)(c0 & 31);
+        const uint32_t a = __ldg(p.cand + (c0 >> 5));
+        const uint32_t b = (c0 >> 5) + 1 < p.nwords ? __ldg(p.cand + (c0 >> 5) + 1) : 0u;
+        fw = sh ? ((a >> sh) | (b << (32 - sh))) : a;
+        if (hi - c0 < 32) fw &= (1u << (hi - c0)) - 1u;
+      }
+    } else {
+      cnt = __ldg(p.tilecnt + T);
+      fw = __ldg(p.lmask + T * kLmWords + kLmFirstChunks + lane);
+    }
     const uint4* recs = p.scratch + (T << g.t0);
     const uint32_t tcap = 1u << g.t0;   // records per tile
     uint4 rec0 = make_uint4(0, 0, 0, 0), rec1 = make_uint4(0, 0, 0, 0);
@@ -141,8 +166,14 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       }
       const uint64_t tq = G0 * 32 + lane;
       if (tq < T) {
-        const uint4 x = __ldg(p.tilecnt + tq);
-        if (x.w == g.epoch) { pF += x.x; pS += x.y; pD += x.z; }
+        if (basic) {   // an earlier tile never holds the short last chunk
+          const unsigned long long x = __ldg(p.tcc + tq);
+          pF += x;
+          pD += x * g.C;
+        } else {
+          const uint4 x = __ldg(p.tilecnt + tq);
+          if (x.w == g.epoch) { pF += x.x; pS += x.y; pD += x.z; }
+        }
       }
     }
     const uint64_t Tcur = T;
@@ -151,7 +182,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       warp_sum3(pF, pS, pD);
       continue;
     }
-    const uint32_t nF = cnt.x, nS = cnt.y;
+    const uint32_t nF = basic ? 0u : cnt.x, nS = basic ? 0u : cnt.y;   // Basic: no entries
     if (p.trace) tg1 = gtime_ns();
     // ranks of the FIRST chunks (chunk order)
     const uint32_t pc = __popc(fw);
@@ -165,8 +196,6 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     gw.fw[lane] = fw;
     const uint32_t nch = __shfl_sync(0xffffffffu, incl, 31);
     __syncwarp();
-    uint64_t lo, hi;
-    chunk_range(g, g.t0, Tcur, lo, hi);
     // the FIRST bytes: unit x of the tile's stream = unit (x mod U) of its (x / U)-th chunk,
     // source found from the mask alone; up to kStageUnits units go global -> shared with
     // cp.async in one round trip, then shared -> the data section at tile offset + 16 x.

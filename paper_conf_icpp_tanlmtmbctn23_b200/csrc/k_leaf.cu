@@ -124,7 +124,21 @@ __device__ __forceinline__ void mark_tree_dirty(const InsertParams& p, uint32_t 
     chunk_range(p.g, p.g.t0, t, lo, hi);
     const uint64_t a = lo > c0 ? lo : c0, b = hi < c1 + 1 ? hi : c1 + 1;
     const uint32_t cnt = a < b ? popc_range(w, (uint32_t)(a - c0), (uint32_t)(b - c0)) : 0u;
-    if (cnt) atomicAdd(p.tcc + t, cnt);
+    if (cnt) {
+      atomicAdd(p.tcc + t, cnt);
+      if (p.mode == kModeBasic) {
+        // Basic: the gather's prefix inputs are the changed chunks and their bytes (the
+        // buffer's last chunk may be short)
+        unsigned long long bytes = (unsigned long long)cnt * p.g.C;
+        const uint64_t last = p.g.n - 1;
+        if (a <= last && last < b && ((w[(last - c0) >> 5] >> ((last - c0) & 31)) & 1u))
+          bytes -= (unsigned long long)p.g.n * p.g.C - p.g.B;
+        atomicAdd(p.blocksum + 3 * (t / kTilesPerBlock), (unsigned long long)cnt);
+        atomicAdd(p.blocksum + 3 * (t / kTilesPerBlock) + 2, bytes);
+        atomicAdd(p.gsum + 3 * (t / 32), (unsigned long long)cnt);
+        atomicAdd(p.gsum + 3 * (t / 32) + 2, bytes);
+      }
+    }
   }
 }
 
@@ -207,7 +221,7 @@ __global__ void __launch_bounds__(kK1Threads, CKPT_K1_CTAS) leaf_hash_kernel(con
       for (int q = 0; q < 8; ++q) { w[q] = sh.words[s][q]; any |= w[q]; pc += __popc(w[q]); }
       if (any) {
         mark_tree_dirty(p.ins, tile, w);
-        defer_tile(p.ins, tile, pc);
+        if (p.ins.mode != kModeBasic) defer_tile(p.ins, tile, pc);   // Basic keeps no record
       }
     };
     uint32_t tile = blockIdx.x, seg = 0, i = 0;
@@ -349,7 +363,7 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
   if (pc && threadIdx.x == 0) {
     const uint32_t tile = (uint32_t)((p.tail_begin >> 8) + blockIdx.x);
     mark_tree_dirty(p.ins, tile, s_w);
-    defer_tile(p.ins, tile, (uint32_t)pc);
+    if (p.ins.mode != kModeBasic) defer_tile(p.ins, tile, (uint32_t)pc);
   }
 }
 
@@ -524,6 +538,7 @@ static int g_insert_blocks_per_sm = 0;
 cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st) {
   const uint64_t tiles = (p.nwords + 7) / 8;
   uint64_t blocks = (tiles + 7) / 8 + 1;   // + block 0: tree work description
+  if (p.mode == kModeBasic) blocks = 1;    // Basic: no record; only the dirty-tile worklist
   // one resident wave: the deferred work is strided statically over the warps
   const uint64_t wave = (uint64_t)num_sms * (g_insert_blocks_per_sm > 0 ? g_insert_blocks_per_sm : 4);
   if (blocks > wave) blocks = wave;

@@ -219,6 +219,23 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
   d.Ssrc[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + (vlo - s.Flo[lo]) * (unsigned long long)g.C);
 }
 
+// Basic diffs: every changed chunk is a one-chunk "FIRST region" of the plan.
+// popcount per bitmap word, then (after an exclusive scan) the chunk ids of the set bits.
+__global__ void basic_count_kernel(const uint8_t* base, uint64_t nwords, unsigned long long* cnt) {
+  const uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w < nwords) cnt[w] = __popc(rd32(base + 64 + 4 * w));
+}
+__global__ void basic_expand_kernel(Geo g, RestoreDiff d, uint64_t nwords, const unsigned long long* off) {
+  const uint64_t w = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (w >= nwords) return;
+  uint32_t m = rd32(d.base + 64 + 4 * w);
+  unsigned long long r = off[w];
+  for (; m; m &= m - 1, ++r) {
+    d.Flo[r] = 32ull * w + (__ffs(m) - 1);
+    d.Foff[r] = r * (unsigned long long)g.C;   // only the buffer's last chunk can be short
+  }
+}
+
 // segment map: region holding the first byte of each 2-KB segment; map[nseg] = nr - 1
 __global__ void segmap_kernel(const unsigned long long* off, uint64_t nr, uint64_t nseg, unsigned long long* map) {
   const uint64_t sg = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -284,6 +301,19 @@ cudaError_t restore_prepare_shift(const Geo& g, RestoreDiff& d, const RestoreDif
   return cudaGetLastError();
 }
 
+cudaError_t restore_prepare_basic(const Geo& g, RestoreDiff& d, uint64_t nwords, unsigned long long* tmp_cnt,
+                                  void* scan_tmp, size_t scan_tmp_bytes, cudaStream_t st) {
+  if (d.nF == 0) return cudaSuccess;
+  const unsigned blocks = (unsigned)((nwords + 255) / 256);
+  basic_count_kernel<<<blocks, 256, 0, st>>>(d.base, nwords, tmp_cnt);
+  note_launch();
+  cudaError_t e = scan_u64_exclusive(tmp_cnt, tmp_cnt + nwords, nwords, scan_tmp, scan_tmp_bytes, st);
+  if (e != cudaSuccess) return e;
+  basic_expand_kernel<<<blocks, 256, 0, st>>>(g, d, nwords, tmp_cnt + nwords);
+  note_launch();
+  return cudaGetLastError();
+}
+
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st) {
   if (d.nF) {
     const uint64_t ns = (d.data_bytes + kPaintSeg - 1) / kPaintSeg;
@@ -319,6 +349,8 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_shift_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, write_total_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, segmap_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_count_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_expand_kernel);
   return e;
 }
 

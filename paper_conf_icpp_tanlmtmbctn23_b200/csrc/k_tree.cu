@@ -524,7 +524,23 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   // updates are far smaller than a tile) hashes, inserts and emits nothing; its root is
   // FIXED iff every child is, else DONE.
   const bool trivial = !c.leaf && !__any_sync(0xffffffffu, (F | S) != 0);
-  if (trivial) {
+  if (p.list) {
+    // List: no compaction — no internal node is hashed, inserted or looked up;
+    // phase 3 emits every FIRST / SHIFT leaf as an entry of its own (R13 order follows
+    // from the stage-0 compaction below), and nothing climbs.
+    if (PHASE == 3) {
+      for (uint32_t m = F | S; m; m &= m - 1) {
+        const uint32_t b = __ffs(m) - 1;
+        emit_region(c, ws, 0, (uint32_t)lane * 32 + b, (F >> b) & 1u, 0ull);
+      }
+      for (uint32_t m = lF1 | lS1; m; m &= m - 1) {   // leaves at height 1 (R3, n != 2^h)
+        const uint32_t b = __ffs(m) - 1;
+        emit_region(c, ws, 1, (uint32_t)lane * 32 + b, (lF1 >> b) & 1u, 0ull);
+      }
+      __syncwarp();
+    }
+    F = 0; S = 0; X = 0;
+  } else if (trivial) {
     const bool allX = __all_sync(0xffffffffu, X == valid_word(P0));
     X = (lane == 0 && allX) ? 1u : 0u;
   } else {
@@ -809,6 +825,7 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   // arrival (K1b counted them) processes the parent. In the steady state no tile is full
   // and nothing climbs.
   auto climb = [&](Ctx& c) {
+    if (p.list) return;   // List: no tree above the leaves
     while (c.s < p.S - 1) {
       const bool full = c.s == 0 ? tile_full(p.g, p.tcc, c.G) : __ldcg(p.st[c.s].dcnt + c.G) == (1u << c.gsz);
       if (!full) return;

@@ -22,6 +22,7 @@ constexpr int kGroupLog = 10;   // upper stages: 1024 positions per group
 constexpr int kLeafThreads = 256;
 constexpr int kTreeThreads = 256;
 constexpr int kTilesPerBlock = 1024;  // compaction: tiles per reduce/offsets CTA
+constexpr int kModeTree = 0, kModeList = 1, kModeBasic = 2;   // = CKPT_MODE_* (include/ckpt.h)
 #ifdef CKPT_K1_STAGES
 constexpr int kLeafStages3d = CKPT_K1_STAGES;   // experiment builds
 #else
@@ -61,6 +62,9 @@ struct InsertParams {
   uint32_t* dcnt[kMaxStages];    // out: s >= 1, FULL children per group (the climb target)
   ulonglong4* trace;             // diagnostics (CKPT_TRACE)
   uint32_t* trace_n;
+  int mode;                      // CKPT_MODE_*: Basic accumulates the gather's prefix inputs in K1
+  unsigned long long* blocksum;  // Basic: per 1024 tree tiles (#changed, 0, changed bytes)
+  unsigned long long* gsum;      // Basic: per 32 tree tiles, the same
 };
 
 struct LeafParams {
@@ -114,6 +118,7 @@ struct TreeParams {
   unsigned long long* gsum;      // per 32 tiles: the same sums
   Totals* tot;
   int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
+  int list;                    // CKPT_MODE_LIST: no compaction, every FIRST/SHIFT leaf is an entry
   ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
   uint32_t* trace_n;
   StageParams st[kMaxStages];
@@ -137,6 +142,10 @@ struct CompactParams {
   int dbg;                       // diagnostics only (CKPT_DBG bits; 0 in production)
   uint4* ctr_next;               // the next call's counter block, zeroed by the data kernel
   uint64_t ctr_next_words;
+  int mode;                      // CKPT_MODE_*: header flags; Basic writes the bitmap instead of entries
+  const uint32_t* cand;          // Basic: the changed-chunk bitmap (K1)
+  uint64_t nwords;               // Basic: its u32 words
+  const uint32_t* tcc;           // Basic: changed chunks per tree tile (K1)
 };
 
 // Per stage-0 tile, written by phase 2: the resolved leaf masks for phase 3 (F0 S0 X0 F1 S1
@@ -204,6 +213,8 @@ cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long lo
                                   size_t scan_tmp_bytes, cudaStream_t st);
 cudaError_t restore_prepare_shift(const Geo& g, RestoreDiff& d, const RestoreDiff* chain_dev, unsigned long long* tmp_len,
                                   int* err, void* scan_tmp, size_t scan_tmp_bytes, cudaStream_t st);
+cudaError_t restore_prepare_basic(const Geo& g, RestoreDiff& d, uint64_t nwords, unsigned long long* tmp_cnt,
+                                  void* scan_tmp, size_t scan_tmp_bytes, cudaStream_t st);
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st);
 uint64_t restore_segments(uint64_t bytes);
 cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,

@@ -34,6 +34,7 @@ def test_strerror_and_create_without_gpu():
     assert "collision" in ckpt.strerror(6)
     h = ctypes.c_void_p()
     assert ckpt.lib().ckpt_create(40, ctypes.byref(h)) == ckpt.CKPT_EINVAL   # argument check first
+    assert ckpt.lib().ckpt_create_mode(128, 3, ctypes.byref(h)) == ckpt.CKPT_EINVAL   # unknown method
 
 
 def test_kernels_are_sm100a_with_tma_and_128bit_cas():

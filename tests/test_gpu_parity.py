@@ -23,10 +23,10 @@ STAT_KEYS = ["n_first_regions", "n_shift_regions", "n_first", "n_fixed", "n_spat
              "list_entries", "meta_bytes", "data_bytes", "bytes", "phase2_inserts"]
 
 
-def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check_restore=True):
+def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check_restore=True, mode=0):
     from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
-    o = oracle_mod.Oracle(C)
-    ck = Checkpointer(C)
+    o = oracle_mod.Oracle(C, mode=mode)
+    ck = Checkpointer(C, mode)
     B = bufs[0].size
     devs = []
     for k, b in enumerate(bufs):
@@ -43,6 +43,7 @@ def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check
         w = o.diff(k)
         if g != w:
             pg, pw = oracle_mod.parse_diff(g), oracle_mod.parse_diff(w)
+            assert pg.get("changed") == pw.get("changed"), k
             assert pg["first"] == pw["first"], k
             assert pg["shift"] == pw["shift"], k
             assert g[:64] == w[:64], k
