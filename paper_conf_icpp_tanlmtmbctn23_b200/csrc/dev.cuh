@@ -43,12 +43,14 @@ __device__ __forceinline__ uint64_t rotl(uint64_t x) {
 }
 __device__ __forceinline__ uint64_t rotl(uint64_t x, int r) { return (x << r) | (x >> (64 - r)); }
 
-// x * C mod 2^64 as IMAD.WIDE.U32 + 2 IMAD (C a compile-time constant)
+// x * C mod 2^64 (C a compile-time constant)
 template <uint64_t C>
 __device__ __forceinline__ uint64_t mulc(uint64_t x) {
   const uint32_t lo = (uint32_t)x, hi = (uint32_t)(x >> 32);
-#ifdef CKPT_MULC3
-  // three IMADs, the high word accumulated through two mad.lo (no separate add)
+#ifndef CKPT_MULC_WIDE
+  // lo*lo as mul.lo / mul.hi and the high word accumulated through two mad.lo (no 64-bit
+  // IMAD.WIDE, no separate add): measured 4-7 % faster K1 at C = 32 / 64, where hashing is
+  // the bound, and neutral at C >= 128 (memory-bound)
   uint32_t wlo, whi, h;
   asm("mul.lo.u32 %0, %3, %4;\n\t"
       "mul.hi.u32 %1, %3, %4;\n\t"

@@ -31,15 +31,16 @@ sys.path.insert(0, ROOT)
 GiB = 1 << 30
 
 
-def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1):
+def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=False):
     import torch
     from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
     from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
     seed = W.seed_of(cfg)
     buf = torch.empty(B, dtype=torch.uint8, device="cuda")
-    ck = Checkpointer(C)
+    ck = Checkpointer(C, mode)
     ck.set_profiling(prof)
-    diffs, ts, walls, phases = [], [], [], []
+    diffs, ts, walls, phases, d2hs = [], [], [], [], []
+    hbuf = torch.empty(B + 64 + 12 * ((B + C - 1) // C) + 16, dtype=torch.uint8).pin_memory() if d2h else None
     t_gen = 0.0
     for k in range(K):
         g0 = time.perf_counter()
@@ -59,6 +60,10 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1):
         pt = ck.phase_times(k)
         ts.append(pt["total"])
         phases.append(pt)
+        if d2h:   # the paper's throughput includes one D2H of the consolidated diff
+            h0 = time.perf_counter()
+            ck.diff_to_host(k, hbuf)
+            d2hs.append(time.perf_counter() - h0)
     out = torch.empty_like(buf)
     r0 = time.perf_counter()
     ck.restore(K - 1, out)
@@ -82,6 +87,7 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1):
     sum_b_st = sum(d["bytes"] for d in st)
     rec = {
         "case": name, "config": cfg, "buffer_bytes": B, "chunk_bytes": C, "checkpoints": K, "update_rate": p,
+        "method": ["tree", "list", "basic"][mode],
         "steady_gbs": round((K - 1) * B / (sum(t_st) / 1e3) / 1e9, 1),
         "steady_ms_median": round(statistics.median(t_st), 4),
         "steady_ms_min": round(min(t_st), 4), "steady_ms_max": round(max(t_st), 4),
@@ -103,6 +109,11 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1):
         "gen_s": round(t_gen, 2),
         "profiling_level": prof,
     }
+    if d2h:
+        # "the size of the original data divided by the time it takes to create and copy
+        # the incremental checkpoint from the GPU to the host memory" (steady checkpoints)
+        rec["paper_throughput_gbs"] = round((K - 1) * B / (sum(t_st) / 1e3 + sum(d2hs[1:])) / 1e9, 1)
+        rec["d2h_s_steady_mean"] = round(sum(d2hs[1:]) / max(1, K - 1), 6)
     if prof >= 2:   # events between every kernel (breaks PDL overlap: a breakdown, not a rate)
         rec["phase_ms_steady_mean"] = {x: round(sum(q[x] for q in phases[1:]) / max(1, K - 1), 4)
                                        for x in ("leaf_hash", "insert", "phase2", "phase3", "compact", "total")}
@@ -116,6 +127,9 @@ def main():
     ap.add_argument("--small", action="store_true", help="quick shapes (CI / smoke of the tool)")
     ap.add_argument("--prof", type=int, default=1, help="library profiling level (2: per-phase breakdown)")
     ap.add_argument("--k", type=int, default=0, help="override the number of checkpoints")
+    ap.add_argument("--methods", action="store_true",
+                    help="Fig. 4 analogue: Tree / List / Basic over C = 32..512 on config 2 (1 GiB, K = 10), "
+                         "with the paper's create + D2H throughput")
     a = ap.parse_args()
     import torch
     from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
@@ -134,11 +148,17 @@ def main():
         cases.append(("cfg4_dup_heavy", 4, GiB // s, 128, 50, 0.0, "dup"))
     if 5 in only:
         cases.append(("cfg5_16GiB_1gpu", 5, 16 * GiB // s, 128, 10, 0.01, None))
+    cases = [c + (0, False) for c in cases]
+    if a.methods:
+        cases = []
+        for C in (32, 64, 128, 256, 512):
+            for m, nm in ((0, "tree"), (1, "list"), (2, "basic")):
+                cases.append((f"methods_{nm}_C{C}", 2, GiB // s, C, 10, 0.01, None, m, True))
     recs = []
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
-    for name, cfg, B, C, K, p, hg in cases:
+    for name, cfg, B, C, K, p, hg, mode, d2h in cases:
         gen = W.DupHeavy(B, C, W.seed_of(cfg)) if hg == "dup" else None
-        r = run_case(name, cfg, B, C, a.k or K, p, stream, gen, a.prof)
+        r = run_case(name, cfg, B, C, a.k or K, p, stream, gen, a.prof, mode, d2h)
         r["device"] = torch.cuda.get_device_name(0)
         print(json.dumps(r), flush=True)
         recs.append(r)
