@@ -644,6 +644,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.cand = h->cand;
   cp.nwords = h->nwords;
   cp.tcc = h->tcc;
+  cp.parts = gather_parts(h->ngroups[0], h->C, h->num_sms);
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
   const auto t_launched = clk::now();

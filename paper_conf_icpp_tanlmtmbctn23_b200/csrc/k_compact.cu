@@ -41,11 +41,12 @@ constexpr int kCT = 256;
 // would serialise those requests.
 constexpr int kGW = kCT / 32;
 
-constexpr int kStageUnits = 768;   // 12 KB of 16-byte units staged per warp and round
+constexpr int kStageUnits = 640;   // 10 KB of 16-byte units staged per warp and round
 
 struct GatherWarp {
   uint32_t pre[32];   // FIRST chunks in the mask words before word i
   uint32_t fw[32];    // the tile's FIRST-chunk mask words
+  uint16_t idx[1 << kTileLog];   // the k-th FIRST chunk of the tile (offset from its first chunk)
   uint4 stage[kStageUnits];
 };
 
@@ -73,9 +74,15 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   const uint64_t nblk = (p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock;
   const uint64_t nwarps = (uint64_t)gridDim.x * kGW;
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
-  uint64_t w = (uint64_t)blockIdx.x * kGW + wid;
+  // worklist entry w -> block w mod grid, warp w / grid: with few dirty tiles (large chunks)
+  // every SM still gets work
+  uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x;
+  // A tile's data may be split over `parts` warps (large chunks, few tiles): work item w is
+  // part w mod parts of the (w / parts)-th dirty tile; part j copies staging rounds
+  // j, j + parts, ... and part 0 also writes the tile's entries.
+  const uint32_t parts = p.parts;
   // the worklist entry is loaded before the count check (the array has n_tiles entries)
-  uint64_t T = w < p.n_tiles ? __ldg(p.wl0 + w) : 0;
+  uint64_t T = w / parts < p.n_tiles ? __ldg(p.wl0 + w / parts) : 0;
 
   // totals = sum of the per-1024-tile block sums (every warp; 8 values at 1 GiB, C = 128)
   unsigned long long nF_tot = 0, nS_tot = 0, data_tot = 0;
@@ -119,8 +126,10 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   uint8_t* const ent_s = p.out + 64 + 4 * nF_tot;
   uint8_t* const dat = p.out + meta;
   const uint32_t U = g.C / 16;   // 16-byte units per chunk
+  const int ulog = (U & (U - 1)) ? -1 : __ffs(U) - 1;   // shift instead of a division when C = 2^j
 
-  for (; w < count; w += nwarps) {
+  for (; w < (uint64_t)count * parts; w += nwarps) {
+    const uint32_t part = (uint32_t)(w % parts);
     unsigned long long tg0 = 0, tg1 = 0, tg2 = 0;
     if (p.trace) tg0 = gtime_ns();
     // one round of loads: counts, FIRST-chunk mask, the first 64 region records, prefix sums
@@ -177,7 +186,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       }
     }
     const uint64_t Tcur = T;
-    if (w + nwarps < count) T = __ldg(p.wl0 + w + nwarps);   // next tile, early
+    if (w + nwarps < (uint64_t)count * parts) T = __ldg(p.wl0 + (w + nwarps) / parts);   // next tile, early
     if (cnt.w != g.epoch) {
       warp_sum3(pF, pS, pD);
       continue;
@@ -194,6 +203,10 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     }
     gw.pre[lane] = incl - pc;
     gw.fw[lane] = fw;
+    {   // the tile's FIRST chunks as a list (k-th FIRST chunk -> offset in the tile)
+      uint32_t r = incl - pc;
+      for (uint32_t m = fw; m; m &= m - 1) gw.idx[r++] = (uint16_t)(32u * lane + (__ffs(m) - 1));
+    }
     const uint32_t nch = __shfl_sync(0xffffffffu, incl, 31);
     __syncwarp();
     // the FIRST bytes: unit x of the tile's stream = unit (x mod U) of its (x / U)-th chunk,
@@ -204,17 +217,13 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     // units entirely past B are skipped.
     const uint32_t nunits = nch * U;
     auto unit_src = [&](uint32_t x) -> unsigned long long {
-      const uint32_t k = x / U, sub = x - k * U;
-      int i = 0;   // last word with pre <= k (words without FIRST chunks are skipped)
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1)
-        if (gw.pre[i + step] <= k) i += step;   // i + step <= 31
-      const uint32_t bit = __fns(gw.fw[i], 0, (int)(k - gw.pre[i] + 1));
-      return (lo + 32u * i + bit) * (unsigned long long)g.C + 16u * sub;
+      const uint32_t k = ulog >= 0 ? x >> ulog : x / U, sub = x - k * U;
+      return (lo + gw.idx[k]) * (unsigned long long)g.C + 16u * sub;
     };
-    bool entries_done = false;
-    for (uint32_t x0 = 0; x0 < nunits || !entries_done; x0 += kStageUnits) {
-      const uint32_t x1 = nunits - x0 < (uint32_t)kStageUnits ? nunits : x0 + kStageUnits;
+    bool entries_done = part != 0;
+    if (entries_done) warp_sum3(pF, pS, pD);   // part 0 sums them while its first round is in flight
+    for (uint32_t x0 = part * kStageUnits; x0 < nunits || !entries_done; x0 += parts * kStageUnits) {
+      const uint32_t x1 = x0 + kStageUnits < nunits ? x0 + kStageUnits : nunits;
       for (uint32_t x = x0 + lane; x < x1; x += 32) {
         const unsigned long long so = unit_src(x);
         if (so < g.B) cp_async16(&gw.stage[x - x0], p.buf + so, g.B - so >= 16 ? 16u : (uint32_t)(g.B - so));
@@ -238,7 +247,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       __syncwarp();
       for (uint32_t x = x0 + lane; x < x1; x += 32) {
         // only the tile's last FIRST chunk, in the tile holding the buffer's end, can be short
-        if (hi == g.n && x / U + 1 == nch && unit_src(x) >= g.B) continue;
+        if (hi == g.n && (ulog >= 0 ? x >> ulog : x / U) + 1 == nch && unit_src(x) >= g.B) continue;
         *reinterpret_cast<uint4*>(dat + pD + 16ull * x) = gw.stage[x - x0];
       }
       __syncwarp();
@@ -258,11 +267,21 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
 
 static int g_gather_blocks_per_sm = 0;
 
+uint32_t gather_parts(uint64_t n_tiles, uint32_t C, int num_sms) {
+  // split tiles over warps only when there are fewer tiles than resident warps and the
+  // tiles carry many bytes (C >= 512: a 1024-chunk tile spans >= 512 KB)
+  const int bps = g_gather_blocks_per_sm > 0 ? g_gather_blocks_per_sm : 2;
+  const uint64_t warps = (uint64_t)num_sms * bps * kGW;
+  if (C < 512 || n_tiles == 0 || n_tiles >= warps) return 1;
+  const uint64_t r = warps / n_tiles;
+  return (uint32_t)(r > 8 ? 8 : r);
+}
+
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st) {
   // one resident wave of gather blocks (the dirty-tile count is only known on the device,
   // and blocks beyond one wave would only arrive late to find no work)
   const int bps = g_gather_blocks_per_sm > 0 ? g_gather_blocks_per_sm : 2;
-  uint64_t grid = (p.n_tiles + kGW - 1) / kGW;
+  uint64_t grid = p.n_tiles * p.parts;   // worklist entries are spread over the blocks first
   if (grid > (uint64_t)num_sms * bps) grid = (uint64_t)num_sms * bps;
   return launch_pdl(gather_kernel, (unsigned)grid, kCT, kGW * sizeof(GatherWarp), st, p);
 }

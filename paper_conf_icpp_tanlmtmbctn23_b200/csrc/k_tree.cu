@@ -886,7 +886,8 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   // dirty stage-0 tiles (K1b's list); climb on the last DIRTY child of each group
   const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
   const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
-  for (uint64_t w = (uint64_t)blockIdx.x * kWarps + wid; w < count; w += nwarps) {
+  // worklist entry w -> block w mod grid, warp w / grid: dirty tiles spread over all SMs
+  for (uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x; w < count; w += nwarps) {
     const uint64_t T = __ldcg(p.wl0 + w);
     Ctx c = run_tile(T);
     climb(c);
@@ -926,8 +927,7 @@ cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_
   // all CTAs resident at once (static tile striding relies on it): occupancy-sized grid
   const int bps = g_tree_blocks_per_sm[phase - 2] > 0 ? g_tree_blocks_per_sm[phase - 2] : 2;
   uint64_t grid = (uint64_t)num_sms * bps;
-  const uint64_t need = (p.n_tiles + kWarps - 1) / kWarps;   // one warp per tile when it fits
-  if (grid > need) grid = need ? need : 1;
+  if (grid > p.n_tiles) grid = p.n_tiles ? p.n_tiles : 1;   // worklist spread over blocks first
   const size_t smem = kWarps * sizeof(WarpSmem);
   if (phase == 2) return launch_pdl(tree_kernel<2>, (unsigned)grid, kTreeThreads, smem, st, p);
   return launch_pdl(tree_kernel<3>, (unsigned)grid, kTreeThreads, smem, st, p);

@@ -146,6 +146,7 @@ struct CompactParams {
   const uint32_t* cand;          // Basic: the changed-chunk bitmap (K1)
   uint64_t nwords;               // Basic: its u32 words
   const uint32_t* tcc;           // Basic: changed chunks per tree tile (K1)
+  uint32_t parts;                // warps per dirty tile (gather_parts)
 };
 
 // Per stage-0 tile, written by phase 2: the resolved leaf masks for phase 3 (F0 S0 X0 F1 S1
@@ -193,6 +194,7 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
 cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st);
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st);
+uint32_t gather_parts(uint64_t n_tiles, uint32_t C, int num_sms);
 cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, uint64_t new_cap, cudaStream_t st);
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
 
