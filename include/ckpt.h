@@ -108,7 +108,8 @@ CKPT_API int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out);
  *            same B (R17: the fixed-duplicate test is positional).
  *   stream   cudaStream_t (as void*) all GPU work is enqueued on, in order.
  *   diff     receives the statistics and the device pointer of the new diff.
- * The call returns after exactly one host synchronisation with `stream` (the process
+ * The call returns after exactly one host synchronisation with `stream` (a spin on the
+ * completion the last kernel publishes to mapped host memory; the process
  * "stops during checkpointing"). Capacity for the record table and the diff is
  * reserved before the first kernel, so an error leaves the lineage unchanged.
  * Errors: CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ESTATE, CKPT_ECOLLIDE. */

@@ -146,12 +146,13 @@ class Checkpointer:
         self._h = h
         self.chunk_bytes = chunk_bytes
         self.mode = mode
+        self._ckpt_fn = lib().ckpt_checkpoint   # bound once: the per-call path is marshalling only
 
     # ------------------------------------------------------------------ core calls
     def checkpoint(self, buf, nbytes: int | None = None, stream=None, raw: bool = False):
         d = CkptDiff()
         n = _nbytes(buf) if nbytes is None else nbytes
-        rc = lib().ckpt_checkpoint(self._h, _ptr(buf), n, _stream_handle(stream), ctypes.byref(d))
+        rc = self._ckpt_fn(self._h, _ptr(buf), n, _stream_handle(stream), ctypes.byref(d))
         if rc != CKPT_OK:
             raise CkptError(rc, "ckpt_checkpoint")
         return d if raw else d.as_dict()

@@ -262,6 +262,16 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     }
   }
   __syncthreads();
+  if (threadIdx.x == 0) {
+    // the last block to finish publishes completion to the host (mapped memory): every
+    // byte of the diff is written, and every read of the caller's buffer is done. The
+    // system-scope fence orders block 0's mapped totals before the publication.
+    __threadfence_system();
+    if (atomicAdd(&p.tot->blocks_done, 1u) + 1 == gridDim.x) {
+      __threadfence_system();
+      *reinterpret_cast<volatile uint32_t*>(&p.tot_host->done) = g.epoch;
+    }
+  }
   trace_block(p.trace, p.trace_n, bt0, bt1, 5);
 }
 

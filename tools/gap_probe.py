@@ -33,3 +33,32 @@ print("events ms/step %.4f" % (e0.elapsed_time(e1) / n))
 print("python wall ms/call %.4f" % (1e3 * statistics.mean(walls)))
 for key in ("total", "leaf_hash", "host_pre", "host_enqueue", "host_sync_wait", "host_post"):
     print("%-15s %.4f" % (key, statistics.mean(h[key] for h in hp)))
+
+# A/B on fresh handles over the same lineage: raw C ABI call with prebuilt ctypes
+# arguments vs Checkpointer.checkpoint (the binding's per-call Python cost)
+import ctypes
+from paper_conf_icpp_tanlmtmbctn23_b200 import ckpt as _ck
+L = _ck.lib()
+f = L.ckpt_checkpoint
+sth = ctypes.c_void_p(st.cuda_stream)
+ptrs = [ctypes.c_void_p(b.data_ptr()) for b in bufs]
+nb = ctypes.c_uint64(B)
+for rep in range(2):
+    for kind in ("raw", "binding"):
+        c2 = Checkpointer(C)
+        c2.set_profiling(1)
+        for k in range(3):
+            c2.checkpoint(bufs[k], stream=st)
+        outs = [_ck.CkptDiff() for _ in range(K)]
+        hh = c2._h
+        torch.cuda.synchronize()
+        e0.record(st)
+        if kind == "raw":
+            for k in range(3, K):
+                f(hh, ptrs[k], nb, sth, ctypes.byref(outs[k]))
+        else:
+            for k in range(3, K):
+                c2.checkpoint(bufs[k], nbytes=B, stream=st, raw=True)
+        e1.record(st); st.synchronize()
+        print("%-8s events ms/step %.4f" % (kind, e0.elapsed_time(e1) / n))
+        c2.close()
