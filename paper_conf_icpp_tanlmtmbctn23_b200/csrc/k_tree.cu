@@ -755,38 +755,45 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
       if (lane >= o) { iF += a; iS += b; }
     }
     const uint32_t nFt = __shfl_sync(0xffffffffu, iF, 31), nSt = __shfl_sync(0xffffffffu, iS, 31);
-    uint32_t rf = iF - __popc(wF), rs = nFt + iS - __popc(wS);
+    // Records j = 0 .. nFt + nSt - 1 spread evenly over the lanes (j = base + 32 t + lane):
+    // record j is the j-th FIRST region start (chunk order) or the (j - nFt)-th SHIFT one,
+    // found by a search over the per-word exclusive prefixes; the source loads of a lane's
+    // SHIFT records are all issued before any record is written.
+    ws.W[lane] = iF - __popc(wF);
+    ws.WP[lane] = iS - __popc(wS);
+    __syncwarp();
     uint4* out = p.scratch + (c.G << g.t0);
-    for (uint32_t m = wF; m; m &= m - 1) {
-      const uint32_t slot = lane * 32 + (__ffs(m) - 1);
-      const int lv = ws.lvl[slot];
-      const uint64_t gpos = (c.G << (gsz - lv)) + (slot >> lv);
-      out[rf++] = make_uint4(node_id(g, lv, gpos), 0u, 0u, L_FIRST);
-
-    }
-    for (uint32_t m = wS; m;) {   // batches of 4: issue the source loads first
-      uint32_t slots[4];
-      unsigned long long src[4];
-      int nb = 0;
+    const uint32_t R = nFt + nSt;
+    constexpr int kE = 4;
+    for (uint32_t base = 0; base < R; base += 32 * kE) {
+      uint32_t slot[kE];
+      int lv[kE];
+      unsigned long long src[kE];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        if (m) {
-          const uint32_t b = __ffs(m) - 1;
-          m &= m - 1;
-          slots[u] = lane * 32 + b;
-          const int lv = ws.lvl[slots[u]];
-          src[u] = child_src(c, lv, rev_n(slots[u] >> lv, gsz - lv));
-          nb = u + 1;
+      for (int t = 0; t < kE; ++t) {
+        const uint32_t j = base + 32 * t + lane;
+        slot[t] = ~0u;
+        if (j < R) {
+          const bool isF = j < nFt;
+          const uint32_t r = isF ? j : j - nFt;
+          const uint32_t* pre = isF ? ws.W : ws.WP;
+          int i = 0;   // last word with pre <= r
+#pragma unroll
+          for (int step = 16; step > 0; step >>= 1)
+            if (pre[i + step] <= r) i += step;
+          const uint32_t wd = isF ? ws.stF[i] : ws.stS[i];
+          slot[t] = 32u * i + __fns(wd, 0, (int)(r - pre[i] + 1));
+          lv[t] = ws.lvl[slot[t]];
+          src[t] = isF ? 0ull : child_src(c, lv[t], rev_n(slot[t] >> lv[t], gsz - lv[t]));
         }
       }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        if (u < nb) {
-          const int lv = ws.lvl[slots[u]];
-          const uint64_t gpos = (c.G << (gsz - lv)) + (slots[u] >> lv);
-          out[rs++] = make_uint4(node_id(g, lv, gpos), (uint32_t)(src[u] & 0xffffffffu), (uint32_t)(src[u] >> 32),
-                                 L_SHIFT);
-        }
+      for (int t = 0; t < kE; ++t) {
+        const uint32_t j = base + 32 * t + lane;
+        if (slot[t] == ~0u) continue;
+        const uint64_t gpos = (c.G << (gsz - lv[t])) + (slot[t] >> lv[t]);
+        out[j] = make_uint4(node_id(g, lv[t], gpos), (uint32_t)(src[t] & 0xffffffffu), (uint32_t)(src[t] >> 32),
+                            j < nFt ? L_FIRST : L_SHIFT);
       }
     }
     if (lane == 0) {
