@@ -690,15 +690,17 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
       // the FIRST/SHIFT children of DONE parents are regions
       const uint32_t dchild = to_children(nD, Nc);
       const uint32_t emF = dchild & F, emS = dchild & S;
-      if (__any_sync(0xffffffffu, (emF | emS) != 0)) {
-        for (uint32_t m = emF | emS; m; m &= m - 1) {
-          const uint32_t b = __ffs(m) - 1;
-          const uint32_t rr = (uint32_t)lane * 32 + b;
-          const bool isF = (emF >> b) & 1u;
-          emit_region(c, ws, lv - 1, rr, isF, (isF || c.leaf) ? 0ull : child_src(c, lv - 1, rr));
-        }
-        __syncwarp();
+      // emissions spread evenly over the lanes (a dense word would serialise one lane)
+      ws.T[lane] = emF;
+      const uint32_t ne = batch_begin(ws, emF | emS);
+      for (uint32_t j = lane; j < ne; j += 32) {
+        uint32_t w, b;
+        batch_item(ws, j, w, b);
+        const bool isF = (ws.T[w] >> b) & 1u;
+        const uint32_t rr = w * 32 + b;
+        emit_region(c, ws, lv - 1, rr, isF, (isF || c.leaf) ? 0ull : child_src(c, lv - 1, rr));
       }
+      __syncwarp();
       F = bothF | (lv == 1 ? lF1 : 0u);
       X = bothX | (lv == 1 ? lX1 : 0u);
       S = hitS | (lv == 1 ? lS1 : 0u);
