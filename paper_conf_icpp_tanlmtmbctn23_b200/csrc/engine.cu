@@ -40,8 +40,11 @@ struct DiffRec {
   bool planned = false;
 };
 
-constexpr double kMaxLoad = 0.8;     // reserve so that even a worst-case checkpoint stays below this
-constexpr double kGrowLoad = 0.6;    // load factor right after a growth
+#ifndef CKPT_TABLE_GROW_LOAD
+#define CKPT_TABLE_GROW_LOAD 0.6
+#endif
+constexpr double kGrowLoad = CKPT_TABLE_GROW_LOAD;   // load factor right after a growth
+constexpr double kMaxLoad = kGrowLoad + 0.2;         // reserve so that even a worst-case checkpoint stays below this
 constexpr uint64_t kArenaVA[] = {4ull << 40, 1ull << 40, 256ull << 30, 64ull << 30};
 
 }  // namespace
