@@ -387,6 +387,22 @@ def run_ours(args):
     rs = time.perf_counter() - r0
     restore_ok = bool(torch.equal(out, bufs[Wm + K - 1]))
 
+    # restart (NEXT #3): rebuild the whole lineage on a fresh handle from host copies of the
+    # diffs (restore + re-de-duplication + byte check per diff), then check the newest restore
+    host_diffs = [ck.diff_to_host(i) for i in range(Wm + K)]
+    ck3 = Checkpointer(C)
+    torch.cuda.synchronize()
+    i0 = time.perf_counter()
+    for hd in host_diffs:
+        ck3.import_diff(hd, stream=stream)
+    torch.cuda.synchronize()
+    imp_s = time.perf_counter() - i0
+    out.zero_()
+    ck3.restore(Wm + K - 1, out)
+    import_ok = bool(torch.equal(out, bufs[Wm + K - 1]))
+    ck3.close()
+    del host_diffs
+
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         try:
@@ -428,6 +444,8 @@ def run_ours(args):
             "restore": {"id": Wm + K - 1, "s": round(rs, 5), "gbs": round(B / rs / 1e9, 2), "ok": restore_ok,
                         "cold_s": round(rs_cold, 5), "note": "host wall time of ckpt_restore (synchronous); cold = "
                                                              "first restore, which builds the per-diff plans"},
+            "restart_import": {"diffs": Wm + K, "s": round(imp_s, 4), "ok": import_ok,
+                               "note": "ckpt_import of every diff from host memory into a fresh handle"},
             "file_offsets_rank0": offsets[0][:3],
             "e2e": {"value": round(e2e_val, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d // max(1, Ke),
                     "d2h_bytes_per_step": d2h // max(1, Ke), "steps": Ke},

@@ -143,6 +143,20 @@ CKPT_API int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint6
 CKPT_API int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, void* stream,
                          void* host_diff, uint64_t host_diff_cap, ckpt_diff* diff);
 
+/* Rebuild a lineage after a restart (the GPU cannot keep the
+ * record across runs, the diffs live in host memory / storage): appends diff `id` =
+ * ckpt_num_checkpoints() from host memory to this handle as if the checkpoint had just been
+ * taken. The checkpoint is restored from the lineage plus the imported diff and
+ * de-duplicated again, which rebuilds the record and the leaf digests (R5) exactly;
+ * the regenerated diff must equal the imported one byte for byte.
+ *   host_diff  a diff produced by a handle of the same chunk size and method (header
+ *              `flags`), for checkpoint number ckpt_num_checkpoints(h); borrowed.
+ *   bytes      its size; stream as for ckpt_checkpoint (the re-de-duplication runs there).
+ * Synchronous. Errors: CKPT_EINVAL (bad header, wrong id / size / chunk size / method: the
+ * handle is unchanged; or the regenerated diff differs: the handle is poisoned), CKPT_ENOMEM,
+ * CKPT_ECUDA, CKPT_ESTATE. */
+CKPT_API int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stream);
+
 /* Number of checkpoints taken so far. */
 CKPT_API int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count);
 

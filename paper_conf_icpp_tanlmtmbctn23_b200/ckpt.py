@@ -22,7 +22,7 @@ CKPT_MODE_TREE, CKPT_MODE_LIST, CKPT_MODE_BASIC = 0, 1, 2   # methods of P:194 (
 
 ABI_FUNCTIONS = [
     "ckpt_create", "ckpt_create_mode", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
-    "ckpt_checkpoint_host", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
+    "ckpt_checkpoint_host", "ckpt_import", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
     "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
     "ckpt_strerror",
 ]
@@ -83,6 +83,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_diff_to_host": ([vp, u32, vp, u64], i32),
             "ckpt_checkpoint_host": ([vp, vp, u64, vp, vp, u64, P(CkptDiff)], i32),
             "ckpt_num_checkpoints": ([vp, P(u32)], i32),
+            "ckpt_import": ([vp, vp, u64, vp], i32),
             "ckpt_leaf_digests": ([vp, vp], i32),
             "ckpt_record_dump": ([vp, vp, vp, vp, u64, P(u64)], i32),
             "ckpt_set_profiling": ([vp, i32], i32),
@@ -166,6 +167,18 @@ class Checkpointer:
         if rc != CKPT_OK:
             raise CkptError(rc, "ckpt_checkpoint_host")
         return d.as_dict()
+
+    def import_diff(self, host_diff, stream=None) -> None:
+        """Append diff number num_checkpoints from host memory (bytes, numpy array or a host
+        tensor) after a restart, rebuilding the record and leaf digests (ckpt_import)."""
+        if isinstance(host_diff, (bytes, bytearray)):
+            buf = ctypes.create_string_buffer(bytes(host_diff), len(host_diff))
+            ptr, n = ctypes.addressof(buf), len(host_diff)
+        else:
+            ptr, n = _ptr(host_diff), _nbytes(host_diff)
+        rc = lib().ckpt_import(self._h, ptr, n, _stream_handle(stream))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_import")
 
     def restore(self, cid: int, out) -> None:
         rc = lib().ckpt_restore(self._h, cid, _ptr(out))

@@ -851,6 +851,98 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
   return CKPT_OK;
 }
 
+static void free_plan(DiffRec& d) {
+  for (unsigned long long** q : {&d.Flo, &d.Foff, &d.Slo, &d.Soff, &d.Ssrc, &d.Fseg, &d.Sseg}) {
+    if (*q) cudaFree(*q);
+    *q = nullptr;
+  }
+  d.planned = false;
+}
+
+int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stream) {
+  if (!h || !host_diff || bytes < 64) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  const uint8_t* hd = static_cast<const uint8_t*>(host_diff);
+  auto rd32h = [&](size_t o) { uint32_t v; std::memcpy(&v, hd + o, 4); return v; };
+  auto rd64h = [&](size_t o) { uint64_t v; std::memcpy(&v, hd + o, 8); return v; };
+  uint16_t ver, flags;
+  std::memcpy(&ver, hd + 4, 2);
+  std::memcpy(&flags, hd + 6, 2);
+  const uint32_t id = (uint32_t)h->diffs.size();
+  const uint64_t B = rd64h(16), n = rd64h(24), nF = rd64h(32), nS = rd64h(40), data = rd64h(48);
+  if (rd32h(0) != 0x44504B43u || ver != 1 || flags != (uint16_t)h->mode || rd32h(8) != id || rd32h(12) != h->C)
+    return CKPT_EINVAL;
+  if (B == 0 || n != (B + h->C - 1) / h->C || n > (1ull << 31) || (h->geo_set && B != h->B)) return CKPT_EINVAL;
+  const uint64_t raw = h->mode == kModeBasic ? 64 + 4 * ((n + 31) / 32) : 64 + 4 * nF + 12 * nS;
+  const uint64_t meta = (raw + 15) & ~15ull;
+  if (meta + data != bytes || data > B || (h->mode == kModeBasic && nS)) return CKPT_EINVAL;
+  if (!h->geo_set) {
+    const int r = setup_geometry(h, B);
+    if (r != CKPT_OK) return r;
+  }
+  if (h->staging_size < B) {
+    if (h->staging) cudaFree(h->staging);
+    h->staging = nullptr;
+    h->staging_size = 0;
+    if (cudaMalloc(&h->staging, B) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
+    h->staging_size = B;
+  }
+  uint8_t* tmp = nullptr;
+  int* flag = nullptr;
+  if (cudaMalloc(&tmp, bytes) != cudaSuccess || cudaMalloc(&flag, sizeof(int)) != cudaSuccess) {
+    cudaGetLastError();
+    cudaFree(tmp);
+    return CKPT_ENOMEM;
+  }
+  auto cleanup = [&]() { cudaFree(tmp); cudaFree(flag); };
+  cudaStream_t in = h->internal;
+  if (cudaMemcpyAsync(tmp, host_diff, bytes, cudaMemcpyHostToDevice, in) != cudaSuccess ||
+      cudaStreamSynchronize(in) != cudaSuccess) {
+    cleanup();
+    h->poisoned = true;
+    return CKPT_ECUDA;
+  }
+  // 1. restore checkpoint `id` from diffs 0..id-1 plus the imported diff
+  DiffRec rec;
+  std::memset(&rec.info, 0, sizeof(rec.info));
+  rec.info.id = id;
+  rec.info.n_first_regions = nF;
+  rec.info.n_shift_regions = nS;
+  rec.info.meta_bytes = meta;
+  rec.info.data_bytes = data;
+  rec.info.bytes = bytes;
+  rec.ptr = tmp;
+  h->diffs.push_back(rec);
+  int rc = ckpt_restore(h, id, h->staging);
+  free_plan(h->diffs.back());
+  h->diffs.pop_back();
+  if (rc != CKPT_OK) { cleanup(); return rc == CKPT_EINVAL ? CKPT_EINVAL : rc; }
+  // 2. de-duplicate it again: rebuilds the record and the leaf digests exactly
+  ckpt_diff d;
+  rc = ckpt_checkpoint(h, h->staging, B, stream, &d);
+  if (rc != CKPT_OK && rc != CKPT_ECOLLIDE) { cleanup(); return rc; }
+  // 3. the regenerated diff must be the imported one
+  int mismatch = d.bytes != bytes;
+  if (!mismatch) {
+    int hf = 0;
+    if (cudaMemsetAsync(flag, 0, sizeof(int), in) != cudaSuccess ||
+        device_compare(d.dev_ptr, tmp, bytes, flag, h->num_sms, in) != cudaSuccess ||
+        cudaMemcpyAsync(&hf, flag, sizeof(int), cudaMemcpyDeviceToHost, in) != cudaSuccess ||
+        cudaStreamSynchronize(in) != cudaSuccess) {
+      cleanup();
+      h->poisoned = true;
+      return CKPT_ECUDA;
+    }
+    mismatch = hf;
+  }
+  cleanup();
+  if (mismatch) {
+    h->poisoned = true;   // the lineage no longer matches the imported diffs
+    return CKPT_EINVAL;
+  }
+  return CKPT_OK;
+}
+
 int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
   if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;

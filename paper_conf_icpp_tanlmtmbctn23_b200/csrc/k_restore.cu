@@ -314,6 +314,24 @@ cudaError_t restore_prepare_basic(const Geo& g, RestoreDiff& d, uint64_t nwords,
   return cudaGetLastError();
 }
 
+__global__ void compare_kernel(const uint4* a, const uint4* b, uint64_t n16, const uint8_t* ta, const uint8_t* tb,
+                               uint32_t ntail, int* diff) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint4 x = a[i], y = b[i];
+    if (x.x != y.x || x.y != y.y || x.z != y.z || x.w != y.w) *diff = 1;
+  }
+  if (blockIdx.x == 0 && threadIdx.x < ntail && ta[threadIdx.x] != tb[threadIdx.x]) *diff = 1;
+}
+
+cudaError_t device_compare(const void* a, const void* b, uint64_t bytes, int* diff, int num_sms, cudaStream_t st) {
+  const uint64_t n16 = bytes / 16;
+  compare_kernel<<<num_sms * 4, 256, 0, st>>>(reinterpret_cast<const uint4*>(a), reinterpret_cast<const uint4*>(b), n16,
+                                              static_cast<const uint8_t*>(a) + 16 * n16,
+                                              static_cast<const uint8_t*>(b) + 16 * n16, (uint32_t)(bytes % 16), diff);
+  note_launch();
+  return cudaGetLastError();
+}
+
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st) {
   if (d.nF) {
     const uint64_t ns = (d.data_bytes + kPaintSeg - 1) / kPaintSeg;
@@ -351,6 +369,7 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, segmap_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_count_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_expand_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, compare_kernel);
   return e;
 }
 
