@@ -58,6 +58,8 @@ def lib() -> ctypes.CDLL:
         L.orc_create.restype = ctypes.c_void_p
         L.orc_create_mode.argtypes = [ctypes.c_uint32, ctypes.c_int, ctypes.c_int]
         L.orc_create_mode.restype = ctypes.c_void_p
+        L.orc_set_variant.argtypes = [ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint32]
+        L.orc_set_variant.restype = ctypes.c_int
         L.orc_destroy.argtypes = [ctypes.c_void_p]
         L.orc_destroy.restype = None
         L.orc_checkpoint.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_uint64]
@@ -103,6 +105,8 @@ def mmh3(data: bytes, seed: int = 0) -> bytes:
 
 
 MODE_TREE, MODE_LIST, MODE_BASIC = 0, 1, 2   # the methods compared in P:194 (Tree = ours)
+VAR_FULL_FIRST, VAR_FULL_SWITCH = 1, 2       # Tree-method variants (NEXT #4)
+FLAGS_FULL = 3                               # header flags of a difference stored in full
 
 
 class Oracle:
@@ -117,6 +121,11 @@ class Oracle:
         self.ideal = ideal
         self.mode = mode
         self.buf_bytes = None
+
+    def set_variant(self, flags: int, switch_permille: int = 1000) -> None:
+        """VAR_FULL_FIRST / VAR_FULL_SWITCH (Tree mode, before the first checkpoint)."""
+        if lib().orc_set_variant(self._h, flags, switch_permille) != 0:
+            raise ValueError("variant rejected")
 
     def close(self):
         if self._h:
