@@ -87,6 +87,27 @@ typedef struct {
  *                    order at their true length. No record. */
 enum { CKPT_MODE_TREE = 0, CKPT_MODE_LIST = 1, CKPT_MODE_BASIC = 2 };
 
+/* Variants of the Tree method (readings R22, R23). Set with
+ * ckpt_set_variant before the handle's first checkpoint.
+ *   CKPT_VARIANT_FULL_FIRST   "a single first checkpoint that was taken fully", "we
+ *                             capture a full initial checkpoint": checkpoint 0 runs
+ *                             Algorithm 1 as usual (same record, same statistics of its
+ *                             leaves), but its difference is stored in full.
+ *   CKPT_VARIANT_FULL_SWITCH  "the worst-case scenario encountered only when the checkpointed
+ *                             data fully changes during the checkpoint interval. This can be
+ *                             easily detected, and incremental checkpointing can be
+ *                             deactivated accordingly": a checkpoint k >= 1 with
+ *                             1000 * (non-FIXED leaves) >= switch_permille * n is stored in
+ *                             full and makes no record operation (Alg.1 l.6-46 skipped; the
+ *                             leaf digests are still updated, l.21). Its statistics count the
+ *                             changed chunks as n_first (n_spatial = n_temporal = 0) and
+ *                             phase2_inserts = 0; record_size is unchanged.
+ * A difference stored in full has header flags CKPT_FLAGS_FULL and the Tree layout with
+ * n_first_regions = 1 (the root, node 0), n_shift_regions = 0 and the whole buffer as data
+ * (meta_bytes = 80, data_bytes = B); ckpt_restore and ckpt_import accept it. */
+enum { CKPT_VARIANT_FULL_FIRST = 1, CKPT_VARIANT_FULL_SWITCH = 2 };
+enum { CKPT_FLAGS_FULL = 3 };
+
 /* Create a handle.  P:77: fixed-size chunks of "tens or hundreds of bytes".
  *   chunk_bytes  C, a multiple of 16 with 32 <= C <= 65536 (C > 2 x 16-B digest).
  *   out          receives the handle (owned by the caller; free with ckpt_destroy).
@@ -100,6 +121,14 @@ CKPT_API int ckpt_create(uint32_t chunk_bytes, ckpt_handle* out);
  * n_first_regions (no spatial / temporal de-duplication).
  * Errors: as ckpt_create, and CKPT_EINVAL for an unknown mode. */
 CKPT_API int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out);
+
+/* Select the Tree-method variants above.
+ *   flags            bitwise OR of CKPT_VARIANT_* (0 = Algorithm 1 only, the default).
+ *   switch_permille  threshold of CKPT_VARIANT_FULL_SWITCH, 0..1000 (1000 = every leaf
+ *                    changed, the paper's "fully changes"); ignored without that flag.
+ * Errors: CKPT_EINVAL (handle not in CKPT_MODE_TREE, a checkpoint already taken, unknown
+ * flag bits, switch_permille > 1000; nothing changed), CKPT_ESTATE. */
+CKPT_API int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_permille);
 
 /* De-duplicate one checkpoint (Alg.1; serialization P:81).
  *   dev_ptr  device buffer of `bytes` bytes, 16-byte aligned, BORROWED for the call; the

@@ -19,9 +19,11 @@ from . import _build
 CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_ECOLLIDE = range(7)
 
 CKPT_MODE_TREE, CKPT_MODE_LIST, CKPT_MODE_BASIC = 0, 1, 2   # methods of P:194 (include/ckpt.h)
+CKPT_VARIANT_FULL_FIRST, CKPT_VARIANT_FULL_SWITCH = 1, 2      # Tree variants
+CKPT_FLAGS_FULL = 3                                           # header flags of a full difference
 
 ABI_FUNCTIONS = [
-    "ckpt_create", "ckpt_create_mode", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
+    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
     "ckpt_checkpoint_host", "ckpt_import", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
     "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
     "ckpt_strerror",
@@ -77,6 +79,7 @@ def lib() -> ctypes.CDLL:
         sig = {
             "ckpt_create": ([u32, P(vp)], i32),
             "ckpt_create_mode": ([u32, i32, P(vp)], i32),
+            "ckpt_set_variant": ([vp, u32, u32], i32),
             "ckpt_checkpoint": ([vp, vp, u64, vp, P(CkptDiff)], i32),
             "ckpt_restore": ([vp, u32, vp], i32),
             "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
@@ -148,6 +151,13 @@ class Checkpointer:
         self.chunk_bytes = chunk_bytes
         self.mode = mode
         self._ckpt_fn = lib().ckpt_checkpoint   # bound once: the per-call path is marshalling only
+
+    def set_variant(self, flags: int, switch_permille: int = 1000) -> None:
+        """CKPT_VARIANT_FULL_FIRST / CKPT_VARIANT_FULL_SWITCH (Tree mode, before the first
+        checkpoint; include/ckpt.h)."""
+        rc = lib().ckpt_set_variant(self._h, flags, switch_permille)
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_set_variant")
 
     # ------------------------------------------------------------------ core calls
     def checkpoint(self, buf, nbytes: int | None = None, stream=None, raw: bool = False):

@@ -55,6 +55,8 @@ struct ckpt_ctx {
   bool poisoned = false;
   uint32_t C = 0;
   int mode = kModeTree;          // CKPT_MODE_*
+  uint32_t variant = 0;          // CKPT_VARIANT_* (Tree mode; R22, R23)
+  uint32_t switch_permille = 1000;
   // geometry (fixed after checkpoint 0, R17)
   bool geo_set = false;
   uint64_t B = 0, n = 0, m = 0;
@@ -428,6 +430,15 @@ int ckpt_kernel_launches(ckpt_handle h, uint64_t* count) {
   return CKPT_OK;
 }
 
+int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_permille) {
+  if (!h) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (h->mode != kModeTree || !h->diffs.empty() || (flags & ~3u) || switch_permille > 1000) return CKPT_EINVAL;
+  h->variant = flags;
+  h->switch_permille = switch_permille;
+  return CKPT_OK;
+}
+
 int ckpt_set_profiling(ckpt_handle h, int enable) {
   if (!h) return CKPT_EINVAL;
   if (enable < 0 || enable > 2) return CKPT_EINVAL;
@@ -539,6 +550,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   }
   ip.trace = h->trace; ip.trace_n = h->trace_n;
   ip.mode = h->mode;
+  ip.sw_permille = (h->variant & CKPT_VARIANT_FULL_SWITCH) ? (int)h->switch_permille : -1;   // R23
   ip.blocksum = h->blocksum;
   ip.gsum = h->gsum;
 
@@ -621,6 +633,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.gm3 = h->gm3[s];
   }
   tp.list = h->mode == kModeList;
+  tp.sw_permille = ip.sw_permille;
   if (h->mode != kModeBasic) {   // Basic: no record, no tree
     CK(launch_tree(tp, 2, h->num_sms, st));
     if (pe) CK(cudaEventRecord(h->ev[3], st));
@@ -649,6 +662,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.nwords = h->nwords;
   cp.tcc = h->tcc;
   cp.parts = gather_parts(h->ngroups[0], h->C, h->num_sms);
+  cp.sw_permille = ip.sw_permille;
+  cp.full_first = (h->variant & CKPT_VARIANT_FULL_FIRST) && k == 0;   // R22
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
   const auto t_launched = clk::now();
@@ -690,7 +705,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
     if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), f); fclose(f); }
   }
-  if (h->mode != kModeBasic) h->live += t.n_first + t.p2_inserts;
+  if (h->mode != kModeBasic && t.full_kind != 2) h->live += t.n_first + t.p2_inserts;   // R23: no record op
   DiffRec rec;
   rec.ptr = out;
   fill_diff(h, k, t, out, &rec.info);
@@ -870,7 +885,9 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
   std::memcpy(&flags, hd + 6, 2);
   const uint32_t id = (uint32_t)h->diffs.size();
   const uint64_t B = rd64h(16), n = rd64h(24), nF = rd64h(32), nS = rd64h(40), data = rd64h(48);
-  if (rd32h(0) != 0x44504B43u || ver != 1 || flags != (uint16_t)h->mode || rd32h(8) != id || rd32h(12) != h->C)
+  const bool full_form = flags == CKPT_FLAGS_FULL && h->mode == kModeTree && h->variant != 0;   // R22 / R23
+  if (rd32h(0) != 0x44504B43u || ver != 1 || (flags != (uint16_t)h->mode && !full_form) || rd32h(8) != id ||
+      rd32h(12) != h->C)
     return CKPT_EINVAL;
   if (B == 0 || n != (B + h->C - 1) / h->C || n > (1ull << 31) || (h->geo_set && B != h->B)) return CKPT_EINVAL;
   const uint64_t raw = h->mode == kModeBasic ? 64 + 4 * ((n + 31) / 32) : 64 + 4 * nF + 12 * nS;

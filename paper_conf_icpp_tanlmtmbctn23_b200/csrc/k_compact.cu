@@ -73,7 +73,50 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   const unsigned long long bt1 = p.trace ? gtime_ns() : 0;
   const uint64_t nblk = (p.n_tiles + kTilesPerBlock - 1) / kTilesPerBlock;
   const uint64_t nwarps = (uint64_t)gridDim.x * kGW;
-  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
+  // R22 / R23: the difference is stored in full (one FIRST region, the root, and the whole
+  // buffer); the dirty-tile work below is skipped
+  const bool sw = switched_full(p.tot, p.sw_permille, g);
+  const bool full = sw || p.full_first;
+  const uint32_t count = full ? 0u : *(volatile uint32_t*)&p.tot->wl_count[0];
+  if (full) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      Totals* t = p.tot;
+      t->nF = 1; t->nS = 0; t->data_bytes = g.B; t->meta_bytes = 80;
+      if (sw) {   // every changed chunk is stored; no record operation ran
+        t->n_first = t->n_nonfixed; t->n_spatial = 0; t->n_temporal = 0; t->p2_inserts = 0;
+      }
+      t->full_kind = sw ? 2 : 1;
+      uint8_t* o = p.out;
+      *reinterpret_cast<uint32_t*>(o + 0) = 0x44504B43u;   // 'CKPD'
+      *reinterpret_cast<uint16_t*>(o + 4) = 1;
+      *reinterpret_cast<uint16_t*>(o + 6) = 3;             // flags: stored in full
+      *reinterpret_cast<uint32_t*>(o + 8) = g.k;
+      *reinterpret_cast<uint32_t*>(o + 12) = g.C;
+      *reinterpret_cast<unsigned long long*>(o + 16) = g.B;
+      *reinterpret_cast<unsigned long long*>(o + 24) = g.n;
+      *reinterpret_cast<unsigned long long*>(o + 32) = 1;
+      *reinterpret_cast<unsigned long long*>(o + 40) = 0;
+      *reinterpret_cast<unsigned long long*>(o + 48) = g.B;
+      *reinterpret_cast<unsigned long long*>(o + 56) = 0;  // hash seed, reserved
+      *reinterpret_cast<uint4*>(o + 64) = make_uint4(0, 0, 0, 0);   // root entry (node 0) + pad
+      *p.tot_host = *t;
+    }
+    // the whole buffer, 16-byte units, four loads in flight per thread before the stores
+    const uint4* src = reinterpret_cast<const uint4*>(p.buf);
+    uint4* dst = reinterpret_cast<uint4*>(p.out + 80);
+    const uint64_t nu = g.B / 16, nth = (uint64_t)gridDim.x * kCT;
+    for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < nu; i += 4 * nth) {
+      uint4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (i + u * nth < nu) v[u] = __ldcs(src + i + u * nth);
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (i + u * nth < nu) dst[i + u * nth] = v[u];
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0)
+      for (uint64_t b = nu * 16; b < g.B; ++b) p.out[80 + b] = p.buf[b];
+  }
   // worklist entry w -> block w mod grid, warp w / grid: with few dirty tiles (large chunks)
   // every SM still gets work
   uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x;
@@ -96,7 +139,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   // Basic: the changed-chunk bitmap replaces the entry lists (nF_tot = changed chunks)
   const unsigned long long raw = basic ? 64 + 4ull * p.nwords : 64 + 4 * nF_tot + 12 * nS_tot;
   const unsigned long long meta = (raw + 15) & ~15ull;
-  if (blockIdx.x == 0 && wid == 0 && lane == 0) {
+  if (blockIdx.x == 0 && wid == 0 && lane == 0 && !full) {
     // totals and the 64-byte header (R13)
     p.tot->nF = nF_tot; p.tot->nS = nS_tot; p.tot->data_bytes = data_tot; p.tot->meta_bytes = meta;
     if (basic) p.tot->n_first = nF_tot;   // every changed chunk is stored (no record)
@@ -292,7 +335,8 @@ cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st)
   // and blocks beyond one wave would only arrive late to find no work)
   const int bps = g_gather_blocks_per_sm > 0 ? g_gather_blocks_per_sm : 2;
   uint64_t grid = p.n_tiles * p.parts;   // worklist entries are spread over the blocks first
-  if (grid > (uint64_t)num_sms * bps) grid = (uint64_t)num_sms * bps;
+  // a difference that may be stored in full (R22 / R23) copies the whole buffer: full wave
+  if (grid > (uint64_t)num_sms * bps || p.full_first || p.sw_permille >= 0) grid = (uint64_t)num_sms * bps;
   return launch_pdl(gather_kernel, (unsigned)grid, kCT, kGW * sizeof(GatherWarp), st, p);
 }
 

@@ -146,6 +146,7 @@ __device__ __forceinline__ void mark_tree_dirty(const InsertParams& p, uint32_t 
 // the rounds of a dense tile run on different warps.
 __device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile, uint32_t ncand_tile) {
   const uint32_t rounds = (ncand_tile + 31) / 32;
+  if (p.sw_permille >= 0) atomicAdd(&p.tot->n_nonfixed, (unsigned long long)ncand_tile);   // R23
   const uint32_t i = atomicAdd(&p.tot->defer_count, rounds);
   for (uint32_t r = 0; r < rounds; ++r) p.defer[i + r] = (tile << 3) | r;
 }
@@ -471,7 +472,8 @@ __global__ void __launch_bounds__(256, CKPT_K1B_BPS) insert_kernel(InsertParams 
   }
   unsigned long long tk0 = 0;
   if (p.trace) asm volatile("mov.u64 %0, %globaltimer;" : "=l"(tk0));
-  const uint32_t count = *(volatile uint32_t*)&p.tot->defer_count;
+  // a switched checkpoint (R23) has no record operation
+  const uint32_t count = switched_full(p.tot, p.sw_permille, p.g) ? 0u : *(volatile uint32_t*)&p.tot->defer_count;
   const uint32_t nwarps = (gridDim.x - 1) * (blockDim.x >> 5);
   unsigned long long ncand = 0;
   for (uint32_t w = (blockIdx.x - 1) * (blockDim.x >> 5) + wid; w < count; w += nwarps) {

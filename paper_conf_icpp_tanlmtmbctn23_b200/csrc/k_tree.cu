@@ -893,7 +893,8 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   };
 
   // dirty stage-0 tiles (K1b's list); climb on the last DIRTY child of each group
-  const uint32_t count = *(volatile uint32_t*)&p.tot->wl_count[0];
+  // a switched checkpoint (R23) has no tree work
+  const uint32_t count = switched_full(p.tot, p.sw_permille, p.g) ? 0u : *(volatile uint32_t*)&p.tot->wl_count[0];
   const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
   // worklist entry w -> block w mod grid, warp w / grid: dirty tiles spread over all SMs
   for (uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x; w < count; w += nwarps) {

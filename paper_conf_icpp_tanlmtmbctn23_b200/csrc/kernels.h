@@ -32,7 +32,10 @@ constexpr int kLeafStages3d = 3;      // K1 TMA stages of 32 KB (+ 4 KB digests)
 struct Totals {                      // per-checkpoint device counters (zeroed each call)
   unsigned long long nF, nS, data_bytes, meta_bytes;
   unsigned long long n_first, n_spatial, n_temporal, p2_inserts;
-  unsigned long long collisions, n_cand, pad0, pad1;
+  unsigned long long collisions, n_cand;
+  unsigned long long full_kind;      // 0, or the difference is stored in full: 1 = full first
+                                     // checkpoint, 2 = switched (gather kernel, R22 / R23)
+  unsigned long long n_nonfixed;     // non-FIXED leaves (K1/K1t, counted only for the switch)
   uint32_t wl_count[kMaxStages];
   uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
   uint32_t gather_next;              // work-stealing cursor of the gather kernel
@@ -66,6 +69,7 @@ struct InsertParams {
   int mode;                      // CKPT_MODE_*: Basic accumulates the gather's prefix inputs in K1
   unsigned long long* blocksum;  // Basic: per 1024 tree tiles (#changed, 0, changed bytes)
   unsigned long long* gsum;      // Basic: per 32 tree tiles, the same
+  int sw_permille;               // full-change switch threshold (R23), -1 = off
 };
 
 struct LeafParams {
@@ -120,6 +124,7 @@ struct TreeParams {
   Totals* tot;
   int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
   int list;                    // CKPT_MODE_LIST: no compaction, every FIRST/SHIFT leaf is an entry
+  int sw_permille;             // full-change switch threshold (R23), -1 = off
   ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
   uint32_t* trace_n;
   StageParams st[kMaxStages];
@@ -148,7 +153,18 @@ struct CompactParams {
   uint64_t nwords;               // Basic: its u32 words
   const uint32_t* tcc;           // Basic: changed chunks per tree tile (K1)
   uint32_t parts;                // warps per dirty tile (gather_parts)
+  int sw_permille;               // full-change switch threshold (R23), -1 = off
+  int full_first;                // checkpoint 0 of a full-first lineage (R22): stored in full
 };
+
+// R23: checkpoint k >= 1 is stored in full, with no record operation, when at least
+// sw_permille / 1000 of its leaves are not FIXED. K1/K1t count them; every later kernel of
+// the call reads the final count after its pdl_wait() and takes the same decision.
+__device__ __forceinline__ bool switched_full(const Totals* tot, int sw_permille, const Geo& g) {
+  if (sw_permille < 0 || g.k == 0) return false;
+  const unsigned long long c = *reinterpret_cast<const volatile unsigned long long*>(&tot->n_nonfixed);
+  return 1000ull * c >= (unsigned long long)sw_permille * g.n;
+}
 
 // Per stage-0 tile, written by phase 2: the resolved leaf masks for phase 3 (F0 S0 X0 F1 S1
 // leaf1, bit-reversed, 32 words each) and the tile's FIRST chunks in chunk order (32

@@ -23,10 +23,14 @@ STAT_KEYS = ["n_first_regions", "n_shift_regions", "n_first", "n_fixed", "n_spat
              "list_entries", "meta_bytes", "data_bytes", "bytes", "phase2_inserts"]
 
 
-def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check_restore=True, mode=0):
+def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check_restore=True, mode=0,
+               variant=None):
     from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
     o = oracle_mod.Oracle(C, mode=mode)
     ck = Checkpointer(C, mode)
+    if variant is not None:   # (flags, switch_permille): Tree-method variants, NEXT #4
+        o.set_variant(*variant)
+        ck.set_variant(*variant)
     B = bufs[0].size
     devs = []
     for k, b in enumerate(bufs):
