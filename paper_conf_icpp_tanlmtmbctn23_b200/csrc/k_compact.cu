@@ -101,18 +101,20 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       *reinterpret_cast<uint4*>(o + 64) = make_uint4(0, 0, 0, 0);   // root entry (node 0) + pad
       *p.tot_host = *t;
     }
-    // the whole buffer, 16-byte units, four loads in flight per thread before the stores
+    // the whole buffer, 16-byte units, kFullUnroll loads in flight per thread before the
+    // stores (2 CTAs x 256 threads per SM: 64 KB in flight per SM covers HBM latency)
+    constexpr int kFullUnroll = 8;
     const uint4* src = reinterpret_cast<const uint4*>(p.buf);
     uint4* dst = reinterpret_cast<uint4*>(p.out + 80);
     const uint64_t nu = g.B / 16, nth = (uint64_t)gridDim.x * kCT;
-    for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < nu; i += 4 * nth) {
-      uint4 v[4];
+    for (uint64_t i = (uint64_t)blockIdx.x * kCT + threadIdx.x; i < nu; i += kFullUnroll * nth) {
+      uint4 v[kFullUnroll];
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < kFullUnroll; ++u)
         if (i + u * nth < nu) v[u] = __ldcs(src + i + u * nth);
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
-        if (i + u * nth < nu) dst[i + u * nth] = v[u];
+      for (int u = 0; u < kFullUnroll; ++u)
+        if (i + u * nth < nu) __stcs(dst + i + u * nth, v[u]);
     }
     if (blockIdx.x == 0 && threadIdx.x == 0)
       for (uint64_t b = nu * 16; b < g.B; ++b) p.out[80 + b] = p.buf[b];

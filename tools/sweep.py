@@ -31,13 +31,15 @@ sys.path.insert(0, ROOT)
 GiB = 1 << 30
 
 
-def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=False):
+def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=False, variant=None):
     import torch
     from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
     from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
     seed = W.seed_of(cfg)
     buf = torch.empty(B, dtype=torch.uint8, device="cuda")
     ck = Checkpointer(C, mode)
+    if variant is not None:
+        ck.set_variant(*variant)
     ck.set_profiling(prof)
     diffs, ts, walls, phases, d2hs = [], [], [], [], []
     hbuf = torch.empty(B + 64 + 12 * ((B + C - 1) // C) + 16, dtype=torch.uint8).pin_memory() if d2h else None
@@ -88,6 +90,9 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=F
     rec = {
         "case": name, "config": cfg, "buffer_bytes": B, "chunk_bytes": C, "checkpoints": K, "update_rate": p,
         "method": ["tree", "list", "basic"][mode],
+        "variant": None if variant is None else {"flags": variant[0], "switch_permille": variant[1]},
+        "full_diffs": sum(1 for d in diffs if d["n_first_regions"] == 1 and d["n_shift_regions"] == 0
+                          and d["data_bytes"] == B and d["meta_bytes"] == 80),
         "steady_gbs": round((K - 1) * B / (sum(t_st) / 1e3) / 1e9, 1),
         "steady_ms_median": round(statistics.median(t_st), 4),
         "steady_ms_min": round(min(t_st), 4), "steady_ms_max": round(max(t_st), 4),
@@ -130,6 +135,8 @@ def main():
     ap.add_argument("--methods", action="store_true",
                     help="Fig. 4 analogue: Tree / List / Basic over C = 32..512 on config 2 (1 GiB, K = 10), "
                          "with the paper's create + D2H throughput")
+    ap.add_argument("--variants", action="store_true",
+                    help="NEXT #4: full first checkpoint on config 2, the full-change switch on configs 2 and 4")
     a = ap.parse_args()
     import torch
     from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
@@ -148,17 +155,24 @@ def main():
         cases.append(("cfg4_dup_heavy", 4, GiB // s, 128, 50, 0.0, "dup"))
     if 5 in only:
         cases.append(("cfg5_16GiB_1gpu", 5, 16 * GiB // s, 128, 10, 0.01, None))
-    cases = [c + (0, False) for c in cases]
+    cases = [c + (0, False, None) for c in cases]
     if a.methods:
         cases = []
         for C in (32, 64, 128, 256, 512):
             for m, nm in ((0, "tree"), (1, "list"), (2, "basic")):
-                cases.append((f"methods_{nm}_C{C}", 2, GiB // s, C, 10, 0.01, None, m, True))
+                cases.append((f"methods_{nm}_C{C}", 2, GiB // s, C, 10, 0.01, None, m, True, None))
+    if a.variants:
+        cases = [
+            ("var_full_first_cfg2_p0.01", 2, GiB // s, 128, 20, 0.01, None, 0, False, (1, 1000)),
+            ("var_switch30_cfg2_p0.05", 2, GiB // s, 128, 20, 0.05, None, 0, False, (2, 30)),
+            ("var_none_cfg4_dup_heavy", 4, GiB // s, 128, 20, 0.0, "dup", 0, False, None),
+            ("var_switch850_cfg4_dup_heavy", 4, GiB // s, 128, 20, 0.0, "dup", 0, False, (2, 850)),
+        ]
     recs = []
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
-    for name, cfg, B, C, K, p, hg, mode, d2h in cases:
+    for name, cfg, B, C, K, p, hg, mode, d2h, var in cases:
         gen = W.DupHeavy(B, C, W.seed_of(cfg)) if hg == "dup" else None
-        r = run_case(name, cfg, B, C, a.k or K, p, stream, gen, a.prof, mode, d2h)
+        r = run_case(name, cfg, B, C, a.k or K, p, stream, gen, a.prof, mode, d2h, var)
         r["device"] = torch.cuda.get_device_name(0)
         print(json.dumps(r), flush=True)
         recs.append(r)
