@@ -164,6 +164,16 @@ CKPT_API int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff);
  * Synchronous. Errors: CKPT_ERANGE, CKPT_EINVAL (capacity < diff bytes), CKPT_ECUDA. */
 CKPT_API int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity);
 
+/* ckpt_diff_to_host without waiting (the single D2H of P:81, overlapped
+ * with the next de-duplication): enqueues the one device-to-host copy of diff `id` on
+ * `stream` (cudaStream_t as void*) and returns. Diffs are immutable and never move, so the
+ * copy may run while later ckpt_checkpoint calls de-duplicate on another stream; the host
+ * data is valid once `stream` has completed the copy (the caller synchronises it).
+ *   host_ptr  caller-owned PINNED host memory of >= capacity bytes (pageable memory would make
+ *             the copy synchronous), borrowed until the copy completes.
+ * Errors: CKPT_ERANGE, CKPT_EINVAL (capacity < diff bytes), CKPT_ECUDA, CKPT_ESTATE. */
+CKPT_API int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity, void* stream);
+
 /* End-to-end convenience path over HOST memory (P:196's throughput definition: create
  * the incremental checkpoint and copy it to host memory): copies `bytes` from host_ptr
  * into a handle-owned device staging buffer, runs ckpt_checkpoint on `stream`, then

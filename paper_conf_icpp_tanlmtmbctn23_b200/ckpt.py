@@ -23,7 +23,7 @@ CKPT_VARIANT_FULL_FIRST, CKPT_VARIANT_FULL_SWITCH = 1, 2      # Tree variants (P
 CKPT_FLAGS_FULL = 3                                           # header flags of a full difference
 
 ABI_FUNCTIONS = [
-    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host",
+    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host", "ckpt_diff_to_host_async",
     "ckpt_checkpoint_host", "ckpt_import", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
     "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
     "ckpt_strerror",
@@ -84,6 +84,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_restore": ([vp, u32, vp], i32),
             "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
             "ckpt_diff_to_host": ([vp, u32, vp, u64], i32),
+            "ckpt_diff_to_host_async": ([vp, u32, vp, u64, vp], i32),
             "ckpt_checkpoint_host": ([vp, vp, u64, vp, vp, u64, P(CkptDiff)], i32),
             "ckpt_num_checkpoints": ([vp, P(u32)], i32),
             "ckpt_import": ([vp, vp, u64, vp], i32),
@@ -215,6 +216,14 @@ class Checkpointer:
         if rc != CKPT_OK:
             raise CkptError(rc, "ckpt_diff_to_host")
         return None
+
+    def diff_to_host_async(self, cid: int, out, stream, nbytes: int | None = None) -> None:
+        """Enqueue the one D2H of diff `cid` into pinned host memory `out` on `stream` and
+        return (NEXT #1: overlap with the next checkpoint); sync `stream` before reading."""
+        cap = _nbytes(out) if nbytes is None else nbytes
+        rc = lib().ckpt_diff_to_host_async(self._h, cid, _ptr(out), cap, _stream_handle(stream))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_diff_to_host_async")
 
     @property
     def num_checkpoints(self) -> int:

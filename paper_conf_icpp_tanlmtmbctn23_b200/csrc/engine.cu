@@ -739,6 +739,16 @@ int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capac
   return CKPT_OK;
 }
 
+int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity, void* stream) {
+  if (!h || !host_ptr) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  if (id >= h->diffs.size()) return CKPT_ERANGE;
+  const DiffRec& d = h->diffs[id];
+  if (capacity < d.info.bytes) return CKPT_EINVAL;
+  CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, static_cast<cudaStream_t>(stream)));
+  return CKPT_OK;
+}
+
 int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, void* stream, void* host_diff,
                          uint64_t host_diff_cap, ckpt_diff* diff) {
   if (!h || !host_ptr || !diff || bytes == 0) return CKPT_EINVAL;

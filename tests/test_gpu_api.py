@@ -161,3 +161,33 @@ def test_kernel_launch_counter():
     ck.restore(1, out)
     assert ck.kernel_launches > b and torch.equal(out, buf)
     ck.close()
+
+
+def test_diff_to_host_async_overlaps_next_checkpoint(oracle_mod):
+    """NEXT #1: the one D2H of diff k (ckpt_diff_to_host_async on a side stream) may run
+    while checkpoint k+1 de-duplicates; every copy equals the oracle's diff."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer, CkptError
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    C = 128
+    bufs = list(W.lineage(2, (1 << 22) + 100, C, 6, p=0.05))
+    B = bufs[0].size
+    o = oracle_mod.Oracle(C)
+    ck = Checkpointer(C)
+    side = torch.cuda.Stream()
+    main = torch.cuda.Stream()
+    devs = [torch.from_numpy(np.ascontiguousarray(b)).cuda() for b in bufs]
+    hosts = []
+    for k, b in enumerate(bufs):
+        d = ck.checkpoint(devs[k], nbytes=B, stream=main)
+        o.checkpoint(b)
+        h = torch.empty(d["bytes"], dtype=torch.uint8).pin_memory()
+        ck.diff_to_host_async(k, h, side)
+        hosts.append(h)
+    side.synchronize()
+    for k in range(len(bufs)):
+        assert bytes(hosts[k].numpy()) == o.diff(k), k
+    with pytest.raises(CkptError):
+        ck.diff_to_host_async(0, torch.empty(8, dtype=torch.uint8).pin_memory(), side)   # too small
+    with pytest.raises(CkptError):
+        ck.diff_to_host_async(len(bufs), hosts[0], side)                                 # no such diff
+    ck.close()
