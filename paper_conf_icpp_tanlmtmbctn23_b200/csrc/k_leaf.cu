@@ -73,7 +73,10 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
       const unsigned m2 = __match_any_sync(active, d.hi);
       const unsigned grp = m1 & m2;
       const int leader = __ffs(grp) - 1;
-      uint32_t minnode = node;   // minimum node id of the group (every active lane shuffles)
+      // minimum node id of the group (every active lane shuffles). Measured on config 4: a
+      // vote that skips this loop for rounds of distinct digests made K1b 14 % slower, and
+      // __reduce_min_sync over the (non-uniform) group masks 30 % slower.
+      uint32_t minnode = node;
       for (unsigned a = active; a; a &= a - 1) {
         const int sl = __ffs(a) - 1;
         const uint32_t vv = __shfl_sync(active, node, sl);

@@ -37,6 +37,9 @@ namespace ckpt {
 namespace {
 
 constexpr int kWarps = kTreeThreads / 32;
+#ifndef CKPT_TREE_CURSOR
+#define CKPT_TREE_CURSOR 1   // worklist entries beyond the first per warp from a cursor (0: static stride)
+#endif
 constexpr int kDigCap = 256;   // on-chip digests per warp (4 KB); dense groups spill to global
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -896,11 +899,20 @@ __global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_cons
   // a switched checkpoint (R23) has no tree work
   const uint32_t count = switched_full(p.tot, p.sw_permille, p.g) ? 0u : *(volatile uint32_t*)&p.tot->wl_count[0];
   const uint64_t nwarps = (uint64_t)gridDim.x * kWarps;
-  // worklist entry w -> block w mod grid, warp w / grid: dirty tiles spread over all SMs
-  for (uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x; w < count; w += nwarps) {
+  // First entry per warp: w -> block w mod grid, warp w / grid (dirty tiles spread over all
+  // SMs; with at most one tile per warp, as in the sparse steady state, no atomic at all).
+  // Later entries come from a cursor, fetched one tile ahead so its latency overlaps the
+  // current tile: dense checkpoints give tiles (and climbs) of very different cost, and a
+  // static stride left warps idle at the end of the kernel.
+  uint32_t* cursor = &p.tot->tree_next[PHASE - 2];
+  uint64_t w = (uint64_t)wid * gridDim.x + blockIdx.x;
+  while (w < count) {
+    uint32_t nx = 0;
+    if (CKPT_TREE_CURSOR && lane == 0 && nwarps < count) nx = atomicAdd(cursor, 1u);
     const uint64_t T = __ldcg(p.wl0 + w);
     Ctx c = run_tile(T);
     climb(c);
+    w = !CKPT_TREE_CURSOR ? w + nwarps : nwarps < count ? nwarps + __shfl_sync(0xffffffffu, nx, 0) : count;
   }
   const unsigned long long ta = p.trace ? gtime_ns() : 0;
   if (PHASE == 2) {
