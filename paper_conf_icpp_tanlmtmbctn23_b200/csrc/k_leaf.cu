@@ -28,6 +28,9 @@ __device__ __forceinline__ bool leaf_is_candidate(const Geo& g, const Digest& d,
 
 // ------------------------------------------------------------------ record insert
 constexpr uint32_t kDenseTile = 64;
+#ifndef CKPT_K1B_DEDUP_ALL
+#define CKPT_K1B_DEDUP_ALL 0   // 1: warp-level key de-duplication at every checkpoint (A/B)
+#endif
 #ifndef CKPT_K1B_BPS
 #define CKPT_K1B_BPS 4   // K1b launch bound: 4 resident blocks per SM (<= 64 registers)
 #endif   // candidates per 256-chunk tile above which inserts read first
@@ -69,15 +72,19 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
       const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(p.prev) + c);
       const Digest d{v.x, v.y};
       const uint32_t node = node_of_chunk(p.g, c);
-      const unsigned m1 = __match_any_sync(active, d.lo);
-      const unsigned m2 = __match_any_sync(active, d.hi);
-      const unsigned grp = m1 & m2;
+      // Warp-level de-duplication of equal digests (one record operation per distinct key)
+      // at checkpoint 0, where hot keys (e.g. all-zero chunks) would otherwise serialise
+      // thousands of atomics on one slot. Later checkpoints skip it: every lane inserts its
+      // own candidate; equal keys then meet in the table, where the R6 atomicMin gives the
+      // same result, and older keys cost one read.
+      const bool dedup = CKPT_K1B_DEDUP_ALL || p.g.k == 0;
+      const unsigned grp = dedup ? (__match_any_sync(active, d.lo) & __match_any_sync(active, d.hi)) : (1u << lane);
       const int leader = __ffs(grp) - 1;
       // minimum node id of the group (every active lane shuffles). Measured on config 4: a
       // vote that skips this loop for rounds of distinct digests made K1b 14 % slower, and
       // __reduce_min_sync over the (non-uniform) group masks 30 % slower.
       uint32_t minnode = node;
-      for (unsigned a = active; a; a &= a - 1) {
+      for (unsigned a = dedup ? active : 0u; a; a &= a - 1) {
         const int sl = __ffs(a) - 1;
         const uint32_t vv = __shfl_sync(active, node, sl);
         if ((grp >> sl) & 1u) minnode = vv < minnode ? vv : minnode;
