@@ -37,6 +37,9 @@ namespace ckpt {
 namespace {
 
 constexpr int kWarps = kTreeThreads / 32;
+#ifndef CKPT_TREE_BPS
+#define CKPT_TREE_BPS 2   // tree-kernel launch bound: resident CTAs per SM (register budget)
+#endif
 #ifndef CKPT_TREE_CURSOR
 #define CKPT_TREE_CURSOR 1   // worklist entries beyond the first per warp from a cursor (0: static stride)
 #endif
@@ -797,7 +800,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
 
 // ================================================================= kernel
 template <int PHASE>
-__global__ void __launch_bounds__(kTreeThreads, 2) tree_kernel(const __grid_constant__ TreeParams p) {
+__global__ void __launch_bounds__(kTreeThreads, CKPT_TREE_BPS) tree_kernel(const __grid_constant__ TreeParams p) {
   extern __shared__ __align__(16) uint8_t tree_smem[];
   WarpSmem* sm = reinterpret_cast<WarpSmem*>(tree_smem);
   __shared__ unsigned long long s_cnt[4];
