@@ -14,3 +14,4 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:"lea
 python tools/ncu_summarize.py gpurun_out/prof.ncu-rep gpurun_out/ncu_summary.json > gpurun_out/ncu_full.txt 2>&1
 cat gpurun_out/ncu_full.txt
 if [ "$SWEEP" = "1" ]; then timeout 1500 python tools/sweep.py > gpurun_out/sweep.log 2>&1; echo "sweep rc=$?"; fi
+timeout 900 python tools/oracle_time.py --out gpurun_out/oracle_time.json > gpurun_out/oracle_time.log 2>&1; echo "oracle_time rc=$?"
