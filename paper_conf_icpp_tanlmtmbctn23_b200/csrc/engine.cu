@@ -40,6 +40,9 @@ struct DiffRec {
   bool planned = false;
 };
 
+#ifndef CKPT_RESTORE_PAINT
+#define CKPT_RESTORE_PAINT 0   // 1: restore by painting each diff's byte streams newest first (A/B)
+#endif
 #ifndef CKPT_TABLE_GROW_LOAD
 #define CKPT_TABLE_GROW_LOAD 0.6
 #endif
@@ -100,7 +103,8 @@ struct ckpt_ctx {
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
   // restore state (lazy): painter mark per chunk, plan scratch, the chain's plans on device
-  uint32_t* painted = nullptr;
+  uint32_t* painted = nullptr;          // restore marks (paint form, CKPT_RESTORE_PAINT)
+  unsigned long long* owner = nullptr;   // restore: source address of every chunk (chunk-major form)
   unsigned long long* rs_len = nullptr;
   uint64_t rs_len_cap = 0;
   void* rs_scan = nullptr;
@@ -405,7 +409,7 @@ int ckpt_destroy(ckpt_handle h) {
   for (auto& d : h->diffs)
     for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg})
       if (q) cudaFree(q);
-  for (void* q : {(void*)h->painted, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
+  for (void* q : {(void*)h->painted, (void*)h->owner, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
     if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
   if (h->tot_host) cudaFreeHost(h->tot_host);
@@ -982,12 +986,17 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
     if (rc == CKPT_ECUDA) h->poisoned = true;
     return rc;
   }
+#if CKPT_RESTORE_PAINT
   if (!h->painted) {
     if (cudaMalloc(&h->painted, h->n * sizeof(uint32_t)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
   }
-  // newest diff first; a chunk is written by the newest diff whose regions cover it
-  // (diff 0 covers every chunk, so the target needs no clearing)
   CK(cudaMemsetAsync(h->painted, 0, h->n * sizeof(uint32_t), st));
+#else
+  if (!h->owner) {
+    if (cudaMalloc(&h->owner, h->n * sizeof(unsigned long long)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
+  }
+  CK(cudaMemsetAsync(h->owner, 0, h->n * sizeof(unsigned long long), st));
+#endif
   uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
   for (int64_t c = id; c >= 0; --c) {
     const DiffRec& d = h->diffs[c];
@@ -999,8 +1008,15 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
     r.data_bytes = d.info.data_bytes;
     r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
     r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
+#if CKPT_RESTORE_PAINT
     CK(restore_paint(g, r, outp, h->painted, (uint32_t)c + 1u, h->num_sms, st));
+#else
+    CK(restore_claim(g, r, h->owner, h->num_sms, st));
+#endif
   }
+#if !CKPT_RESTORE_PAINT
+  CK(restore_copy(g, h->owner, outp, h->num_sms, st));
+#endif
   CK(cudaStreamSynchronize(st));
   return CKPT_OK;
 }

@@ -86,8 +86,14 @@ __global__ void prepare_first_kernel(Geo g, RestoreDiff d, unsigned long long* l
   len[i] = range_bytes(g, lo, hi);
 }
 
-constexpr uint32_t kPaintSeg = 2048;                 // bytes per warp segment
-constexpr uint32_t kPaintUnits = kPaintSeg / 16 / 32;   // 16-B units per lane per segment (4)
+#ifndef CKPT_PAINT_SEG
+#define CKPT_PAINT_SEG 2048
+#endif
+#ifndef CKPT_PAINT_BPS
+#define CKPT_PAINT_BPS 4
+#endif
+constexpr uint32_t kPaintSeg = CKPT_PAINT_SEG;       // bytes per warp segment
+constexpr uint32_t kPaintUnits = kPaintSeg / 16 / 32;   // 16-B units per lane per segment (4 at 2 KB)
 constexpr uint32_t kPaintSlots = kPaintSeg / 32 + 3;    // regions per segment (C >= 32), tail, next start
 constexpr int kPaintWarps = kRT / 32;
 
@@ -101,7 +107,7 @@ __device__ __forceinline__ uint64_t region_at(const unsigned long long* off, uin
   return lo;
 }
 
-__global__ void __launch_bounds__(kRT, 4) paint_kernel(Geo g, RestoreDiff d, uint8_t* out, uint32_t* painted,
+__global__ void __launch_bounds__(kRT, CKPT_PAINT_BPS) paint_kernel(Geo g, RestoreDiff d, uint8_t* out, uint32_t* painted,
                                                    uint32_t mark) {
   __shared__ unsigned long long s_off[kPaintWarps][kPaintSlots + 1];
   pdl_launch_dependents();
@@ -195,6 +201,89 @@ __global__ void __launch_bounds__(kRT, 4) paint_kernel(Geo g, RestoreDiff d, uin
       if ((setmark >> j) & 1u) painted[chk[j]] = mark;
     }
     __syncwarp();
+  }
+}
+
+// ---- chunk-major restore: claim, then one copy pass
+// claim_kernel (one launch per diff, newest first): one thread per chunk of the diff's
+// FIRST stream and SHIFT stream; the chunk's first claimer (the newest diff covering it)
+// records the device address of its bytes in owner[chunk]. Regions of one diff are
+// disjoint, so a diff never races with itself; diffs run in stream order.
+__global__ void __launch_bounds__(kRT) claim_kernel(Geo g, RestoreDiff d, unsigned long long* owner) {
+  pdl_launch_dependents();
+  pdl_wait();   // the newer diffs' claims are complete
+  const unsigned long long C = g.C;
+  const uint64_t nxF = (d.data_bytes + C - 1) / C, nxS = (d.shift_bytes + C - 1) / C;
+  const uint8_t* data = d.base + d.meta_bytes;
+  for (uint64_t t = (uint64_t)blockIdx.x * kRT + threadIdx.x; t < nxF + nxS; t += (uint64_t)gridDim.x * kRT) {
+    const bool first = t < nxF;
+    const unsigned long long o = (first ? t : t - nxF) * C;   // stream offset (every region but the
+                                                              // stream's last is whole chunks)
+    const unsigned long long* off = first ? d.Foff : d.Soff;
+    const unsigned long long* seg = first ? d.Fseg : d.Sseg;
+    const uint64_t nr = first ? d.nF : d.nS;
+    const uint64_t sg = o / kPaintSeg;
+    // last region r with off[r] <= o, between the regions holding this segment's first byte
+    // and the next segment's
+    uint64_t lo = __ldg(seg + sg), hi = __ldg(seg + sg + 1) + 1;
+    if (hi > nr) hi = nr;
+    while (hi - lo > 1) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (__ldg(off + mid) <= o) lo = mid; else hi = mid;
+    }
+    const unsigned long long rel = o - __ldg(off + lo);
+    const uint64_t chunk = (first ? __ldg(d.Flo + lo) : __ldg(d.Slo + lo)) + rel / C;
+    if (__ldcg(owner + chunk) == 0)
+      owner[chunk] = first ? (unsigned long long)(data + o) : __ldg(d.Ssrc + lo) + rel;
+  }
+}
+
+// copy_kernel: the output as a stream of 16-byte units (C is a multiple of 16, so a unit
+// never straddles chunks); each unit reads its chunk's owner address, then its 16 bytes.
+// kCopyUnroll units per thread are in flight before any store. A chunk no diff claimed
+// (impossible for a well-formed lineage: diff 0 covers every chunk) reads as zeros, the
+// replay's starting buffer.
+constexpr int kCopyUnroll = 4;
+__global__ void __launch_bounds__(kRT) copy_kernel(Geo g, const unsigned long long* owner, uint8_t* out) {
+  pdl_launch_dependents();
+  pdl_wait();
+  const uint64_t U = g.C / 16;
+  const uint64_t nu = (g.B + 15) / 16;
+  const uint64_t nth = (uint64_t)gridDim.x * kRT;
+  for (uint64_t u0 = (uint64_t)blockIdx.x * kRT + threadIdx.x; u0 < nu; u0 += kCopyUnroll * nth) {
+    unsigned long long src[kCopyUnroll];
+#pragma unroll
+    for (int j = 0; j < kCopyUnroll; ++j) {
+      const uint64_t u = u0 + j * nth;
+      src[j] = u < nu ? __ldg(owner + u / U) : 0ull;
+      if (src[j]) src[j] += (u % U) * 16;
+    }
+    uint4 v[kCopyUnroll];
+#pragma unroll
+    for (int j = 0; j < kCopyUnroll; ++j) {
+      const uint64_t u = u0 + j * nth;
+      v[j] = make_uint4(0, 0, 0, 0);
+      if (u >= nu || !src[j]) continue;
+      if (16 * u + 16 <= g.B) {
+        v[j] = __ldcs(reinterpret_cast<const uint4*>(src[j]));
+      } else {   // the buffer's last, partial unit: only its bytes (the source may end there)
+        const uint8_t* sp = reinterpret_cast<const uint8_t*>(src[j]);
+        uint32_t w[4] = {0, 0, 0, 0};
+        for (uint32_t q = 0; q < (uint32_t)(g.B - 16 * u); ++q) w[q >> 2] |= (uint32_t)sp[q] << (8 * (q & 3));
+        v[j] = make_uint4(w[0], w[1], w[2], w[3]);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < kCopyUnroll; ++j) {
+      const uint64_t u = u0 + j * nth;
+      if (u >= nu) continue;
+      if (16 * u + 16 <= g.B) {
+        __stcs(reinterpret_cast<uint4*>(out + 16 * u), v[j]);
+      } else {
+        const uint32_t w[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
+        for (uint32_t q = 0; q < (uint32_t)(g.B - 16 * u); ++q) out[16 * u + q] = (uint8_t)(w[q >> 2] >> (8 * (q & 3)));
+      }
+    }
   }
 }
 
@@ -348,10 +437,28 @@ cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st) {
 
 uint64_t restore_segments(uint64_t bytes) { return (bytes + kPaintSeg - 1) / kPaintSeg; }
 
+cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st) {
+  if (d.nF == 0 && d.nS == 0) return cudaSuccess;
+  const uint64_t nx = (d.data_bytes + g.C - 1) / g.C + (d.shift_bytes + g.C - 1) / g.C;
+  uint64_t grid = (nx + kRT - 1) / kRT;
+  const uint64_t cap = (uint64_t)num_sms * 8;
+  if (grid > cap) grid = cap;
+  if (grid == 0) grid = 1;
+  return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, g, d, owner);
+}
+
+cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st) {
+  const uint64_t nu = (g.B + 15) / 16;
+  uint64_t grid = (nu + kRT * kCopyUnroll - 1) / (kRT * kCopyUnroll);
+  const uint64_t cap = (uint64_t)num_sms * 8;
+  if (grid > cap) grid = cap;
+  return launch_pdl(copy_kernel, (unsigned)grid, kRT, 0, st, g, owner, out);
+}
+
 cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
                           int num_sms, cudaStream_t st) {
   if (d.nF == 0 && d.nS == 0) return cudaSuccess;
-  return launch_pdl(paint_kernel, (unsigned)(num_sms * 4), kRT, 0, st, g, d, out, painted, mark);
+  return launch_pdl(paint_kernel, (unsigned)(num_sms * CKPT_PAINT_BPS), kRT, 0, st, g, d, out, painted, mark);
 }
 
 
@@ -364,6 +471,8 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_add_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_first_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, paint_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, claim_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_shift_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, write_total_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, segmap_kernel);

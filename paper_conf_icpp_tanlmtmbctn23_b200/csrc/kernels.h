@@ -237,6 +237,8 @@ cudaError_t restore_prepare_basic(const Geo& g, RestoreDiff& d, uint64_t nwords,
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st);
 cudaError_t device_compare(const void* a, const void* b, uint64_t bytes, int* diff, int num_sms, cudaStream_t st);
 uint64_t restore_segments(uint64_t bytes);
+cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st);
+cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st);
 cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
                           int num_sms, cudaStream_t st);
 size_t scan_tmp_bytes_for(uint64_t count);
