@@ -36,13 +36,12 @@ struct DiffRec {
   unsigned long long* Ssrc = nullptr;
   unsigned long long* Fseg = nullptr;
   unsigned long long* Sseg = nullptr;
+  uint32_t* Cch = nullptr;              // claim list (chunk-major restore)
+  unsigned long long* Csrc = nullptr;
   unsigned long long shift_bytes = 0;
   bool planned = false;
 };
 
-#ifndef CKPT_RESTORE_PAINT
-#define CKPT_RESTORE_PAINT 0   // 1: restore by painting each diff's byte streams newest first (A/B)
-#endif
 #ifndef CKPT_TABLE_GROW_LOAD
 #define CKPT_TABLE_GROW_LOAD 0.6
 #endif
@@ -102,8 +101,7 @@ struct ckpt_ctx {
   std::vector<DiffRec> diffs;
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
-  // restore state (lazy): painter mark per chunk, plan scratch, the chain's plans on device
-  uint32_t* painted = nullptr;          // restore marks (paint form, CKPT_RESTORE_PAINT)
+  // restore state (lazy): chunk owners, plan scratch, the chain's plans on device
   unsigned long long* owner = nullptr;   // restore: source address of every chunk (chunk-major form)
   unsigned long long* rs_len = nullptr;
   uint64_t rs_len_cap = 0;
@@ -407,9 +405,10 @@ int ckpt_destroy(ckpt_handle h) {
   for (void* p : h->allocs) cudaFree(p);
   h->arena.release_all();
   for (auto& d : h->diffs)
-    for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg})
+    for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg,
+                    (void*)d.Cch, (void*)d.Csrc})
       if (q) cudaFree(q);
-  for (void* q : {(void*)h->painted, (void*)h->owner, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
+  for (void* q : {(void*)h->owner, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
     if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
   if (h->tot_host) cudaFreeHost(h->tot_host);
@@ -874,6 +873,14 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     rd[c].Fseg = d.Fseg;
     rd[c].Sseg = d.Sseg;
     if (restore_segmaps(rd[c], st) != cudaSuccess) return CKPT_ECUDA;
+    const uint64_t ncl = (rd[c].data_bytes + h->C - 1) / h->C + (shb[c] + h->C - 1) / h->C;
+    if (ncl && (cudaMalloc(&d.Cch, ncl * 4) != cudaSuccess || cudaMalloc(&d.Csrc, ncl * 8) != cudaSuccess)) {
+      cudaGetLastError();
+      return CKPT_ENOMEM;
+    }
+    rd[c].Cch = d.Cch;
+    rd[c].Csrc = d.Csrc;
+    if (restore_claimlist(g, rd[c], h->num_sms, st) != cudaSuccess) return CKPT_ECUDA;
   }
   if (cudaStreamSynchronize(st) != cudaSuccess) return CKPT_ECUDA;
   for (uint32_t c = 0; c <= id; ++c) h->diffs[c].planned = true;
@@ -881,10 +888,12 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
 }
 
 static void free_plan(DiffRec& d) {
-  for (unsigned long long** q : {&d.Flo, &d.Foff, &d.Slo, &d.Soff, &d.Ssrc, &d.Fseg, &d.Sseg}) {
+  for (unsigned long long** q : {&d.Flo, &d.Foff, &d.Slo, &d.Soff, &d.Ssrc, &d.Fseg, &d.Sseg, &d.Csrc}) {
     if (*q) cudaFree(*q);
     *q = nullptr;
   }
+  if (d.Cch) cudaFree(d.Cch);
+  d.Cch = nullptr;
   d.planned = false;
 }
 
@@ -986,17 +995,10 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
     if (rc == CKPT_ECUDA) h->poisoned = true;
     return rc;
   }
-#if CKPT_RESTORE_PAINT
-  if (!h->painted) {
-    if (cudaMalloc(&h->painted, h->n * sizeof(uint32_t)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
-  }
-  CK(cudaMemsetAsync(h->painted, 0, h->n * sizeof(uint32_t), st));
-#else
   if (!h->owner) {
     if (cudaMalloc(&h->owner, h->n * sizeof(unsigned long long)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
   }
   CK(cudaMemsetAsync(h->owner, 0, h->n * sizeof(unsigned long long), st));
-#endif
   uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
   for (int64_t c = id; c >= 0; --c) {
     const DiffRec& d = h->diffs[c];
@@ -1008,15 +1010,10 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
     r.data_bytes = d.info.data_bytes;
     r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
     r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
-#if CKPT_RESTORE_PAINT
-    CK(restore_paint(g, r, outp, h->painted, (uint32_t)c + 1u, h->num_sms, st));
-#else
+    r.Cch = d.Cch; r.Csrc = d.Csrc;
     CK(restore_claim(g, r, h->owner, h->num_sms, st));
-#endif
   }
-#if !CKPT_RESTORE_PAINT
   CK(restore_copy(g, h->owner, outp, h->num_sms, st));
-#endif
   CK(cudaStreamSynchronize(st));
   return CKPT_OK;
 }

@@ -8,20 +8,20 @@
 // Replaying diffs 0..id writes every chunk once per diff that touches it, and the LAST
 // such diff wins: a FIXED chunk of diff c keeps what an earlier diff wrote. So the result
 // is, per chunk, the bytes of the latest diff c <= id whose regions cover it, and every
-// chunk is covered by diff 0 (no FIXED leaf at checkpoint 0, R5). The restore therefore
-// PAINTS diffs newest first: diff c writes a chunk only if no later diff painted it
-// (painted[chunk] holds c+1 of its painter), so every output byte is written exactly once
-// and FIXED chunks cost nothing — B bytes written, B bytes read, plus one 4-byte mark per
-// chunk, instead of one full copy per diff.
+// chunk is covered by diff 0 (no FIXED leaf at checkpoint 0, R5). The restore is therefore
+// CHUNK-MAJOR: per diff, newest first, claim_kernel records in owner[chunk] the device
+// address of the chunk's bytes unless a newer diff already claimed it (8 B per covered
+// chunk); then ONE copy_kernel writes every output chunk once from its owner, coalesced on
+// the output side — B bytes written, at most B read, instead of one copy per diff.
 //
 // Per diff, a restore plan is built once and cached (diffs are immutable):
 //   FIRST: Flo[r] (first chunk of region r), Foff[r] (its offset in the data section)
 //   SHIFT: Slo[r] (first chunk), Soff[r] (exclusive scan of byte lengths, Soff[nS] = total),
 //          Ssrc[r] (device address of the source bytes: v's bytes inside the FIRST region of
 //          diff c' holding v's first chunk, binary search over c''s sorted region starts)
-// paint_kernel streams a diff's FIRST bytes then its SHIFT bytes in 2-KB segments, one
-// warp per segment; the regions of a segment are located once per segment (two binary
-// searches) and their offsets staged in shared memory.
+//   segment maps Fseg / Sseg (region holding the first byte of every 2-KB stream segment)
+//   claim list Cch / Csrc: the chunk and source address of every C-byte step of the FIRST
+//          then SHIFT stream (claimlist_kernel), so a warm claim is two coalesced loads.
 #include "kernels.h"
 #include "tma.cuh"
 
@@ -86,16 +86,7 @@ __global__ void prepare_first_kernel(Geo g, RestoreDiff d, unsigned long long* l
   len[i] = range_bytes(g, lo, hi);
 }
 
-#ifndef CKPT_PAINT_SEG
-#define CKPT_PAINT_SEG 2048
-#endif
-#ifndef CKPT_PAINT_BPS
-#define CKPT_PAINT_BPS 4
-#endif
-constexpr uint32_t kPaintSeg = CKPT_PAINT_SEG;       // bytes per warp segment
-constexpr uint32_t kPaintUnits = kPaintSeg / 16 / 32;   // 16-B units per lane per segment (4 at 2 KB)
-constexpr uint32_t kPaintSlots = kPaintSeg / 32 + 3;    // regions per segment (C >= 32), tail, next start
-constexpr int kPaintWarps = kRT / 32;
+constexpr uint32_t kSegBytes = 2048;   // segment map granularity of a diff's byte streams
 
 // first index r in [0, nr) with off[r] > x, minus one (off[0] == 0 <= x)
 __device__ __forceinline__ uint64_t region_at(const unsigned long long* off, uint64_t nr, unsigned long long x) {
@@ -107,111 +98,10 @@ __device__ __forceinline__ uint64_t region_at(const unsigned long long* off, uin
   return lo;
 }
 
-__global__ void __launch_bounds__(kRT, CKPT_PAINT_BPS) paint_kernel(Geo g, RestoreDiff d, uint8_t* out, uint32_t* painted,
-                                                   uint32_t mark) {
-  __shared__ unsigned long long s_off[kPaintWarps][kPaintSlots + 1];
-  pdl_launch_dependents();
-  pdl_wait();   // the previous (newer) diff's marks are complete
-  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  unsigned long long* so = s_off[wid];
-  const uint8_t* data = d.base + d.meta_bytes;
-  const unsigned long long totF = d.data_bytes;
-  const unsigned long long totS = d.shift_bytes;
-  const uint64_t nsegF = (totF + kPaintSeg - 1) / kPaintSeg, nsegS = (totS + kPaintSeg - 1) / kPaintSeg;
-  const uint32_t U = g.C / 16;   // units per chunk
-  const uint64_t nw = ((uint64_t)gridDim.x * kRT) >> 5;
-  for (uint64_t sg = ((uint64_t)blockIdx.x * kRT + threadIdx.x) >> 5; sg < nsegF + nsegS; sg += nw) {
-    const bool first = sg < nsegF;
-    const unsigned long long* off = first ? d.Foff : d.Soff;
-    const uint64_t nr = first ? d.nF : d.nS;
-    const unsigned long long total = first ? totF : totS;
-    const unsigned long long s0 = (first ? sg : sg - nsegF) * kPaintSeg;
-    const unsigned long long s1 = s0 + kPaintSeg < total ? s0 + kPaintSeg : total;
-    // regions of the segment: from the region holding its first byte (cached segment map)
-    // to the region holding the next segment's first byte (one extra slot at most)
-    const unsigned long long* segmap = first ? d.Fseg : d.Sseg;
-    const uint64_t sl = first ? sg : sg - nsegF;
-    const uint64_t r0 = __ldg(segmap + sl), r1 = __ldg(segmap + sl + 1);
-    const uint32_t nloc = (uint32_t)(r1 - r0 + 1);   // <= kPaintSlots (regions are >= 32 B but the last)
-    for (uint32_t i = lane; i <= nloc; i += 32) so[i] = (r0 + i < nr) ? __ldg(off + r0 + i) : total;
-    __syncwarp();
-    // units of this lane: o_j = s0 + 16 (lane + 32 j). Loads are issued in batches across
-    // the 8 units (region fields, then the painter marks, then the bytes) before any store.
-    uint32_t loc[kPaintUnits];
-    unsigned long long clo[kPaintUnits], sbase[kPaintUnits];
-#pragma unroll
-    for (uint32_t j = 0; j < kPaintUnits; ++j) {
-      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
-      uint32_t lo = 0, hi = nloc;   // last local region with so[lo] <= o
-      while (hi - lo > 1) {
-        const uint32_t mid = (lo + hi) >> 1;
-        if (so[mid] <= o) lo = mid; else hi = mid;
-      }
-      loc[j] = o < s1 ? lo : ~0u;
-    }
-#pragma unroll
-    for (uint32_t j = 0; j < kPaintUnits; ++j) {
-      if (loc[j] == ~0u) continue;
-      const uint64_t rr = r0 + loc[j];
-      clo[j] = first ? __ldg(d.Flo + rr) : __ldg(d.Slo + rr);
-      sbase[j] = first ? 0ull : __ldg(d.Ssrc + rr);
-    }
-    uint64_t chk[kPaintUnits];
-    uint32_t mk[kPaintUnits];
-#pragma unroll
-    for (uint32_t j = 0; j < kPaintUnits; ++j) {
-      if (loc[j] == ~0u) continue;
-      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
-      const uint32_t ur = (uint32_t)((o - so[loc[j]]) >> 4);
-      chk[j] = clo[j] + ur / U;
-      mk[j] = __ldcg(painted + chk[j]);
-    }
-    uint4 v[kPaintUnits];
-    uint32_t len[kPaintUnits];
-    uint32_t setmark = 0;   // bit j: unit j starts a chunk this diff paints
-#pragma unroll
-    for (uint32_t j = 0; j < kPaintUnits; ++j) {
-      len[j] = 0;
-      if (loc[j] == ~0u || mk[j] > mark) continue;   // a newer diff painted this chunk
-      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
-      const unsigned long long rel = o - so[loc[j]];
-      const unsigned long long rem = so[loc[j] + 1] - o;
-      len[j] = rem >= 16 ? 16u : (uint32_t)rem;
-      if ((rel >> 4) % U == 0) setmark |= 1u << j;
-      const uint8_t* src = first ? data + o : reinterpret_cast<const uint8_t*>(sbase[j]) + rel;
-      if (len[j] == 16) {
-        v[j] = __ldg(reinterpret_cast<const uint4*>(src));
-      } else {
-        uint32_t w[4] = {0, 0, 0, 0};
-        for (uint32_t q = 0; q < len[j]; ++q) w[q >> 2] |= (uint32_t)src[q] << (8 * (q & 3));
-        v[j] = make_uint4(w[0], w[1], w[2], w[3]);
-      }
-    }
-#pragma unroll
-    for (uint32_t j = 0; j < kPaintUnits; ++j) {
-      if (!len[j]) continue;
-      const unsigned long long o = s0 + 16ull * (lane + 32u * j);
-      uint8_t* dst = out + clo[j] * (unsigned long long)g.C + (o - so[loc[j]]);
-      if (len[j] == 16) {
-        *reinterpret_cast<uint4*>(dst) = v[j];
-      } else {
-        const uint32_t w[4] = {v[j].x, v[j].y, v[j].z, v[j].w};
-        for (uint32_t q = 0; q < len[j]; ++q) dst[q] = (uint8_t)(w[q >> 2] >> (8 * (q & 3)));
-      }
-      if ((setmark >> j) & 1u) painted[chk[j]] = mark;
-    }
-    __syncwarp();
-  }
-}
-
 // ---- chunk-major restore: claim, then one copy pass
-// claim_kernel (one launch per diff, newest first): one thread per chunk of the diff's
-// FIRST stream and SHIFT stream; the chunk's first claimer (the newest diff covering it)
-// records the device address of its bytes in owner[chunk]. Regions of one diff are
-// disjoint, so a diff never races with itself; diffs run in stream order.
-__global__ void __launch_bounds__(kRT) claim_kernel(Geo g, RestoreDiff d, unsigned long long* owner) {
-  pdl_launch_dependents();
-  pdl_wait();   // the newer diffs' claims are complete
+// claimlist_kernel (plan building, once per diff): one thread per chunk of the diff's FIRST
+// stream then SHIFT stream writes the chunk's id and the device address of its bytes.
+__global__ void __launch_bounds__(kRT) claimlist_kernel(Geo g, RestoreDiff d) {
   const unsigned long long C = g.C;
   const uint64_t nxF = (d.data_bytes + C - 1) / C, nxS = (d.shift_bytes + C - 1) / C;
   const uint8_t* data = d.base + d.meta_bytes;
@@ -222,7 +112,7 @@ __global__ void __launch_bounds__(kRT) claim_kernel(Geo g, RestoreDiff d, unsign
     const unsigned long long* off = first ? d.Foff : d.Soff;
     const unsigned long long* seg = first ? d.Fseg : d.Sseg;
     const uint64_t nr = first ? d.nF : d.nS;
-    const uint64_t sg = o / kPaintSeg;
+    const uint64_t sg = o / kSegBytes;
     // last region r with off[r] <= o, between the regions holding this segment's first byte
     // and the next segment's
     uint64_t lo = __ldg(seg + sg), hi = __ldg(seg + sg + 1) + 1;
@@ -232,9 +122,21 @@ __global__ void __launch_bounds__(kRT) claim_kernel(Geo g, RestoreDiff d, unsign
       if (__ldg(off + mid) <= o) lo = mid; else hi = mid;
     }
     const unsigned long long rel = o - __ldg(off + lo);
-    const uint64_t chunk = (first ? __ldg(d.Flo + lo) : __ldg(d.Slo + lo)) + rel / C;
-    if (__ldcg(owner + chunk) == 0)
-      owner[chunk] = first ? (unsigned long long)(data + o) : __ldg(d.Ssrc + lo) + rel;
+    d.Cch[t] = (uint32_t)((first ? __ldg(d.Flo + lo) : __ldg(d.Slo + lo)) + rel / C);
+    d.Csrc[t] = first ? (unsigned long long)(data + o) : __ldg(d.Ssrc + lo) + rel;
+  }
+}
+
+// claim_kernel (one launch per diff, newest first): the chunk's first claimer (the newest
+// diff covering it) records the address of its bytes in owner[chunk]. Regions of one diff
+// are disjoint, so a diff never races with itself; diffs run in stream order.
+__global__ void __launch_bounds__(kRT) claim_kernel(RestoreDiff d, uint64_t ncl, unsigned long long* owner) {
+  pdl_launch_dependents();
+  pdl_wait();   // the newer diffs' claims are complete
+  for (uint64_t t = (uint64_t)blockIdx.x * kRT + threadIdx.x; t < ncl; t += (uint64_t)gridDim.x * kRT) {
+    const uint32_t ch = __ldg(d.Cch + t);
+    const unsigned long long src = __ldg(d.Csrc + t);
+    if (__ldcg(owner + ch) == 0) owner[ch] = src;
   }
 }
 
@@ -243,7 +145,13 @@ __global__ void __launch_bounds__(kRT) claim_kernel(Geo g, RestoreDiff d, unsign
 // kCopyUnroll units per thread are in flight before any store. A chunk no diff claimed
 // (impossible for a well-formed lineage: diff 0 covers every chunk) reads as zeros, the
 // replay's starting buffer.
-constexpr int kCopyUnroll = 4;
+#ifndef CKPT_COPY_UNROLL
+#define CKPT_COPY_UNROLL 2
+#endif
+constexpr int kCopyUnroll = CKPT_COPY_UNROLL;   // measured: 2 ~ 1 < 4 < 8 (0.56 / 0.60 / 0.69 ms, config 2)
+#ifndef CKPT_COPY_LDG
+#define CKPT_COPY_LDG 1
+#endif
 __global__ void __launch_bounds__(kRT) copy_kernel(Geo g, const unsigned long long* owner, uint8_t* out) {
   pdl_launch_dependents();
   pdl_wait();
@@ -265,7 +173,11 @@ __global__ void __launch_bounds__(kRT) copy_kernel(Geo g, const unsigned long lo
       v[j] = make_uint4(0, 0, 0, 0);
       if (u >= nu || !src[j]) continue;
       if (16 * u + 16 <= g.B) {
+#if CKPT_COPY_LDG
+        v[j] = __ldg(reinterpret_cast<const uint4*>(src[j]));
+#else
         v[j] = __ldcs(reinterpret_cast<const uint4*>(src[j]));
+#endif
       } else {   // the buffer's last, partial unit: only its bytes (the source may end there)
         const uint8_t* sp = reinterpret_cast<const uint8_t*>(src[j]);
         uint32_t w[4] = {0, 0, 0, 0};
@@ -329,7 +241,7 @@ __global__ void basic_expand_kernel(Geo g, RestoreDiff d, uint64_t nwords, const
 __global__ void segmap_kernel(const unsigned long long* off, uint64_t nr, uint64_t nseg, unsigned long long* map) {
   const uint64_t sg = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (sg > nseg) return;
-  map[sg] = sg == nseg ? nr - 1 : region_at(off, nr, sg * (unsigned long long)kPaintSeg);
+  map[sg] = sg == nseg ? nr - 1 : region_at(off, nr, sg * (unsigned long long)kSegBytes);
 }
 
 __global__ void write_total_kernel(unsigned long long* off, const unsigned long long* len, uint64_t n) {
@@ -423,43 +335,56 @@ cudaError_t device_compare(const void* a, const void* b, uint64_t bytes, int* di
 
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st) {
   if (d.nF) {
-    const uint64_t ns = (d.data_bytes + kPaintSeg - 1) / kPaintSeg;
+    const uint64_t ns = (d.data_bytes + kSegBytes - 1) / kSegBytes;
     segmap_kernel<<<(unsigned)((ns + 256) / 256), 256, 0, st>>>(d.Foff, d.nF, ns, d.Fseg);
     note_launch();
   }
   if (d.nS) {
-    const uint64_t ns = (d.shift_bytes + kPaintSeg - 1) / kPaintSeg;
+    const uint64_t ns = (d.shift_bytes + kSegBytes - 1) / kSegBytes;
     segmap_kernel<<<(unsigned)((ns + 256) / 256), 256, 0, st>>>(d.Soff, d.nS, ns, d.Sseg);
     note_launch();
   }
   return cudaGetLastError();
 }
 
-uint64_t restore_segments(uint64_t bytes) { return (bytes + kPaintSeg - 1) / kPaintSeg; }
+uint64_t restore_segments(uint64_t bytes) { return (bytes + kSegBytes - 1) / kSegBytes; }
 
-cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st) {
-  if (d.nF == 0 && d.nS == 0) return cudaSuccess;
-  const uint64_t nx = (d.data_bytes + g.C - 1) / g.C + (d.shift_bytes + g.C - 1) / g.C;
+static int g_copy_bps = 0, g_claim_bps = 0;   // resident blocks per SM (occupancy, preload_restore)
+
+static uint64_t claim_count(const Geo& g, const RestoreDiff& d) {
+  return (d.data_bytes + g.C - 1) / g.C + (d.shift_bytes + g.C - 1) / g.C;
+}
+
+cudaError_t restore_claimlist(const Geo& g, const RestoreDiff& d, int num_sms, cudaStream_t st) {
+  const uint64_t nx = claim_count(g, d);
+  if (nx == 0) return cudaSuccess;
   uint64_t grid = (nx + kRT - 1) / kRT;
   const uint64_t cap = (uint64_t)num_sms * 8;
   if (grid > cap) grid = cap;
-  if (grid == 0) grid = 1;
-  return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, g, d, owner);
+  claimlist_kernel<<<(unsigned)grid, kRT, 0, st>>>(g, d);
+  note_launch();
+  return cudaGetLastError();
+}
+
+cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st) {
+  const uint64_t nx = claim_count(g, d);
+  if (nx == 0) return cudaSuccess;
+  uint64_t grid = (nx + kRT - 1) / kRT;
+  const uint64_t cap = (uint64_t)num_sms * (g_claim_bps > 0 ? g_claim_bps : 4);
+  if (grid > cap) grid = cap;
+  return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, d, nx, owner);
 }
 
 cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st) {
   const uint64_t nu = (g.B + 15) / 16;
   uint64_t grid = (nu + kRT * kCopyUnroll - 1) / (kRT * kCopyUnroll);
-  const uint64_t cap = (uint64_t)num_sms * 8;
+  // one resident wave: the grid-stride loop gives every block the same share, so blocks
+  // beyond what fits would run as a second, mostly idle wave
+  const uint64_t cap = (uint64_t)num_sms * (g_copy_bps > 0 ? g_copy_bps : 4);
   if (grid > cap) grid = cap;
   return launch_pdl(copy_kernel, (unsigned)grid, kRT, 0, st, g, owner, out);
 }
 
-cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
-                          int num_sms, cudaStream_t st) {
-  if (d.nF == 0 && d.nS == 0) return cudaSuccess;
-  return launch_pdl(paint_kernel, (unsigned)(num_sms * CKPT_PAINT_BPS), kRT, 0, st, g, d, out, painted, mark);
-}
 
 
 // Load this file's kernels now (CUDA lazy module loading would otherwise stall the first
@@ -470,9 +395,11 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_block_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, scan_add_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_first_kernel);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, paint_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, claim_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, claimlist_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, copy_kernel);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_copy_bps, copy_kernel, kRT, 0);
+  if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_claim_bps, claim_kernel, kRT, 0);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, prepare_shift_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, write_total_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, segmap_kernel);

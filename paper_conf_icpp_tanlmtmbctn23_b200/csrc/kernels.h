@@ -226,7 +226,9 @@ struct RestoreDiff {           // one diff of the chain, as the restore kernels 
   unsigned long long* Ssrc;    // per SHIFT region: device address of its source bytes
   unsigned long long shift_bytes;  // = Soff[nS]
   unsigned long long* Fseg;    // per 2-KB segment of the FIRST stream: region of its first byte (+1 entry)
-  unsigned long long* Sseg;    // same for the SHIFT stream
+  unsigned long long* Sseg;     // same for the SHIFT stream
+  uint32_t* Cch;               // claim list: per C-byte step of the FIRST then SHIFT stream, its
+  unsigned long long* Csrc;    //   chunk and the device address of its bytes (chunk-major restore)
 };
 cudaError_t restore_prepare_first(const Geo& g, RestoreDiff& d, unsigned long long* tmp_len, void* scan_tmp,
                                   size_t scan_tmp_bytes, cudaStream_t st);
@@ -237,10 +239,9 @@ cudaError_t restore_prepare_basic(const Geo& g, RestoreDiff& d, uint64_t nwords,
 cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st);
 cudaError_t device_compare(const void* a, const void* b, uint64_t bytes, int* diff, int num_sms, cudaStream_t st);
 uint64_t restore_segments(uint64_t bytes);
+cudaError_t restore_claimlist(const Geo& g, const RestoreDiff& d, int num_sms, cudaStream_t st);
 cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st);
 cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st);
-cudaError_t restore_paint(const Geo& g, const RestoreDiff& d, uint8_t* out, uint32_t* painted, uint32_t mark,
-                          int num_sms, cudaStream_t st);
 size_t scan_tmp_bytes_for(uint64_t count);
 cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long* out, uint64_t count, void* tmp,
                                size_t tmp_bytes, cudaStream_t st);
