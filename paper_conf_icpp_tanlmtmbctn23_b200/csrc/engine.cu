@@ -42,6 +42,9 @@ struct DiffRec {
   bool planned = false;
 };
 
+#ifndef CKPT_K1_GRAB_BYTES
+#define CKPT_K1_GRAB_BYTES 32768
+#endif
 #ifndef CKPT_TABLE_GROW_LOAD
 #define CKPT_TABLE_GROW_LOAD 0.6
 #endif
@@ -582,6 +585,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     lp.n_main = 0;   // odd chunk sizes above 128 B: direct-load pass only
   }
   lp.tail_begin = lp.n_main;
+  // one cursor grab per >= 32 KB of input (CKPT_K1_GRAB_BYTES): a tile is 256 C bytes
+  lp.tpg = (uint32_t)std::max<uint64_t>(1, (uint64_t)CKPT_K1_GRAB_BYTES / (kLeafThreads * (uint64_t)h->C));
   CUtensorMap tmap;
   if (lp.n_main) {
     r = make_tmap(h, buf, lp, &tmap);

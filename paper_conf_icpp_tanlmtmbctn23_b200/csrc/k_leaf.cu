@@ -235,8 +235,13 @@ __global__ void __launch_bounds__(kK1Threads, CKPT_K1_CTAS) leaf_hash_kernel(con
         if (p.ins.mode != kModeBasic) defer_tile(p.ins, tile, pc);   // Basic keeps no record
       }
     };
-    uint32_t tile = blockIdx.x, seg = 0, i = 0;
-    uint32_t nxt = tile < n_tiles ? gridDim.x + atomicAdd(cursor, 1u) : kNoTile;   // one tile ahead
+    // tiles are handed out in groups of tpg consecutive tiles (one cursor atomic per group:
+    // at small C a tile is only 256 C bytes, and one atomic per tile on one address
+    // throttled the producers)
+    const uint32_t tpg = p.tpg;
+    uint32_t grp = blockIdx.x, ing = 0;
+    uint32_t tile = grp * tpg, seg = 0, i = 0;
+    uint32_t nxt = tile < n_tiles ? gridDim.x + atomicAdd(cursor, 1u) : kNoTile;   // one group ahead
     for (;; ++i) {
       const int s = (int)(i % (uint32_t)nst);
       if (i >= (uint32_t)nst) {
@@ -262,8 +267,14 @@ __global__ void __launch_bounds__(kK1Threads, CKPT_K1_CTAS) leaf_hash_kernel(con
                   pol_stream);
       if ((int)++seg == segs) {
         seg = 0;
-        tile = nxt;
-        if (tile < n_tiles) nxt = gridDim.x + atomicAdd(cursor, 1u);
+        if (++ing < tpg && tile + 1 < n_tiles) {
+          ++tile;
+        } else {
+          ing = 0;
+          grp = nxt;
+          tile = grp < (n_tiles + tpg - 1) / tpg ? grp * tpg : n_tiles;
+          if (tile < n_tiles) nxt = gridDim.x + atomicAdd(cursor, 1u);
+        }
       }
     }
     // drain: the real steps after the last one handled above (i - nst + 1 .. i - 1)
@@ -530,7 +541,8 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   leaf_smem_config(p, &smem);
   const uint64_t n_tiles = p.n_main / kLeafThreads;
   uint64_t grid = (uint64_t)num_sms * CKPT_K1_CTAS;
-  if (grid > n_tiles) grid = n_tiles;
+  const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
+  if (grid > groups) grid = groups;
   if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else leaf_hash_kernel<0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   note_launch();

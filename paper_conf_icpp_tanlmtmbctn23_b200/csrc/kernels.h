@@ -81,6 +81,7 @@ struct LeafParams {
   int mode3d;            // 1: C % 128 == 0 (3-D map: row r of 256 chunks); 0: C < 128 (2-D rows)
   uint32_t stage_bytes;  // TMA bytes per pipeline stage
   int nst;               // pipeline stages
+  uint32_t tpg;          // tiles per cursor grab (>= 1; more at small C, see the K1 producer)
   Digest* prev;          // persistent leaf digests Tree(leaf), 16 n bytes
   uint32_t* cand;        // candidate (non-FIXED) bit per chunk
   InsertParams ins;      // record insert state (K1's producer warp marks/defers, K1b inserts)
