@@ -29,6 +29,20 @@ __device__ __forceinline__ void warp_sum3(unsigned long long& a, unsigned long l
 
 constexpr int kCT = 256;
 
+// Every counter the host reports is final once the gather kernel runs (tree kernels done,
+// pdl_wait): block 0 copies them to mapped host memory early, in 16-byte stores, so the
+// PCIe writes are long done when the last block publishes the epoch.
+__device__ __forceinline__ void host_totals(const CompactParams& p) {
+  static_assert(offsetof(Totals, done) % 4 == 0, "Totals layout");
+  const uint4* src = reinterpret_cast<const uint4*>(p.tot);
+  uint4* dst = reinterpret_cast<uint4*>(p.tot_host);
+  constexpr uint32_t nv = (uint32_t)(offsetof(Totals, done) / 16);
+  for (uint32_t i = 0; i < nv; ++i) dst[i] = __ldcg(src + i);
+  const uint32_t* s32 = reinterpret_cast<const uint32_t*>(p.tot);
+  uint32_t* d32 = reinterpret_cast<uint32_t*>(p.tot_host);
+  for (uint32_t w = nv * 4; w < (uint32_t)(offsetof(Totals, done) / 4); ++w) d32[w] = __ldcg(s32 + w);
+}
+
 // KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata
 // entries (its region records from phase 3) and copies its FIRST bytes. The data section
 // is the FIRST chunks in chunk order (every FIRST leaf lies in exactly one FIRST region,
@@ -99,7 +113,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       *reinterpret_cast<unsigned long long*>(o + 48) = g.B;
       *reinterpret_cast<unsigned long long*>(o + 56) = 0;  // hash seed, reserved
       *reinterpret_cast<uint4*>(o + 64) = make_uint4(0, 0, 0, 0);   // root entry (node 0) + pad
-      *p.tot_host = *t;
+      host_totals(p);
     }
     // the whole buffer, 16-byte units, kFullUnroll loads in flight per thread before the
     // stores (2 CTAs x 256 threads per SM: 64 KB in flight per SM covers HBM latency)
@@ -159,8 +173,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     *reinterpret_cast<uint32_t*>(o + 56) = 0;            // hash seed
     *reinterpret_cast<uint32_t*>(o + 60) = 0;            // reserved
     for (unsigned long long x = raw; x < meta; ++x) o[x] = 0;
-    // every counter the host reports is final here (tree kernels done, pdl_wait above)
-    *p.tot_host = *p.tot;
+    host_totals(p);
   }
   if (basic) {   // the bitmap: K1's candidate words, all n bits
     uint32_t* bm = reinterpret_cast<uint32_t*>(p.out + 64);
@@ -308,12 +321,14 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   }
   __syncthreads();
   if (threadIdx.x == 0) {
-    // the last block to finish publishes completion to the host (mapped memory): every
-    // byte of the diff is written, and every read of the caller's buffer is done. The
-    // system-scope fence orders block 0's mapped totals before the publication.
-    __threadfence_system();
+    // The last block to finish publishes completion to the host: every byte of the diff is
+    // written and every read of the caller's buffer is done. Blocks arrive with a gpu-scope
+    // fence (cumulative through the arrival counter); only the last one issues the system-
+    // scope fence before the epoch.
+    __threadfence();
     if (atomicAdd(&p.tot->blocks_done, 1u) + 1 == gridDim.x) {
-      __threadfence_system();
+      __threadfence();
+      __threadfence_system();   // block 0's mapped totals (written early) before the epoch
       *reinterpret_cast<volatile uint32_t*>(&p.tot_host->done) = g.epoch;
     }
   }
