@@ -175,8 +175,11 @@ __device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile,
 constexpr int kK1Threads = kLeafThreads + 32;
 constexpr int kMaxStagesK1 = 8;
 #ifndef CKPT_K1_CTAS
-#define CKPT_K1_CTAS 2   // resident K1 CTAs per SM (3 stages each when C % 128 == 0)
+#define CKPT_K1_CTAS 2   // resident K1 CTAs per SM when C % 128 == 0 (3 stages of 36 KB each)
 #endif
+#ifndef CKPT_K1_CTAS_SMALLC
+#define CKPT_K1_CTAS_SMALLC 3   // C < 128: a tile is only 256 C bytes and one producer thread per
+#endif                          // CTA bounds the rate (C = 32: 2 CTAs 320 us, 3 CTAs 288 us / GiB)
 constexpr uint32_t kNoTile = 0xFFFFFFFFu;
 
 struct K1Shared {
@@ -192,7 +195,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 }
 
 template <int MODE3D>
-__global__ void __launch_bounds__(kK1Threads, CKPT_K1_CTAS) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
+__global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
   const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -540,7 +543,7 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   size_t smem;
   leaf_smem_config(p, &smem);
   const uint64_t n_tiles = p.n_main / kLeafThreads;
-  uint64_t grid = (uint64_t)num_sms * CKPT_K1_CTAS;
+  uint64_t grid = (uint64_t)num_sms * (p.mode3d ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC);
   const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
   if (grid > groups) grid = groups;
   if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
