@@ -100,7 +100,7 @@ struct ckpt_ctx {
   unsigned long long* blocksum = nullptr;
   unsigned long long* gsum = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
-  Totals* tot_host = nullptr;   // pinned + mapped: written by the offsets kernel
+  Totals* tot_host = nullptr;   // pinned + mapped: written by the gather kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
   DiffArena arena;
@@ -701,7 +701,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   const auto t_synced = clk::now();
 
-  const Totals t = *h->tot_host;   // written by the offsets kernel (mapped host memory)
+  const Totals t = *h->tot_host;   // written by the gather kernel (mapped host memory)
   if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
     std::vector<uint32_t> cnt(8 * kTraceLanes);
     cudaMemcpy(cnt.data(), h->trace_n, cnt.size() * 4, cudaMemcpyDeviceToHost);

@@ -393,8 +393,8 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
 }
 
 // ------------------------------------------------------------------ K1b
-// Record inserts of the deferred 256-chunk tiles (all tiles at checkpoint 0, the ragged
-// tail, and whatever overflowed K1's ring): one warp per (tile, round of 32 candidates).
+// Record inserts of every 256-chunk tile with candidates (K1 and K1t defer them here, so
+// the streaming loop never waits on an atomic): one warp per (tile, round of 32 candidates).
 // Block 0 of K1b turns the dirty-tile bitmap into the tree kernels' work description: the
 // compact list of dirty stage-0 tiles (block scan) and, per upper group, the number of
 // dirty children (the climb target of the tree kernels).

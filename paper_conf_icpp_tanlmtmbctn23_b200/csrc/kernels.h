@@ -6,7 +6,7 @@
 //   K1b record inserts of the candidate chunks                 Alg.1 l.6-19 (R6)
 //   P2  phase 2, all stages in one launch (warp per group)     Alg.1 l.24-32
 //   P3  phase 3 + emission, all stages in one launch           Alg.1 l.33-46 (R7-R10)
-//   KR/KO/KG/KD tile reduce, offsets + header, entries, data
+//   KG  gather: offsets, header, entries and data in one launch
 #pragma once
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -147,7 +147,7 @@ struct CompactParams {
   uint32_t* trace_n;
   Totals* tot_host;              // mapped pinned host copy of the final totals (no D2H op)
   int dbg;                       // diagnostics only (CKPT_DBG bits; 0 in production)
-  uint4* ctr_next;               // the next call's counter block, zeroed by the data kernel
+  uint4* ctr_next;               // the next call's counter block, zeroed by the gather kernel
   uint64_t ctr_next_words;
   int mode;                      // CKPT_MODE_*: header flags; Basic writes the bitmap instead of entries
   const uint32_t* cand;          // Basic: the changed-chunk bitmap (K1)
