@@ -326,11 +326,9 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
         sh.words[st][wid] = mask;
       }
       if (cand) {
-        st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);
-        // a candidate's bytes may be copied into the diff by the gather kernel: keep the
-        // lines that TMA just brought in (evict_first) resident past the rest of the stream
-        const uint8_t* cp = p.buf + c * (uint64_t)p.g.C;
-        for (uint32_t o = 0; o < p.g.C; o += 128) l2_keep_line(cp + o);
+        // (raising the L2 priority of the candidate chunk's own lines for the gather kernel
+        // was measured neutral on configs 2 and 4 and is not done)
+        st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);   // K1b / the tree kernels re-read it
       }
     }
     __syncwarp();

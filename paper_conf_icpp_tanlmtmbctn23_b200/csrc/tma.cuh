@@ -67,12 +67,6 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
                : "memory");
 }
 
-// Raise the L2 eviction priority of the 128-B line at p (e.g. from the stream's evict_first)
-// to evict_normal; a no-op if the line is no longer resident.
-__device__ __forceinline__ void l2_keep_line(const void* p) {
-  asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(p) : "memory");
-}
-
 // L2 prefetch of a contiguous global range (16-B aligned, size a multiple of 16).
 __device__ __forceinline__ void prefetch_l2_bulk(const void* src, uint32_t bytes) {
   asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(src), "r"(bytes) : "memory");
