@@ -163,3 +163,20 @@ def test_alternate_engine_modes(oracle_mod, monkeypatch, dbg):
     run_parity(oracle_mod, bufs, 128)
     bufs = dup_lineage(77, 5000 * 64 - 7, 64, K=4, alphabet=5)
     run_parity(oracle_mod, bufs, 64)
+
+
+@pytest.mark.parametrize("nbytes", [1, 15, 16, 17, 31, 33, 47, 100])
+@pytest.mark.parametrize("variant", [None, (3, 500)])
+def test_tiny_buffers(oracle_mod, nbytes, variant):
+    """Buffers below one chunk up to a few chunks, with partial last 16-byte units: diffs,
+    digests, record and the chunk-major restore's partial-unit path (R4)."""
+    rng = np.random.default_rng(nbytes)
+    C = 32
+    base = rng.integers(0, 256, nbytes, dtype=np.uint8)
+    bufs = [base.copy()]
+    for k in range(1, 5):
+        b = bufs[-1].copy()
+        if k % 2:
+            b[int(rng.integers(0, nbytes))] ^= 0x5A
+        bufs.append(b)
+    run_parity(oracle_mod, bufs, C, variant=variant)
