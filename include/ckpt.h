@@ -148,8 +148,11 @@ CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes,
  * first-time occurrences, then fill the fixed duplicates and finally assemble the shifted
  * duplicates from the corresponding checkpoint ID"). Equivalent to replaying diffs 0..id
  * (R16), computed directly: each chunk is written once, from the newest diff <= id whose
- * regions cover it. Per-diff restore plans are built by the first
- * restore that needs them and cached (about 2-3x the diff's metadata in device memory).
+ * regions cover it: per diff, newest first, the chunks it covers
+ * are claimed (source address per chunk), then one kernel copies every chunk once.
+ * Per-diff restore plans are built by the first restore that needs them and cached: about
+ * 2-3x the diff's metadata plus 12 bytes per chunk the diff covers, in device memory; the
+ * handle also keeps 8 bytes per chunk of the buffer for the claims.
  *   dev_ptr  device buffer of B bytes, 16-byte aligned, owned by the caller; overwritten.
  * Synchronous (runs on an internal stream of the handle).
  * Errors: CKPT_ERANGE (id >= number of checkpoints), CKPT_EINVAL, CKPT_ECUDA, CKPT_ESTATE. */
