@@ -240,18 +240,23 @@ __device__ __forceinline__ uint64_t table_claim_cas(Slot* tab, uint64_t cap, con
 // Insert-or-min: Map.insert(digest, entry) of Alg.1 l.7 with the R6 tie-break. The value
 // only decreases, so a value already <= packed (an entry of an earlier checkpoint, the
 // common case for temporal duplicates) needs no atomic at all.
+// *seen_out: the value observed when the key already existed (kEmpty when this call claimed
+// it); a value below (ckpt k) << 32 is an entry of an earlier checkpoint and final.
 __device__ __forceinline__ uint64_t table_insert_min(Slot* tab, uint64_t cap, const Digest& d, unsigned long long packed,
-                                                    bool* claimed, bool cas_first = false) {
+                                                    bool* claimed, bool cas_first, unsigned long long* seen_out) {
   if (cas_first) {
     const uint64_t s = table_claim_cas(tab, cap, d, claimed);
     Slot* p = tab + s;
-    if (*claimed || ld_val_relaxed(p) > packed) atomicMin(&p->val, packed);
+    const unsigned long long v = *claimed ? kEmpty : ld_val_relaxed(p);
+    if (*claimed || v > packed) atomicMin(&p->val, packed);
+    *seen_out = v;
     return s;
   }
   unsigned long long seen;
   const uint64_t s = table_find_or_claim(tab, cap, d, claimed, &seen);
   Slot* p = tab + s;
   if (*claimed || seen > packed) atomicMin(&p->val, packed);
+  *seen_out = *claimed ? kEmpty : seen;
   return s;
 }
 

@@ -76,7 +76,7 @@ struct ckpt_ctx {
   Digest* prev = nullptr;
   uint32_t* cand = nullptr;
   uint64_t nwords = 0;
-  uint32_t* slot_of = nullptr;
+  unsigned long long* res_of = nullptr;   // per chunk (candidates only): K1b's resolution
   LevelIO lvl[kMaxStages] = {};
   Digest* tdig[kMaxStages] = {};
   unsigned long long* tsrc[kMaxStages] = {};
@@ -197,7 +197,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   } while (0)
   AL(h->prev, n);
   AL(h->cand, h->nwords + 32);
-  AL(h->slot_of, n);
+  AL(h->res_of, n);
   for (int s = 0; s < h->S; ++s) {
     if (s >= 1) {
       const uint64_t P = 1ull << (h->h - h->Lin[s]);
@@ -545,7 +545,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   InsertParams ip;
   std::memset(&ip, 0, sizeof(ip));
   ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
-  ip.tab = h->tab; ip.cap = h->cap; ip.slot_of = h->slot_of;
+  ip.tab = h->tab; ip.cap = h->cap; ip.res_of = h->res_of;
   ip.tot = h->tot;
   ip.defer = h->defer;
   ip.dbits = h->dbits;
@@ -622,7 +622,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.wl0 = h->wl0;
   tp.buf = buf;
   tp.tcc = h->tcc;
-  tp.cand = h->cand; tp.slot_of = h->slot_of; tp.prev = h->prev;
+  tp.cand = h->cand; tp.res_of = h->res_of; tp.prev = h->prev;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
   tp.blocksum = h->blocksum;

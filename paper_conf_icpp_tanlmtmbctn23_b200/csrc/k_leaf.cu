@@ -89,17 +89,21 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
         const uint32_t vv = __shfl_sync(active, node, sl);
         if ((grp >> sl) & 1u) minnode = vv < minnode ? vv : minnode;
       }
-      uint32_t slot = 0;
+      unsigned long long res = 0;
       if (lane == leader) {
         bool claimed;
+        unsigned long long seen;
         // Sparse candidates after checkpoint 0 are mostly new keys (CAS first: one round trip).
         // Checkpoint 0 and dense tiles (moved or repeated content) mostly hit existing keys:
         // read key + value first, no atomic when the entry is older (one round trip).
-        slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed,
-                                          p.g.k > 0 && total < kDenseTile);
+        const uint32_t slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, minnode), &claimed,
+                                                         p.g.k > 0 && total < kDenseTile, &seen);
+        // an entry of an earlier checkpoint never changes again (R6): the leaf is resolved
+        // here (SHIFT to it); otherwise phase 2 reads the final value from the slot
+        res = seen < ((unsigned long long)p.g.k << 32) ? seen : (kResPending | slot);
       }
-      slot = __shfl_sync(active, slot, leader);
-      st_evict_last_u32(p.slot_of + c, slot, pol);
+      res = __shfl_sync(active, res, leader);
+      st_evict_last_u64(p.res_of + c, res, pol);
     }
   }
   ncand += b_end - b_begin;

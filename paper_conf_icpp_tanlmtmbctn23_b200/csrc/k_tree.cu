@@ -310,7 +310,7 @@ __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint6
   const uint32_t total = batch_begin(ws, cand);
   for (uint32_t base = 0; base < total; base += 32 * kB) {
     uint64_t ch[kB];
-    uint32_t iw[kB], ib[kB], slot[kB];
+    uint32_t iw[kB], ib[kB];
     unsigned long long val[kB];
 #pragma unroll
     for (int t = 0; t < kB; ++t) {
@@ -323,10 +323,12 @@ __device__ __forceinline__ void resolve_leaves(const Ctx& c, WarpSmem& ws, uint6
     }
 #pragma unroll
     for (int t = 0; t < kB; ++t)
-      if (ch[t] != ~0ull) slot[t] = __ldg(p.slot_of + ch[t]);
+      if (ch[t] != ~0ull) val[t] = __ldg(p.res_of + ch[t]);
+    // leaves K1b could not resolve (their key was claimed or lowered in this checkpoint):
+    // the final value after every insert
 #pragma unroll
     for (int t = 0; t < kB; ++t)
-      if (ch[t] != ~0ull) val[t] = __ldcg(&p.tab[slot[t]].val);
+      if (ch[t] != ~0ull && (val[t] & kResPending)) val[t] = __ldcg(&p.tab[(uint32_t)val[t]].val);
 #pragma unroll
     for (int t = 0; t < kB; ++t) {
       if (ch[t] == ~0ull) continue;

@@ -22,6 +22,7 @@ constexpr int kGroupLog = 10;   // upper stages: 1024 positions per group
 constexpr int kLeafThreads = 256;
 constexpr int kTreeThreads = 256;
 constexpr int kTilesPerBlock = 1024;  // compaction: tiles per reduce/offsets CTA
+constexpr unsigned long long kResPending = 1ull << 63;   // res_of: value not final after K1b
 constexpr int kModeTree = 0, kModeList = 1, kModeBasic = 2;   // = CKPT_MODE_* (include/ckpt.h)
 #ifdef CKPT_K1_STAGES
 constexpr int kLeafStages3d = CKPT_K1_STAGES;   // experiment builds
@@ -53,7 +54,7 @@ struct InsertParams {
   uint64_t nwords;
   Slot* tab;
   uint64_t cap;
-  uint32_t* slot_of;
+  unsigned long long* res_of;    // per candidate: final record value, or kResPending | slot
   Totals* tot;
   uint32_t* defer;               // (tile << 3 | round) entries left for K1b
   // tree work discovery (K1/K1t mark, K1b block 0 compacts)
@@ -113,7 +114,7 @@ struct TreeParams {
   const uint8_t* buf;          // checkpoint buffer (phase 3 prefetches FIRST bytes into L2)
   const uint32_t* tcc;         // candidate leaves per stage-0 tile (K1/K1t)
   const uint32_t* cand;
-  const uint32_t* slot_of;
+  const unsigned long long* res_of;   // per candidate (K1b): final value or kResPending | slot
   const Digest* prev;
   Slot* tab;
   uint64_t cap;

@@ -75,6 +75,9 @@ __device__ __forceinline__ void prefetch_l2_bulk(const void* src, uint32_t bytes
 __device__ __forceinline__ void st_evict_last_v2(void* p, uint64_t a, uint64_t b, uint64_t pol) {
   asm volatile("st.global.L2::cache_hint.v2.u64 [%0], {%1, %2}, %3;" ::"l"(p), "l"(a), "l"(b), "l"(pol) : "memory");
 }
+__device__ __forceinline__ void st_evict_last_u64(void* p, uint64_t a, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(a), "l"(pol) : "memory");
+}
 __device__ __forceinline__ void st_evict_last_u32(void* p, uint32_t a, uint64_t pol) {
   asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(a), "l"(pol) : "memory");
 }
