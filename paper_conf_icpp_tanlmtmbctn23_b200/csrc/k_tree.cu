@@ -40,6 +40,9 @@ constexpr int kWarps = kTreeThreads / 32;
 #ifndef CKPT_TREE_BPS
 #define CKPT_TREE_BPS 2   // tree-kernel launch bound: resident CTAs per SM (register budget)
 #endif
+#ifndef CKPT_SIBLING_SHORTCUT
+#define CKPT_SIBLING_SHORTCUT 1   // phase 3: level-1 pairs whose sources are siblings need no lookup
+#endif
 #ifndef CKPT_TREE_CURSOR
 #define CKPT_TREE_CURSOR 1   // worklist entries beyond the first per warp from a cursor (0: static stride)
 #endif
@@ -74,6 +77,7 @@ struct WarpSmem {
   uint32_t W[32];       // pass-1 nodes of all levels (layout below)
   uint32_t WP[32];      // exclusive prefix of popc(W): a pass-1 node's rank = its compact digest index
   uint32_t H[32];       // pass-2 lookup hits (same layout)
+  uint32_t K[32];       // phase 3: level-1 pairs resolved without a lookup (same layout)
   uint16_t items[1 << kTileLog];   // the set bits of the current work mask as a list (word << 5 | bit)
   Digest dig[kDigCap];  // compact on-chip digests of pass-1 nodes (rank < kDigCap; others: global)
   uint8_t lvl[1 << kTileLog];   // level of the region starting at each slot
@@ -538,6 +542,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   } else {
   // ---- pass 1: digests bottom-up, no record traffic (see file header)
   ws.W[lane] = 0;
+  ws.K[lane] = 0;
   __syncwarp();
   if (__any_sync(0xffffffffu, ((PHASE == 2 ? F : S) | (PHASE == 2 ? lF1 : lS1)) != 0)) {
     uint32_t P = PHASE == 2 ? F : S;
@@ -569,6 +574,20 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
       }
       __syncwarp();
       for_each_bit_balanced(ws, work, [&](uint32_t, uint32_t, uint32_t q) {
+        if (PHASE == 3 && lv == 1 && CKPT_SIBLING_SHORTCUT) {
+          // Both children are SHIFT with known sources. If they are the two children of one
+          // node v of checkpoint c (left = 2v+1, right = 2v+2), both were FIRST in c, so
+          // phase 2 of c inserted (v, c) for exactly this digest (the record never replaces
+          // an entry, R6): the lookup of Alg.1 l.39 would return it, and is skipped.
+          // (Applying the same rule at higher levels, from children resolved this way,
+          // measured slower: config 4 phase 3 425 -> 434 us.)
+          const unsigned long long sL = child_src(c, 0, q), sR = child_src(c, 0, q + (uint32_t)Np);
+          const uint32_t nl = (uint32_t)sL, nr = (uint32_t)sR;
+          if ((sL >> 32) == (sR >> 32) && (nl & 1u) && nr == nl + 1) {
+            atomicOr(&ws.K[q >> 5], 1u << (q & 31));
+            c.tsrc[P0 + lvl_off(P0, 1) + q] = (sL & 0xFFFFFFFF00000000ull) | ((nl - 1) >> 1);
+          }
+        }
         const Digest d = mm::node(child_digest(c, ws, lv - 1, q), child_digest(c, ws, lv - 1, q + (uint32_t)Np));
         dig_store(ws, c.tdig, lay_rank(ws, lv, q), d);
       });
@@ -578,12 +597,13 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   __syncwarp();
   if (p.trace && lane == 0) ws.tp[1] = gtimer();
 
-  // ---- pass 2: record operations for all pass-1 nodes at once
-  ws.H[lane] = 0;
+  // ---- pass 2: record operations for all pass-1 nodes at once (phase 3: but the pairs
+  // pass 1 resolved from their children's sources)
+  ws.H[lane] = PHASE == 3 ? ws.K[lane] : 0u;
   __syncwarp();
   {
     constexpr int kB2 = 2;
-    const uint32_t total = batch_begin(ws, ws.W[lane]);
+    const uint32_t total = batch_begin(ws, PHASE == 3 ? (ws.W[lane] & ~ws.K[lane]) : ws.W[lane]);
     for (uint32_t base = 0; base < total; base += 32 * kB2) {
       uint32_t iw[kB2], ib[kB2];
       int lvs[kB2];
