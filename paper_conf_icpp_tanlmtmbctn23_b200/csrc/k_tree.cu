@@ -40,6 +40,9 @@ constexpr int kWarps = kTreeThreads / 32;
 #ifndef CKPT_TREE_BPS
 #define CKPT_TREE_BPS 2   // tree-kernel launch bound: resident CTAs per SM (register budget)
 #endif
+#ifndef CKPT_TREE_KB2
+#define CKPT_TREE_KB2 2   // pass-2 record operations per lane in flight (3 and 4 spill: config 4 phase 3 +40-55 %)
+#endif
 #ifndef CKPT_SIBLING_SHORTCUT
 #define CKPT_SIBLING_SHORTCUT 1   // phase 3: level-1 pairs whose sources are siblings need no lookup
 #endif
@@ -602,7 +605,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   ws.H[lane] = PHASE == 3 ? ws.K[lane] : 0u;
   __syncwarp();
   {
-    constexpr int kB2 = 2;
+    constexpr int kB2 = CKPT_TREE_KB2;
     const uint32_t total = batch_begin(ws, PHASE == 3 ? (ws.W[lane] & ~ws.K[lane]) : ws.W[lane]);
     for (uint32_t base = 0; base < total; base += 32 * kB2) {
       uint32_t iw[kB2], ib[kB2];
