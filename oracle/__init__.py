@@ -195,6 +195,20 @@ class Oracle:
             raise RuntimeError("record dump unavailable in ideal mode")
         return {(keys[i].tobytes(), int(nodes[i]), int(ckpts[i])) for i in range(m)}
 
+    def record_array(self) -> np.ndarray:
+        """The record as a sorted array of rows (key lo, key hi, ckpt << 32 | node), u64 each
+        (the same content as record(), for fast comparison at millions of entries)."""
+        m = self.record_size()
+        keys = np.zeros((max(m, 1), 16), dtype=np.uint8)
+        nodes = np.zeros(max(m, 1), dtype=np.uint32)
+        ckpts = np.zeros(max(m, 1), dtype=np.uint32)
+        if lib().orc_record_dump(self._h, _ptr(keys), _ptr(nodes), _ptr(ckpts)) != 0:
+            raise RuntimeError("record dump unavailable in ideal mode")
+        rows = np.empty((m, 3), dtype=np.uint64)
+        rows[:, :2] = keys[:m].view(np.uint64)
+        rows[:, 2] = (ckpts[:m].astype(np.uint64) << np.uint64(32)) | nodes[:m]
+        return rows[np.lexsort((rows[:, 2], rows[:, 1], rows[:, 0]))]
+
     def restore(self, cid: int) -> bytes:
         out = np.zeros(max(self.buf_bytes or 1, 1), dtype=np.uint8)
         rc = lib().orc_restore(self._h, cid, _ptr(out))

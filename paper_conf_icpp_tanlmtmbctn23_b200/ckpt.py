@@ -257,6 +257,29 @@ class Checkpointer:
         k = cnt.value
         return {(keys[i].tobytes(), int(nodes[i]), int(ckpts[i])) for i in range(k)}
 
+    def record_array(self):
+        """Historical record as a sorted numpy array of rows (key lo, key hi, ckpt << 32 | node),
+        u64 each: the same content as record(), comparable with np.array_equal at millions of
+        entries."""
+        import numpy as np
+        cnt = ctypes.c_uint64()
+        rc = lib().ckpt_record_dump(self._h, None, None, None, 0, ctypes.byref(cnt))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_record_dump")
+        m = cnt.value + 16
+        keys = np.zeros((m, 16), dtype=np.uint8)
+        nodes = np.zeros(m, dtype=np.uint32)
+        ckpts = np.zeros(m, dtype=np.uint32)
+        rc = lib().ckpt_record_dump(self._h, keys.ctypes.data, nodes.ctypes.data, ckpts.ctypes.data, m,
+                                    ctypes.byref(cnt))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_record_dump")
+        k = cnt.value
+        rows = np.empty((k, 3), dtype=np.uint64)
+        rows[:, :2] = keys[:k].view(np.uint64)
+        rows[:, 2] = (ckpts[:k].astype(np.uint64) << np.uint64(32)) | nodes[:k]
+        return rows[np.lexsort((rows[:, 2], rows[:, 1], rows[:, 0]))]
+
     def set_profiling(self, level: int | bool = 2) -> None:
         """0/False off; 1 = CUDA events around K1 and the whole call only (keeps the
         kernels' programmatic early launch, so this is the level to time under); 2/True =

@@ -42,3 +42,33 @@ def test_fig2(oracle_mod):
     assert st["list_entries"] == g["ckpt1_list_entries"]
     assert st["n_first_regions"] + st["n_shift_regions"] == g["ckpt1_tree_entries"]
     assert o.restore(0) == b0 and o.restore(1) == b1
+
+
+def test_fig2_internal_node_keys(oracle_mod):
+    """R2 ("hashing the left child's hash with the right child's hash"): the record
+    keys of Figure 2's phase-2 nodes are MMH3 over the 32-byte concatenation T[l] || T[r],
+    seed 0. The expected keys are composed here from the SMHasher-pinned leaf hash
+    (tests/test_oracle_murmur.py), not from the oracle's tree code, so an oracle that hashed
+    r || l, used another seed or a domain separator would fail."""
+    g = json.load(open(GOLD))
+    C = g["chunk_bytes"]
+    cont = {nm: _content(nm, C) for nm in set(g["ckpt0"] + g["ckpt1"])}
+    o = oracle_mod.Oracle(C)
+    o.checkpoint(b"".join(cont[x] for x in g["ckpt0"]))
+    o.checkpoint(b"".join(cont[x] for x in g["ckpt1"]))
+    h = oracle_mod.mmh3
+    T = {7: h(cont["I"]), 8: h(cont["J"]), 9: h(cont["K"]), 10: h(cont["L"])}
+    T[3] = h(T[7] + T[8])
+    T[4] = h(T[9] + T[10])
+    T[1] = h(T[3] + T[4])
+    rec = {(key, node, ck) for (key, node, ck) in o.record()}
+    for u in (7, 8, 9, 10, 3, 4, 1):
+        assert (T[u], u, 1) in rec, u
+    keys = {key for (key, _, _) in rec}
+    assert h(T[8] + T[7]) not in keys          # not r || l
+    assert h(T[7] + T[8], 1) not in keys       # not another seed
+    # checkpoint 0 taken whole: the root key is the Merkle root of A0..A7 (P:95)
+    L = [h(cont[f"A{i}"]) for i in range(8)]
+    while len(L) > 1:
+        L = [h(L[2 * i] + L[2 * i + 1]) for i in range(len(L) // 2)]
+    assert (L[0], 0, 0) in rec
