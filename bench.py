@@ -8,8 +8,11 @@ C = 128 B, row-run update rate p = 1 %), inputs already resident in HBM.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-N > 1: launched by torchrun, one process per GPU; each rank de-duplicates its own buffer
-(seed + rank, the paper's setting P:184, weak scaling); timing = max over ranks.
+N > 1: one process per GPU — launched by torchrun, or by bench.py itself (it re-runs the
+command under torch.distributed.run when WORLD_SIZE is absent); each rank de-duplicates its
+own buffer (seed + rank, the paper's setting P:184, weak scaling); timing = max over ranks.
+--config 5 (16 GiB per GPU) mutates one buffer in place between steps (the lineage would
+not fit in HBM); the default config 2 pre-generates the whole lineage in HBM.
 """
 from __future__ import annotations
 
@@ -37,12 +40,16 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", type=int, default=2)
-    ap.add_argument("--bytes", type=int, default=GiB)
+    ap.add_argument("--bytes", type=int, default=None, help="buffer bytes per GPU (default: 1 GiB; config 5: 16 GiB)")
     ap.add_argument("--chunk", type=int, default=128)
     ap.add_argument("--p", type=float, default=0.01)
     ap.add_argument("--e2e-steps", type=int, default=4)
-    ap.add_argument("--cpu-sample-bytes", type=int, default=256 << 20)
+    ap.add_argument("--cpu-sample-bytes", type=int, default=GiB)
+    ap.add_argument("--cpu-steps", type=int, default=8, help="steady checkpoints the CPU oracle times")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--inplace", action="store_true",
+                    help="one buffer mutated between steps (automatic when the lineage does not fit)")
+    ap.add_argument("--dist-selftest", action="store_true", help=argparse.SUPPRESS)
     return ap.parse_args()
 
 
@@ -109,6 +116,7 @@ def dist_setup(n_gpus):
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert ws == n_gpus, f"--gpus {n_gpus} but WORLD_SIZE={ws}"
     if ws > 1:
         import torch.distributed as dist
         torch.cuda.set_device(local)
@@ -177,87 +185,140 @@ def file_offsets(gathered):
 
 
 # ------------------------------------------------------------------ CPU oracle arm
-def oracle_sample(cfg, nbytes, C, p, n_timed, seed, use_device_gen=True):
-    """Runs the CPU oracle (as it stands) on a bounded sample of the workload:
-    checkpoint 0 untimed, then n_timed steady checkpoints. Returns (GB/s, seconds, n)."""
+def cpu_info():
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for ln in f:
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"nproc": os.cpu_count(), "cpu_model": model}
+
+
+def oracle_lineage_timed(cfg, nbytes, C, p, n_untimed, n_timed, seed):
+    """The CPU oracle (as it stands, single-threaded) over checkpoints 0 .. n_untimed +
+    n_timed - 1 of the config's lineage at `nbytes`; the buffers are generated on the device
+    (or on the host without a GPU) one at a time and handed over as host arrays, and only
+    the oracle's calls on the last n_timed checkpoints are timed. Returns (GB/s, seconds)."""
     import numpy as np
     import oracle
     from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
-    bufs = []
-    if use_device_gen:
-        import torch
-        t = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
-        W.DeviceGen.initial(cfg, t, nbytes, seed)
-        bufs.append(t.cpu().numpy())
-        for k in range(1, n_timed + 1):
-            W.DeviceGen.mutate(cfg, t, nbytes, k, C, seed, p)
-            bufs.append(t.cpu().numpy())
-        del t
-    else:
-        it = W.lineage(cfg, nbytes, C, n_timed + 1, seed=seed, p=p)
-        bufs = [np.array(b) for b in it]
-    o = oracle.Oracle(C)
-    o.checkpoint(bufs[0])
-    t0 = time.perf_counter()
-    for b in bufs[1:]:
-        o.checkpoint(b)
-    dt = time.perf_counter() - t0
-    return n_timed * nbytes / dt / 1e9, dt, n_timed
-
-
-def run_reference(args):
-    ws = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    if rank != 0:
-        return 0
-    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
-    nb = args.cpu_sample_bytes
-    seed = W.seed_of(args.config)
     try:
         import torch
         have_gpu = torch.cuda.is_available()
     except Exception:
         have_gpu = False
-    K, Wm = args.steps, args.warmup
-    import numpy as np
-    import oracle
-    it = None
-    bufs = []
+    o = oracle.Oracle(C)
+    dt = 0.0
     if have_gpu:
-        import torch
-        t = torch.empty(nb, dtype=torch.uint8, device="cuda")
-        W.DeviceGen.initial(args.config, t, nb, seed)
-        bufs.append(t.cpu().numpy())
-        for k in range(1, Wm + K):
-            W.DeviceGen.mutate(args.config, t, nb, k, args.chunk, seed, args.p)
-            bufs.append(t.cpu().numpy())
+        t = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+        for k in range(n_untimed + n_timed):
+            if k == 0:
+                W.DeviceGen.initial(cfg, t, nbytes, seed)
+            else:
+                W.DeviceGen.mutate(cfg, t, nbytes, k, C, seed, p)
+            b = t.cpu().numpy()
+            t0 = time.perf_counter()
+            o.checkpoint(b)
+            if k >= n_untimed:
+                dt += time.perf_counter() - t0
+        del t
     else:
-        bufs = list(W.lineage(args.config, nb, args.chunk, Wm + K, seed=seed, p=args.p))
-    o = oracle.Oracle(args.chunk)
-    for b in bufs[:Wm]:
-        o.checkpoint(b)
-    t0 = time.perf_counter()
-    for b in bufs[Wm:]:
-        o.checkpoint(b)
-    dt = time.perf_counter() - t0
-    val = K * nb / dt / 1e9
+        for k, b in enumerate(W.lineage(cfg, nbytes, C, n_untimed + n_timed, seed=seed, p=p)):
+            t0 = time.perf_counter()
+            o.checkpoint(np.asarray(b))
+            if k >= n_untimed:
+                dt += time.perf_counter() - t0
+    return n_timed * nbytes / dt / 1e9, dt
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0   # N > 1: rank 0 alone times the oracle (it is a CPU program)
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    B = args.bytes
+    nb = min(B, args.cpu_sample_bytes)
+    seed = W.seed_of(args.config)
+    K, Wm = args.steps, args.warmup
+    val, dt = oracle_lineage_timed(args.config, nb, args.chunk, args.p, Wm, K, seed)
+    same = nb == B
     line = {
         "impl": "reference", "metric": METRIC, "value": round(val, 4), "unit": "GB/s",
         "n_gpus": args.gpus, "steps": K, "warmup": Wm, "ms_per_step": round(1e3 * dt / K, 3),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": f"config{args.config} GDV-like (BASELINE configs[1] recipe)", "buffer_bytes": nb,
-                   "chunk_bytes": args.chunk, "update_rate": args.p},
-        "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                         "sample": f"config-{args.config} lineage at {nb >> 20} MiB: {Wm} untimed checkpoints "
-                                   f"(incl. checkpoint 0) then {K} timed steady checkpoints, single-threaded C++ "
-                                   f"oracle (oracle/oracle.cpp)"},
+        "config": workload_config(args, 1),
+        "cpu_baseline": {"value": round(val, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", **cpu_info(),
+                         "sample": (f"config-{args.config} lineage at {nb >> 20} MiB"
+                                    + ("" if same else f" (of the {B >> 20} MiB workload)")
+                                    + f": {Wm} untimed checkpoints (incl. checkpoint 0) then {K} timed steady "
+                                      f"checkpoints, single-threaded C++ oracle (oracle/oracle.cpp)")},
         "e2e": {"value": round(val, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
     return 0
 
 
+def workload_config(args, ws, inplace=False):
+    B, C, p, cfg = args.bytes, args.chunk, args.p, args.config
+    if cfg in (2, 5) and C == 128:
+        name = (f"config{cfg}: {B / GiB:g} GiB GDV-like buffer per GPU (73 x u32 rows), C = 128 B, "
+                f"row-run updates p = {p}")
+    else:
+        name = f"config{cfg} B={B} C={C} p={p}"
+    return {"workload": name, "buffer_bytes": B, "chunk_bytes": C, "update_rate": p,
+            "parallelism": f"independent x{ws}",
+            "l2": ("one buffer per GPU mutated in place between steps (outside the timed events), L2 flushed "
+                   "(256 MiB write) before each step; value = K B / sum of per-step event times"
+                   if inplace else
+                   f"inputs ({B / GiB:g} GiB per step, distinct buffers) larger than the 126 MB L2; no flush")}
+
+
 # ------------------------------------------------------------------ our arm
+class Lineage:
+    """Checkpoint k's input buffer on the device. Resident: the whole lineage pre-generated
+    in HBM (inputs resident when timing starts). In place: one buffer advanced by the
+    generator (k must not decrease except to restart at 0); used when the lineage does not
+    fit (config 5: 16 GiB per GPU)."""
+
+    def __init__(self, cfg, B, C, p, seed, n, stream, inplace):
+        import torch
+        from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+        self.W, self.cfg, self.B, self.C, self.p, self.seed, self.stream = W, cfg, B, C, p, seed, stream
+        self.inplace = inplace
+        if inplace:
+            self.buf = torch.empty(B, dtype=torch.uint8, device="cuda")
+            self.cur = -1
+        else:
+            self.bufs = [torch.empty(B, dtype=torch.uint8, device="cuda") for _ in range(n)]
+            with torch.cuda.stream(stream):
+                W.DeviceGen.initial(cfg, self.bufs[0], B, seed, stream)
+                for k in range(1, n):
+                    self.bufs[k].copy_(self.bufs[k - 1])
+                    W.DeviceGen.mutate(cfg, self.bufs[k], B, k, C, seed, p, stream)
+            stream.synchronize()
+
+    def get(self, k):
+        if not self.inplace:
+            return self.bufs[k]
+        if k < self.cur:
+            self.cur = -1
+        while self.cur < k:
+            self.cur += 1
+            if self.cur == 0:
+                self.W.DeviceGen.initial(self.cfg, self.buf, self.B, self.seed, self.stream)
+            else:
+                self.W.DeviceGen.mutate(self.cfg, self.buf, self.B, self.cur, self.C, self.seed, self.p, self.stream)
+        return self.buf
+
+    def release(self):
+        self.bufs = None
+        self.buf = None
+
+
 def run_ours(args):
     import torch
     from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
@@ -269,14 +330,10 @@ def run_ours(args):
     assert Wm >= 3, "timing rules: at least 3 warm-up steps"
     seed = W.seed_of(cfg, rank)
     stream = torch.cuda.Stream()
-    # whole lineage pre-generated in HBM (inputs resident when timing starts; 1 GiB each > L2)
-    bufs = [torch.empty(B, dtype=torch.uint8, device="cuda") for _ in range(Wm + K)]
-    with torch.cuda.stream(stream):
-        W.DeviceGen.initial(cfg, bufs[0], B, seed, stream)
-        for k in range(1, Wm + K):
-            bufs[k].copy_(bufs[k - 1])
-            W.DeviceGen.mutate(cfg, bufs[k], B, k, C, seed, p, stream)
-    stream.synchronize()
+    total_mem = torch.cuda.get_device_properties(local).total_memory
+    inplace = args.inplace or (Wm + K) * B > 0.45 * total_mem
+    lin = Lineage(cfg, B, C, p, seed, Wm + K, stream, inplace)
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if inplace else None
 
     ck = Checkpointer(C)
     # level 1: CUDA events only around K1 (the roofline kernel) and the whole call; events
@@ -285,54 +342,60 @@ def run_ours(args):
     diffs = []
     ck0 = None
     for k in range(Wm):
-        diffs.append(ck.checkpoint(bufs[k], stream=stream))
+        diffs.append(ck.checkpoint(lin.get(k), nbytes=B, stream=stream))
         if k == 0:
             ck0 = ck.phase_times(0)
     n = (B + C - 1) // C
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     k1_ms, phase = [], []
+    raw = []
     barrier(ws)
     torch.cuda.synchronize()
-    raw = []
     launches0 = ck.kernel_launches
     with ClockSampler(local) as clk:
-        ev0.record(stream)
-        for k in range(Wm, Wm + K):
-            raw.append(ck.checkpoint(bufs[k], nbytes=B, stream=stream, raw=True))
-        ev1.record(stream)
-        stream.synchronize()
+        if not inplace:
+            ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ev0.record(stream)
+            for k in range(Wm, Wm + K):
+                raw.append(ck.checkpoint(lin.get(k), nbytes=B, stream=stream, raw=True))
+            ev1.record(stream)
+            stream.synchronize()
+            ms_local = ev0.elapsed_time(ev1)
+        else:
+            evs = []
+            for k in range(Wm, Wm + K):
+                buf = lin.get(k)                       # generator, outside the events
+                with torch.cuda.stream(stream):
+                    flush.fill_(k & 255)               # L2 flush, outside the events
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                raw.append(ck.checkpoint(buf, nbytes=B, stream=stream, raw=True))
+                b.record(stream)
+                evs.append((a, b))
+            stream.synchronize()
+            ms_local = sum(a.elapsed_time(b) for a, b in evs)
     launches = ck.kernel_launches - launches0
+    torch.cuda.synchronize()
+    barrier(ws)
+    ms = max_over_ranks(ms_local, ws)
+    total_bytes = sum_over_ranks(float(K * B), ws)
+    value = total_bytes / (ms / 1e3) / 1e9
     # K1 and whole-call device times of the timed checkpoints (CUDA events recorded by the
     # library on `stream` during the timed region; queried only now)
     for k in range(Wm, Wm + K):
         pt = ck.phase_times(k)
         phase.append(pt)
         k1_ms.append(pt["leaf_hash"])
-    # per-phase breakdown (events between every kernel): a replay of the same lineage on a
-    # second handle, outside the timed region
-    ckp = Checkpointer(C)
-    ckp.set_profiling(2)
-    for k in range(Wm + K):
-        ckp.checkpoint(bufs[k], nbytes=B, stream=stream)
-    phase_full = [ckp.phase_times(k) for k in range(Wm, Wm + K)]
-    ckp.close()
     diffs.extend(r.as_dict() for r in raw)
-    torch.cuda.synchronize()
-    barrier(ws)
-    ms_local = ev0.elapsed_time(ev1)
-    ms = max_over_ranks(ms_local, ws)
-    total_bytes = sum_over_ranks(float(K * B), ws)
-    value = total_bytes / (ms / 1e3) / 1e9
+    steady = diffs[Wm:]
 
     # §8(e): all-gather per-rank 32-B records, file offsets (off the timed region)
     recs = [[int(d["bytes"]), int(d["meta_bytes"]), int(d["data_bytes"]), int(1e6 * pt["total"])]
-            for d, pt in zip(diffs[Wm:], phase)]
+            for d, pt in zip(steady, phase)]
     gathered = allgather_sizes(recs, ws)
     offsets = file_offsets(gathered)
 
     # roofline of the dominant kernel (K1): algorithmic bytes = B input + 16 n prev digests
     # + n/8 candidate bits + 16 per candidate digest write
-    steady = diffs[Wm:]
     cand = [d["n_first"] + d["n_spatial"] + d["n_temporal"] for d in steady]
     alg = [B + 16 * n + n / 8 + 16 * c for c in cand]
     k1_avg_ms = sum(k1_ms) / len(k1_ms)
@@ -344,16 +407,77 @@ def run_ours(args):
             traffic = json.load(f).get("leaf_hash_kernel", {}).get("dram_bytes_per_launch")
     except Exception:
         pass
+
+    # restore throughput (a8), reported separately: restore the newest checkpoint
+    # the first restore of a lineage builds and caches the per-diff restore plans (cold);
+    # the second is the steady restore cost (direct restore: each chunk written once)
+    last = lin.get(Wm + K - 1)
+    out = torch.empty(B, dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    r0 = time.perf_counter()
+    ck.restore(Wm + K - 1, out)
+    rs_cold = time.perf_counter() - r0
+    out.zero_()
+    torch.cuda.synchronize()
+    r0 = time.perf_counter()
+    ck.restore(Wm + K - 1, out)
+    rs = time.perf_counter() - r0
+    restore_ok = bool(torch.equal(out, last))
+
+    # per-phase breakdown (events between every kernel): a replay of the same lineage on a
+    # second handle, outside the timed region (resident lineages only)
+    if not inplace:
+        ckp = Checkpointer(C)
+        ckp.set_profiling(2)
+        for k in range(Wm + K):
+            ckp.checkpoint(lin.get(k), nbytes=B, stream=stream)
+        phase_full = [ckp.phase_times(k) for k in range(Wm, Wm + K)]
+        ckp.close()
+    else:
+        phase_full = [{"leaf_hash": pt["leaf_hash"], "total": pt["total"]} for pt in phase]
     phase_avg = {k: round(sum(pt[k] for pt in phase_full) / len(phase_full), 4) for k in phase_full[0]}
     phase_avg["total_timed"] = round(sum(pt["total"] for pt in phase) / len(phase), 4)
 
+    # restart (NEXT #3): rebuild the whole lineage on a fresh handle from host copies of the
+    # diffs (restore + re-de-duplication + byte check per diff), then check the newest restore
+    import_res = None
+    if not inplace:
+        host_diffs = [ck.diff_to_host(i) for i in range(Wm + K)]
+        ck3 = Checkpointer(C)
+        torch.cuda.synchronize()
+        i0 = time.perf_counter()
+        for hd in host_diffs:
+            ck3.import_diff(hd, stream=stream)
+        torch.cuda.synchronize()
+        imp_s = time.perf_counter() - i0
+        out.zero_()
+        ck3.restore(Wm + K - 1, out)
+        import_res = {"diffs": Wm + K, "s": round(imp_s, 4), "ok": bool(torch.equal(out, last)),
+                      "note": "ckpt_import of every diff from host memory into a fresh handle"}
+        ck3.close()
+        del host_diffs
+    check_first = ck.diff_to_host(Wm) if not inplace else None
+    check_last = ck.diff_to_host(Wm + K - 1) if not inplace else None
+    ck.close()
+    del out
+    if inplace:
+        del flush
+        torch.cuda.empty_cache()
+
     # e2e: same metric through the public host-memory call (H2D of the input from pinned
     # memory + de-dup + D2H of the diff), on a second handle replaying the same lineage
-    Ke = min(args.e2e_steps, K)
+    Ke = min(args.e2e_steps, K) if not inplace else 1
     ck2 = Checkpointer(C)
     for k in range(Wm):
-        ck2.checkpoint(bufs[k], stream=stream)
-    hosts = [bufs[Wm + i].cpu().pin_memory() for i in range(Ke)]
+        ck2.checkpoint(lin.get(k), nbytes=B, stream=stream)
+    hosts = []
+    for i in range(Ke):
+        h = torch.empty(B, dtype=torch.uint8, pin_memory=True)
+        h.copy_(lin.get(Wm + i))
+        hosts.append(h)
+    if inplace:
+        lin.release()
+        torch.cuda.empty_cache()
     hdiff = torch.empty(B + 64 + 12 * n + 16, dtype=torch.uint8).pin_memory()
     h2d = d2h = 0
     barrier(ws)
@@ -369,79 +493,57 @@ def run_ours(args):
     e2e_ms = max_over_ranks(e0.elapsed_time(e1), ws)
     e2e_val = sum_over_ranks(float(Ke * B), ws) / (e2e_ms / 1e3) / 1e9
     ck2.close()
-    del hosts
+    del hosts, hdiff
 
     # the paper's throughput ("the size of the original data divided by the time it
     # takes to create and copy the incremental checkpoint from the GPU to the host memory"),
     # with the one D2H per diff overlapped with the next de-duplication (NEXT #1):
     # device-resident inputs, ckpt_checkpoint on `stream`, ckpt_diff_to_host_async of the
     # finished diff on a second stream into pinned host memory; timed from the first
-    # checkpoint to the last D2H completed
-    ckq = Checkpointer(C)
-    for k in range(Wm):
-        ckq.checkpoint(bufs[k], nbytes=B, stream=stream)
-    sizes = [int(d["bytes"]) for d in diffs[Wm:]]   # same lineage -> same diffs as the timed run
-    offs = [0]
-    for sz in sizes:
-        offs.append(offs[-1] + ((sz + 4095) & ~4095))
-    hpipe = torch.empty(max(offs[-1], 1), dtype=torch.uint8).pin_memory()
-    d2h_stream = torch.cuda.Stream()
-    barrier(ws)
-    torch.cuda.synchronize()
-    q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    q0.record(stream)
-    for i, k in enumerate(range(Wm, Wm + K)):
-        dq = ckq.checkpoint(bufs[k], nbytes=B, stream=stream)   # returns with the diff complete
-        ckq.diff_to_host_async(k, hpipe[offs[i]:offs[i + 1]], d2h_stream, nbytes=dq["bytes"])
-    q1.record(d2h_stream)
-    d2h_stream.synchronize()
-    stream.synchronize()
-    pipe_ms = max_over_ranks(q0.elapsed_time(q1), ws)
-    pipe_val = sum_over_ranks(float(K * B), ws) / (pipe_ms / 1e3) / 1e9
-    pipe_ok = all(bytes(hpipe[offs[i]:offs[i] + sizes[i]].numpy()) == ck.diff_to_host(Wm + i) for i in (0, K - 1))
-    ckq.close()
-    del hpipe
-
-    # restore throughput (a8), reported separately: restore the newest checkpoint
-    # the first restore of a lineage builds and caches the per-diff restore plans (cold);
-    # the second is the steady restore cost (direct restore: each chunk written once)
-    out = torch.empty(B, dtype=torch.uint8, device="cuda")
-    r0 = time.perf_counter()
-    ck.restore(Wm + K - 1, out)
-    torch.cuda.synchronize()
-    rs_cold = time.perf_counter() - r0
-    out.zero_()
-    torch.cuda.synchronize()
-    r0 = time.perf_counter()
-    ck.restore(Wm + K - 1, out)
-    torch.cuda.synchronize()
-    rs = time.perf_counter() - r0
-    restore_ok = bool(torch.equal(out, bufs[Wm + K - 1]))
-
-    # restart (NEXT #3): rebuild the whole lineage on a fresh handle from host copies of the
-    # diffs (restore + re-de-duplication + byte check per diff), then check the newest restore
-    host_diffs = [ck.diff_to_host(i) for i in range(Wm + K)]
-    ck3 = Checkpointer(C)
-    torch.cuda.synchronize()
-    i0 = time.perf_counter()
-    for hd in host_diffs:
-        ck3.import_diff(hd, stream=stream)
-    torch.cuda.synchronize()
-    imp_s = time.perf_counter() - i0
-    out.zero_()
-    ck3.restore(Wm + K - 1, out)
-    import_ok = bool(torch.equal(out, bufs[Wm + K - 1]))
-    ck3.close()
-    del host_diffs
+    # checkpoint to the last D2H completed (resident lineages only)
+    paper = None
+    if not inplace:
+        ckq = Checkpointer(C)
+        for k in range(Wm):
+            ckq.checkpoint(lin.get(k), nbytes=B, stream=stream)
+        sizes = [int(d["bytes"]) for d in steady]   # same lineage -> same diffs as the timed run
+        offs = [0]
+        for sz in sizes:
+            offs.append(offs[-1] + ((sz + 4095) & ~4095))
+        hpipe = torch.empty(max(offs[-1], 1), dtype=torch.uint8).pin_memory()
+        d2h_stream = torch.cuda.Stream()
+        barrier(ws)
+        torch.cuda.synchronize()
+        q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        q0.record(stream)
+        for i, k in enumerate(range(Wm, Wm + K)):
+            dq = ckq.checkpoint(lin.get(k), nbytes=B, stream=stream)   # returns with the diff complete
+            ckq.diff_to_host_async(k, hpipe[offs[i]:offs[i + 1]], d2h_stream, nbytes=dq["bytes"])
+        q1.record(d2h_stream)
+        d2h_stream.synchronize()
+        stream.synchronize()
+        pipe_ms = max_over_ranks(q0.elapsed_time(q1), ws)
+        pipe_val = sum_over_ranks(float(K * B), ws) / (pipe_ms / 1e3) / 1e9
+        pipe_ok = (bytes(hpipe[offs[0]:offs[0] + sizes[0]].numpy()) == check_first and
+                   bytes(hpipe[offs[K - 1]:offs[K - 1] + sizes[K - 1]].numpy()) == check_last)
+        ckq.close()
+        del hpipe
+        paper = {"value": round(pipe_val, 3), "unit": "GB/s", "steps": K, "ok": pipe_ok,
+                 "d2h_bytes_per_step": sum(sizes) // max(1, K),
+                 "note": "P:196 create + D2H into pinned host memory, each diff's one D2H "
+                         "(ckpt_diff_to_host_async) overlapped with the next de-duplication"}
+    lin.release()
 
     cpu = None
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
+        nb = min(B, args.cpu_sample_bytes)
         try:
-            v, dt, nt = oracle_sample(cfg, args.cpu_sample_bytes, C, p, 3, seed)
-            cpu = {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                   "sample": f"config-{cfg} lineage at {args.cpu_sample_bytes >> 20} MiB (same recipe, smaller "
-                             f"buffer): checkpoint 0 untimed, {nt} steady checkpoints timed ({dt:.1f} s), "
-                             f"single-threaded C++ oracle"}
+            v, dt = oracle_lineage_timed(cfg, nb, C, p, 1, args.cpu_steps, seed)
+            cpu = {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", **cpu_info(),
+                   "sample": f"config-{cfg} lineage at {nb >> 20} MiB"
+                             + ("" if nb == B else f" (same recipe, of the {B >> 20} MiB workload)")
+                             + f": checkpoint 0 untimed, {args.cpu_steps} steady checkpoints timed ({dt:.1f} s), "
+                               f"single-threaded C++ oracle"}
         except Exception as e:  # pragma: no cover
             cpu = {"value": None, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": f"failed: {e}"}
 
@@ -451,11 +553,7 @@ def run_ours(args):
             "metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": ws,
             "steps": K, "warmup": Wm, "ms_per_step": round(ms / K, 4), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-            "config": {"workload": "config2: 1 GiB GDV-like buffer per GPU (73 x u32 rows), C = 128 B, "
-                                   f"row-run updates p = {p}" if B == GiB and cfg == 2 and C == 128 else
-                                   f"config{cfg} B={B} C={C} p={p}",
-                       "buffer_bytes": B, "chunk_bytes": C, "update_rate": p, "parallelism": f"independent x{ws}",
-                       "l2": "inputs (1 GiB per step, distinct buffers) larger than the 126 MB L2; no flush"},
+            "config": workload_config(args, ws, inplace),
             "per_gpu_gbs": round(value / ws, 3),
             "hbm_frac_of_measured": round((value / ws) * (1 + 16 / C) / peak, 4),
             "roofline": {"bound": "hbm", "kernel": "leaf_hash_kernel (K1)", "achieved": round(achieved, 1),
@@ -465,7 +563,9 @@ def run_ours(args):
                          "context": "K1 is a read stream: the read-only TMA ceiling measured on this box type by "
                                     "tools/bw_probe.cu is ~6.9-7.1 TB/s (profiles/bw_probe_r1.txt), above the copy peak"},
             "phase_ms": phase_avg,
-            "phase_ms_note": "per-phase split from an untimed replay with events between kernels; total_timed = timed-run first-to-last-kernel span",
+            "phase_ms_note": ("per-phase split from an untimed replay with events between kernels; total_timed = "
+                              "timed-run first-to-last-kernel span" if not inplace else
+                              "K1 and whole-call events of the timed steps (no per-phase replay in place)"),
             "diff_ratio": round(ratio, 2),
             "meta_over_diff": round(sum(d["meta_bytes"] for d in steady) / max(1, sum(d["bytes"] for d in steady)), 4),
             "compaction_vs_list": round(sum(d["list_entries"] for d in steady) /
@@ -475,29 +575,68 @@ def run_ours(args):
             "restore": {"id": Wm + K - 1, "s": round(rs, 5), "gbs": round(B / rs / 1e9, 2), "ok": restore_ok,
                         "cold_s": round(rs_cold, 5), "note": "host wall time of ckpt_restore (synchronous); cold = "
                                                              "first restore, which builds the per-diff plans"},
-            "restart_import": {"diffs": Wm + K, "s": round(imp_s, 4), "ok": import_ok,
-                               "note": "ckpt_import of every diff from host memory into a fresh handle"},
+            "restart_import": import_res,
             "file_offsets_rank0": offsets[0][:3],
             "e2e": {"value": round(e2e_val, 3), "unit": "GB/s", "h2d_bytes_per_step": h2d // max(1, Ke),
                     "d2h_bytes_per_step": d2h // max(1, Ke), "steps": Ke},
-            "paper_throughput": {"value": round(pipe_val, 3), "unit": "GB/s", "steps": K, "ok": pipe_ok,
-                                 "d2h_bytes_per_step": sum(sizes) // max(1, K),
-                                 "note": "P:196 create + D2H into pinned host memory, each diff's one D2H "
-                                         "(ckpt_diff_to_host_async) overlapped with the next de-duplication"},
+            "paper_throughput": paper,
             "cpu_baseline": cpu,
             "gpu_launches": launches,
             "clocks": clk.summary(),
         }
         print(json.dumps(line), flush=True)
-    ck.close()
     if ws > 1:
         import torch.distributed as dist
         dist.destroy_process_group()
     return 0
 
 
+# ------------------------------------------------------------------ multi-process plumbing
+def free_port():
+    import socket
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def self_launch(argv, n):
+    """`bench.py --gpus N` without torchrun's environment: re-run this command under
+    torch.distributed.run, one process per GPU (rendezvous on 127.0.0.1)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + argv
+    return subprocess.call(cmd)
+
+
+def run_dist_selftest(args):
+    """The multi-rank plumbing of run_ours without a GPU (gloo): rendezvous, barrier,
+    max / sum over ranks, the all-gather of the 32-B records and the file offsets. Each rank
+    fakes its step time; rank 0 prints one line in the bench format."""
+    import torch.distributed as dist
+    ws, rank = int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0"))
+    if ws > 1:
+        dist.init_process_group("gloo")
+    assert ws == args.gpus, (ws, args.gpus)
+    barrier(ws)
+    ms = max_over_ranks(10.0 + rank, ws)
+    tot = sum_over_ranks(float(args.steps * args.bytes), ws)
+    recs = [[1000 * (rank + 1) + k, 64, 1000 * (rank + 1) + k - 64, 10 + rank] for k in range(args.steps)]
+    offs = file_offsets(allgather_sizes(recs, ws))
+    if rank == 0:
+        print(json.dumps({"metric": METRIC, "value": tot / (ms / 1e3) / 1e9, "n_gpus": ws, "ms": ms,
+                          "file_offsets": [o[0] for o in offs], "selftest": True}), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+    return 0
+
+
 def main():
     args = parse()
+    if args.bytes is None:
+        args.bytes = (16 * GiB) if args.config == 5 else GiB
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        return self_launch(sys.argv[1:], args.gpus)
+    if args.dist_selftest:
+        return run_dist_selftest(args)
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

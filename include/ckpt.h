@@ -43,8 +43,10 @@ enum {
   CKPT_ECUDA = 3,  /* CUDA runtime/driver error; the handle is now poisoned            */
   CKPT_ERANGE = 4, /* checkpoint id out of range                                       */
   CKPT_ESTATE = 5, /* handle poisoned by an earlier CUDA error                          */
-  CKPT_ECOLLIDE = 6 /* a 128-bit digest collision was detected (R14: out of scope; the
-                       checkpoint is committed but its phase-2 record insert was skipped) */
+  CKPT_ECOLLIDE = 6 /* a 128-bit digest collision was detected (R14: out of scope). A WARNING,
+                       not a failure: the checkpoint IS committed (diff filled, id advanced),
+                       only the colliding phase-2 record insert was skipped. The one status
+                       after which the lineage has changed. */
 };
 
 /* Statistics and location of one consolidated difference. */
@@ -139,8 +141,10 @@ CKPT_API int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_per
  *   diff     receives the statistics and the device pointer of the new diff.
  * The call returns after exactly one host synchronisation with `stream` (a spin on the
  * completion the last kernel publishes to mapped host memory; the process
- * "stops during checkpointing"). Capacity for the record table and the diff is
- * reserved before the first kernel, so an error leaves the lineage unchanged.
+ * "stops during checkpointing"); a call that grows the record table does so in
+ * stream order on `stream` and still synchronises once (ckpt_host_syncs). Capacity for the
+ * record table and the diff is reserved before the first kernel, so an error leaves the
+ * lineage unchanged (CKPT_ECOLLIDE is a committed checkpoint, see above).
  * Errors: CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ESTATE, CKPT_ECOLLIDE. */
 CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff);
 
@@ -154,9 +158,17 @@ CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes,
  * 2-3x the diff's metadata plus 12 bytes per chunk the diff covers, in device memory; the
  * handle also keeps 8 bytes per chunk of the buffer for the claims.
  *   dev_ptr  device buffer of B bytes, 16-byte aligned, owned by the caller; overwritten.
- * Synchronous (runs on an internal stream of the handle).
+ * Synchronous. Runs on an internal stream of the handle that is a BLOCKING stream: work
+ * enqueued earlier on the legacy default stream (and on other blocking streams) completes
+ * before the restore touches dev_ptr; work on non-blocking streams is NOT ordered — use
+ * ckpt_restore_stream for those.
  * Errors: CKPT_ERANGE (id >= number of checkpoints), CKPT_EINVAL, CKPT_ECUDA, CKPT_ESTATE. */
 CKPT_API int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr);
+
+/* ckpt_restore with every kernel enqueued on `stream` (cudaStream_t as void*), in order
+ * after the caller's earlier work there; returns after synchronising `stream`. The plan
+ * building of a diff's first restore runs on `stream` too.  Errors as ckpt_restore. */
+CKPT_API int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream);
 
 /* Statistics / device pointer of an earlier diff.  Errors: CKPT_ERANGE, CKPT_EINVAL. */
 CKPT_API int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff);
@@ -231,6 +243,13 @@ CKPT_API int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n
  * calls built on them), counted at the launch sites; bench.py reports the difference over
  * its timed region. */
 CKPT_API int ckpt_kernel_launches(ckpt_handle h, uint64_t* count);
+
+/* Number of times this handle has blocked the host on the device so far (stream
+ * synchronisations and the completion spin of ckpt_checkpoint), counted at the wait sites.
+ * ckpt_checkpoint adds exactly one, including a call that grows the record table (the
+ * growth is stream-ordered: allocation, rehash and release of the old table run on the
+ * caller's stream).  Errors: CKPT_EINVAL. */
+CKPT_API int ckpt_host_syncs(ckpt_handle h, uint64_t* count);
 
 /* Release all device memory of the handle (record, leaf digests, every diff). */
 CKPT_API int ckpt_destroy(ckpt_handle h);

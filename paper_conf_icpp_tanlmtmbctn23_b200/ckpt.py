@@ -23,10 +23,11 @@ CKPT_VARIANT_FULL_FIRST, CKPT_VARIANT_FULL_SWITCH = 1, 2      # Tree variants (P
 CKPT_FLAGS_FULL = 3                                           # header flags of a full difference
 
 ABI_FUNCTIONS = [
-    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore", "ckpt_diff_info", "ckpt_diff_to_host", "ckpt_diff_to_host_async",
+    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore",
+    "ckpt_restore_stream", "ckpt_diff_info", "ckpt_diff_to_host", "ckpt_diff_to_host_async",
     "ckpt_checkpoint_host", "ckpt_import", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
-    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches", "ckpt_destroy",
-    "ckpt_strerror",
+    "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches",
+    "ckpt_host_syncs", "ckpt_destroy", "ckpt_strerror",
 ]
 
 
@@ -82,6 +83,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_set_variant": ([vp, u32, u32], i32),
             "ckpt_checkpoint": ([vp, vp, u64, vp, P(CkptDiff)], i32),
             "ckpt_restore": ([vp, u32, vp], i32),
+            "ckpt_restore_stream": ([vp, u32, vp, vp], i32),
             "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
             "ckpt_diff_to_host": ([vp, u32, vp, u64], i32),
             "ckpt_diff_to_host_async": ([vp, u32, vp, u64, vp], i32),
@@ -94,6 +96,7 @@ def lib() -> ctypes.CDLL:
             "ckpt_phase_times": ([vp, P(ctypes.c_float), i32], i32),
             "ckpt_phase_times_of": ([vp, u32, P(ctypes.c_float), i32], i32),
             "ckpt_kernel_launches": ([vp, P(ctypes.c_uint64)], i32),
+            "ckpt_host_syncs": ([vp, P(ctypes.c_uint64)], i32),
             "ckpt_destroy": ([vp], i32),
             "ckpt_strerror": ([i32], ctypes.c_char_p),
         }
@@ -166,8 +169,22 @@ class Checkpointer:
         n = _nbytes(buf) if nbytes is None else nbytes
         rc = self._ckpt_fn(self._h, _ptr(buf), n, _stream_handle(stream), ctypes.byref(d))
         if rc != CKPT_OK:
+            if rc == CKPT_ECOLLIDE:   # committed with a warning (include/ckpt.h, R14)
+                return self._collided(d, raw)
             raise CkptError(rc, "ckpt_checkpoint")
         return d if raw else d.as_dict()
+
+    @staticmethod
+    def _collided(d, raw):
+        import warnings
+        warnings.warn(f"ckpt_checkpoint: 128-bit digest collision in checkpoint {d.id} (R14); "
+                      "the checkpoint is committed, its colliding record insert was skipped",
+                      RuntimeWarning, stacklevel=3)
+        if raw:
+            return d
+        out = d.as_dict()
+        out["collision"] = True
+        return out
 
     def checkpoint_host(self, host_buf, host_diff=None, nbytes: int | None = None, stream=None):
         d = CkptDiff()
@@ -176,6 +193,8 @@ class Checkpointer:
         rc = lib().ckpt_checkpoint_host(self._h, _ptr(host_buf), n, _stream_handle(stream),
                                         _ptr(host_diff) if host_diff is not None else None, cap, ctypes.byref(d))
         if rc != CKPT_OK:
+            if rc == CKPT_ECOLLIDE:
+                return self._collided(d, False)
             raise CkptError(rc, "ckpt_checkpoint_host")
         return d.as_dict()
 
@@ -191,10 +210,12 @@ class Checkpointer:
         if rc != CKPT_OK:
             raise CkptError(rc, "ckpt_import")
 
-    def restore(self, cid: int, out) -> None:
-        rc = lib().ckpt_restore(self._h, cid, _ptr(out))
+    def restore(self, cid: int, out, stream=None) -> None:
+        """Rebuild checkpoint cid into device tensor `out`, ordered after the work already
+        enqueued on `stream` (default: torch's current stream); synchronous."""
+        rc = lib().ckpt_restore_stream(self._h, cid, _ptr(out), _stream_handle(stream))
         if rc != CKPT_OK:
-            raise CkptError(rc, "ckpt_restore")
+            raise CkptError(rc, "ckpt_restore_stream")
 
     def diff_info(self, cid: int) -> dict:
         d = CkptDiff()
@@ -303,6 +324,13 @@ class Checkpointer:
             if rc != CKPT_OK:
                 raise CkptError(rc, "ckpt_phase_times_of")
         return {self.PHASES[i]: t[i] for i in range(10)}
+
+    @property
+    def host_syncs(self) -> int:
+        """Host waits on the device this handle has performed so far (ckpt_host_syncs)."""
+        c = ctypes.c_uint64()
+        lib().ckpt_host_syncs(self._h, ctypes.byref(c))
+        return c.value
 
     @property
     def kernel_launches(self) -> int:

@@ -10,6 +10,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -118,6 +119,7 @@ struct ckpt_ctx {
   uint64_t rs_chain_cap = 0;
   cudaStream_t internal = nullptr;
   uint64_t launches = 0;         // kernels this handle has enqueued (all calls)
+  uint64_t host_syncs = 0;       // host waits on the device this handle has performed (all calls)
   int prof = 0;                  // 0 off, 1 K1 + whole call, 2 every phase
   // per-checkpoint event sets (ring), queried lazily so the call itself never waits on them
   static constexpr int kEvRing = 256;
@@ -147,6 +149,13 @@ struct ckpt_ctx {
 
 namespace {
 
+// Every place the library blocks the host on the device goes through here (counted: the
+// one-synchronisation contract of ckpt_checkpoint is tested with ckpt_host_syncs).
+cudaError_t sync_stream(ckpt_ctx* h, cudaStream_t st) {
+  ++h->host_syncs;
+  return cudaStreamSynchronize(st);
+}
+
 template <class T>
 cudaError_t dalloc(ckpt_ctx* h, T** p, size_t count) {
   void* q = nullptr;
@@ -163,7 +172,9 @@ int ceil_log2(uint64_t n) {
   return h;
 }
 
-int setup_geometry(ckpt_ctx* h, uint64_t B) {
+// Per-geometry state, allocated by the first checkpoint (or import) of a handle. The
+// counter blocks are zeroed on `st`, the stream the call's kernels then run on.
+int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
   h->B = B;
   h->n = (B + h->C - 1) / h->C;
   h->h = ceil_log2(h->n);
@@ -230,7 +241,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
     }
     AL(h->ctr2[0], bytes);
     AL(h->ctr2[1], bytes);
-    if (cudaMemset(h->ctr2[0], 0, bytes) != cudaSuccess || cudaMemset(h->ctr2[1], 0, bytes) != cudaSuccess)
+    if (cudaMemsetAsync(h->ctr2[0], 0, bytes, st) != cudaSuccess || cudaMemsetAsync(h->ctr2[1], 0, bytes, st) != cudaSuccess)
       return CKPT_ECUDA;
     h->ctr_bytes = bytes;
     h->ctr_dbits_off = dbits_off;
@@ -245,7 +256,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B) {
   AL(h->lmask, n_tiles * kLmWords);
   AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
 #undef AL
-  if (cudaMemset(h->tilecnt, 0, n_tiles * sizeof(uint4)) != cudaSuccess) return CKPT_ECUDA;
+  if (cudaMemsetAsync(h->tilecnt, 0, n_tiles * sizeof(uint4), st) != cudaSuccess) return CKPT_ECUDA;
   if (h->trace_path) {
     if (dalloc(h, &h->trace, (uint64_t)kTraceLanes * kTraceLaneCap) != cudaSuccess ||
         dalloc(h, &h->trace_n, 8 * kTraceLanes) != cudaSuccess)
@@ -279,16 +290,18 @@ int ensure_table(ckpt_ctx* h, cudaStream_t st) {
   uint64_t new_cap = (uint64_t)((double)need / kGrowLoad) + 1;
   if (new_cap < 4096) new_cap = 4096;
   if (new_cap >= (1ull << 32)) return CKPT_ENOMEM;   // slot ids are u32
+  // Stream-ordered growth (no host synchronisation, ckpt.h: one sync per call): the new
+  // table is allocated, filled and rehashed on the caller's stream, and the old one is
+  // freed in stream order behind the rehash that reads it.
   Slot* nt = nullptr;
-  if (cudaMalloc(&nt, new_cap * sizeof(Slot)) != cudaSuccess) {
+  if (cudaMallocAsync(reinterpret_cast<void**>(&nt), new_cap * sizeof(Slot), st) != cudaSuccess) {
     cudaGetLastError();
     return CKPT_ENOMEM;
   }
   if (cudaMemsetAsync(nt, 0xFF, new_cap * sizeof(Slot), st) != cudaSuccess) return CKPT_ECUDA;
   if (h->tab) {
     if (launch_rehash(h->tab, h->cap, nt, new_cap, st) != cudaSuccess) return CKPT_ECUDA;
-    if (cudaStreamSynchronize(st) != cudaSuccess) return CKPT_ECUDA;
-    cudaFree(h->tab);
+    if (cudaFreeAsync(h->tab, st) != cudaSuccess) return CKPT_ECUDA;
   }
   h->tab = nt;
   h->cap = new_cap;
@@ -338,6 +351,84 @@ void fill_diff(const ckpt_ctx* h, uint32_t id, const Totals& t, uint8_t* ptr, ck
   d->record_size = h->live;
   d->record_capacity = h->cap;
   d->phase2_inserts = t.p2_inserts;
+}
+
+// ---- host twins of dev.cuh's tree geometry (R3), used only to validate imported diffs
+// before any kernel reads them (ckpt_import: a corrupted body must not steer device writes)
+struct HostGeo {
+  uint64_t B, n, m;
+  uint32_t C;
+  int h;
+};
+
+uint64_t hg_chunk_of_vslot(const HostGeo& g, uint64_t v) { return v <= g.m ? v : g.m + (v - g.m) / 2; }
+
+// chunk range [lo, hi) of heap node `node`; false if the id names no node of the tree
+bool hg_node_range(const HostGeo& g, uint64_t node, uint64_t& lo, uint64_t& hi) {
+  if (node >= 2 * g.n - 1) return false;
+  const int depth = 63 - __builtin_clzll(node + 1);
+  if (depth > g.h) return false;
+  const int L = g.h - depth;
+  const uint64_t j = node + 1 - (1ull << depth);
+  lo = hg_chunk_of_vslot(g, j << L);
+  hi = hg_chunk_of_vslot(g, (j + 1) << L);
+  return lo < hi;
+}
+
+uint64_t hg_range_bytes(const HostGeo& g, uint64_t lo, uint64_t hi) {
+  const uint64_t e = std::min<uint64_t>(hi * g.C, g.B);
+  return e - lo * g.C;
+}
+
+// The body of a diff to import: every node id names a tree node; FIRST and
+// SHIFT regions are sorted by first chunk and pairwise disjoint; a SHIFT source checkpoint is
+// <= id and its source node covers as many bytes as the region; the FIRST regions' bytes
+// sum to data_bytes. Basic: the bitmap's popcount is nF, no bit at or past n, and the
+// changed chunks' bytes sum to data_bytes. Full form: the root alone, the whole buffer.
+bool validate_import_body(const HostGeo& g, const uint8_t* hd, uint32_t id, int mode, bool full, uint64_t nF,
+                          uint64_t nS, uint64_t data) {
+  auto rd32 = [&](uint64_t o) { uint32_t v; std::memcpy(&v, hd + o, 4); return v; };
+  if (mode == kModeBasic) {
+    const uint64_t words = (g.n + 31) / 32;
+    uint64_t cnt = 0;
+    bool last_set = false;
+    for (uint64_t w = 0; w < words; ++w) {
+      uint32_t x = rd32(64 + 4 * w);
+      if (w + 1 == words && (g.n & 31)) {
+        if (x >> (g.n & 31)) return false;   // bits past n
+      }
+      if (w + 1 == words) last_set = (x >> ((g.n - 1) & 31)) & 1u;
+      cnt += __builtin_popcount(x);
+    }
+    if (cnt != nF) return false;
+    const uint64_t bytes = nF * g.C - (last_set ? g.n * g.C - g.B : 0);
+    return bytes == data;
+  }
+  if (full) return nF == 1 && nS == 0 && rd32(64) == 0 && data == g.B;
+  uint64_t sum = 0, prev_hi = 0;
+  std::vector<std::pair<uint64_t, uint64_t>> fr;
+  fr.reserve(nF);
+  for (uint64_t i = 0; i < nF; ++i) {
+    uint64_t lo, hi;
+    if (!hg_node_range(g, rd32(64 + 4 * i), lo, hi) || lo < prev_hi) return false;
+    prev_hi = hi;
+    sum += hg_range_bytes(g, lo, hi);
+    fr.emplace_back(lo, hi);
+  }
+  if (sum != data) return false;
+  prev_hi = 0;
+  uint64_t f = 0;   // FIRST regions before the current SHIFT region (disjointness by merge)
+  for (uint64_t i = 0; i < nS; ++i) {
+    const uint64_t e = 64 + 4 * nF + 12 * i;
+    uint64_t lo, hi, vlo, vhi;
+    if (!hg_node_range(g, rd32(e), lo, hi) || lo < prev_hi) return false;
+    if (!hg_node_range(g, rd32(e + 4), vlo, vhi) || rd32(e + 8) > id) return false;
+    if (hg_range_bytes(g, lo, hi) != hg_range_bytes(g, vlo, vhi)) return false;
+    while (f < fr.size() && fr[f].second <= lo) ++f;
+    if (f < fr.size() && fr[f].first < hi) return false;   // overlaps a FIRST region
+    prev_hi = hi;
+  }
+  return true;
 }
 
 }  // namespace
@@ -394,7 +485,10 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
     delete h;
     return CKPT_ECUDA;
   }
-  if (cudaStreamCreateWithFlags(&h->internal, cudaStreamNonBlocking) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  // The internal stream is a BLOCKING stream: work the caller enqueued earlier on the legacy
+  // default stream (torch's default) completes before ckpt_restore / ckpt_import /
+  // ckpt_leaf_digests touch memory on it (ckpt.h ordering contract).
+  if (cudaStreamCreateWithFlags(&h->internal, cudaStreamDefault) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaHostAlloc(&h->tot_host, sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   std::memset(h->tot_host, 0, sizeof(Totals));   // done = 0: no call completed yet (epochs start at 1)
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
@@ -436,6 +530,12 @@ int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count) {
 int ckpt_kernel_launches(ckpt_handle h, uint64_t* count) {
   if (!h || !count) return CKPT_EINVAL;
   *count = h->launches;
+  return CKPT_OK;
+}
+
+int ckpt_host_syncs(ckpt_handle h, uint64_t* count) {
+  if (!h || !count) return CKPT_EINVAL;
+  *count = h->host_syncs;
   return CKPT_OK;
 }
 
@@ -527,7 +627,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (!h->geo_set) {
-    const int r = setup_geometry(h, bytes);
+    const int r = setup_geometry(h, bytes, st);
     if (r != CKPT_OK) return r;
   }
   const uint32_t k = (uint32_t)h->diffs.size();
@@ -683,6 +783,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   // cudaStreamSynchronize). The stream is queried now and then, so a failed kernel (which
   // never publishes) surfaces as an error instead of a hang.
   {
+    ++h->host_syncs;
     volatile uint32_t* done = &h->tot_host->done;
     for (uint32_t it = 1;; ++it) {
       if (*done == g.epoch) break;
@@ -699,6 +800,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     }
   }
 
+  std::atomic_thread_fence(std::memory_order_acquire);   // the totals after the epoch
   const auto t_synced = clk::now();
 
   const Totals t = *h->tot_host;   // written by the gather kernel (mapped host memory)
@@ -746,7 +848,7 @@ int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capac
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
   CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, h->internal));   // one D2H
-  CK(cudaStreamSynchronize(h->internal));
+  CK(sync_stream(h, h->internal));
   return CKPT_OK;
 }
 
@@ -779,7 +881,7 @@ int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, vo
   if (host_diff) {
     if (host_diff_cap < diff->bytes) return CKPT_EINVAL;
     CK(cudaMemcpyAsync(host_diff, diff->dev_ptr, diff->bytes, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
+    CK(sync_stream(h, st));
   }
   return CKPT_OK;
 }
@@ -827,6 +929,7 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
   for (uint32_t c = 0; c <= id; ++c) {
     DiffRec& d = h->diffs[c];
     RestoreDiff& r = rd[c];
+    r.id = c;
     r.base = d.ptr;
     r.nF = d.info.n_first_regions;
     r.nS = d.info.n_shift_regions;
@@ -865,7 +968,7 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
       return CKPT_ECUDA;
   int herr = 0;
   if (cudaMemcpyAsync(&herr, h->rs_err, sizeof(int), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-      cudaStreamSynchronize(st) != cudaSuccess)
+      sync_stream(h, st) != cudaSuccess)
     return CKPT_ECUDA;
   if (herr) return CKPT_EINVAL;   // malformed chain (a source outside any FIRST region)
   for (uint32_t c = 0; c <= id; ++c) {
@@ -890,7 +993,7 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     rd[c].Csrc = d.Csrc;
     if (restore_claimlist(g, rd[c], h->num_sms, st) != cudaSuccess) return CKPT_ECUDA;
   }
-  if (cudaStreamSynchronize(st) != cudaSuccess) return CKPT_ECUDA;
+  if (sync_stream(h, st) != cudaSuccess) return CKPT_ECUDA;
   for (uint32_t c = 0; c <= id; ++c) h->diffs[c].planned = true;
   return CKPT_OK;
 }
@@ -924,8 +1027,17 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
   const uint64_t raw = h->mode == kModeBasic ? 64 + 4 * ((n + 31) / 32) : 64 + 4 * nF + 12 * nS;
   const uint64_t meta = (raw + 15) & ~15ull;
   if (meta + data != bytes || data > B || (h->mode == kModeBasic && nS)) return CKPT_EINVAL;
+  {
+    HostGeo hg;
+    hg.B = B;
+    hg.n = n;
+    hg.C = h->C;
+    hg.h = ceil_log2(n);
+    hg.m = 2 * n - (1ull << hg.h);
+    if (!validate_import_body(hg, hd, id, h->mode, flags == CKPT_FLAGS_FULL, nF, nS, data)) return CKPT_EINVAL;
+  }
   if (!h->geo_set) {
-    const int r = setup_geometry(h, B);
+    const int r = setup_geometry(h, B, h->internal);
     if (r != CKPT_OK) return r;
   }
   if (h->staging_size < B) {
@@ -945,7 +1057,7 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
   auto cleanup = [&]() { cudaFree(tmp); cudaFree(flag); };
   cudaStream_t in = h->internal;
   if (cudaMemcpyAsync(tmp, host_diff, bytes, cudaMemcpyHostToDevice, in) != cudaSuccess ||
-      cudaStreamSynchronize(in) != cudaSuccess) {
+      sync_stream(h, in) != cudaSuccess) {
     cleanup();
     h->poisoned = true;
     return CKPT_ECUDA;
@@ -976,7 +1088,7 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
     if (cudaMemsetAsync(flag, 0, sizeof(int), in) != cudaSuccess ||
         device_compare(d.dev_ptr, tmp, bytes, flag, h->num_sms, in) != cudaSuccess ||
         cudaMemcpyAsync(&hf, flag, sizeof(int), cudaMemcpyDeviceToHost, in) != cudaSuccess ||
-        cudaStreamSynchronize(in) != cudaSuccess) {
+        sync_stream(h, in) != cudaSuccess) {
       cleanup();
       h->poisoned = true;
       return CKPT_ECUDA;
@@ -992,11 +1104,16 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
 }
 
 int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
+  if (!h) return CKPT_EINVAL;
+  return ckpt_restore_stream(h, id, dev_ptr, h->internal);
+}
+
+int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream) {
   if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   LaunchCount lc(h);
-  cudaStream_t st = h->internal;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
   const Geo g = make_geo(h, id);
   int rc = ensure_plans(h, id, g, st);
   if (rc != CKPT_OK) {
@@ -1011,6 +1128,7 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
   for (int64_t c = id; c >= 0; --c) {
     const DiffRec& d = h->diffs[c];
     RestoreDiff r;
+    r.id = (uint32_t)c;
     r.base = d.ptr;
     r.nF = d.info.n_first_regions;
     r.nS = d.info.n_shift_regions;
@@ -1022,7 +1140,7 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
     CK(restore_claim(g, r, h->owner, h->num_sms, st));
   }
   CK(restore_copy(g, h->owner, outp, h->num_sms, st));
-  CK(cudaStreamSynchronize(st));
+  CK(sync_stream(h, st));
   return CKPT_OK;
 }
 
@@ -1031,7 +1149,7 @@ int ckpt_leaf_digests(ckpt_handle h, void* dev_out) {
   if (h->poisoned) return CKPT_ESTATE;
   if (!h->geo_set) return CKPT_ERANGE;
   CK(cudaMemcpyAsync(dev_out, h->prev, h->n * 16, cudaMemcpyDeviceToDevice, h->internal));
-  CK(cudaStreamSynchronize(h->internal));
+  CK(sync_stream(h, h->internal));
   return CKPT_OK;
 }
 
@@ -1043,7 +1161,7 @@ int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_nodes, ui
   if (!h->tab || cap == 0) return CKPT_OK;
   std::vector<Slot> all(h->cap);
   CK(cudaMemcpyAsync(all.data(), h->tab, h->cap * sizeof(Slot), cudaMemcpyDeviceToHost, h->internal));
-  CK(cudaStreamSynchronize(h->internal));
+  CK(sync_stream(h, h->internal));
   uint64_t i = 0;
   for (const Slot& s : all) {
     if (s.klo == kEmpty && s.khi == kEmpty) continue;

@@ -30,8 +30,10 @@ __device__ __forceinline__ void warp_sum3(unsigned long long& a, unsigned long l
 constexpr int kCT = 256;
 
 // Every counter the host reports is final once the gather kernel runs (tree kernels done,
-// pdl_wait): block 0 copies them to mapped host memory early, in 16-byte stores, so the
-// PCIe writes are long done when the last block publishes the epoch.
+// pdl_wait): block 0 copies them to mapped host memory early, in 16-byte stores, and
+// orders them at system scope right away (one fence, one thread), so they are visible to
+// the host before the epoch the last block publishes (which is ordered after block 0's
+// arrival on the completion counter).
 __device__ __forceinline__ void host_totals(const CompactParams& p) {
   static_assert(offsetof(Totals, done) % 4 == 0, "Totals layout");
   const uint4* src = reinterpret_cast<const uint4*>(p.tot);
@@ -41,6 +43,7 @@ __device__ __forceinline__ void host_totals(const CompactParams& p) {
   const uint32_t* s32 = reinterpret_cast<const uint32_t*>(p.tot);
   uint32_t* d32 = reinterpret_cast<uint32_t*>(p.tot_host);
   for (uint32_t w = nv * 4; w < (uint32_t)(offsetof(Totals, done) / 4); ++w) d32[w] = __ldcg(s32 + w);
+  __threadfence_system();
 }
 
 // KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata

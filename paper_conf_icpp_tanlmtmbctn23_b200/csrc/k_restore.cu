@@ -130,13 +130,13 @@ __global__ void __launch_bounds__(kRT) claimlist_kernel(Geo g, RestoreDiff d) {
 // claim_kernel (one launch per diff, newest first): the chunk's first claimer (the newest
 // diff covering it) records the address of its bytes in owner[chunk]. Regions of one diff
 // are disjoint, so a diff never races with itself; diffs run in stream order.
-__global__ void __launch_bounds__(kRT) claim_kernel(RestoreDiff d, uint64_t ncl, unsigned long long* owner) {
+__global__ void __launch_bounds__(kRT) claim_kernel(RestoreDiff d, uint64_t ncl, uint64_t n, unsigned long long* owner) {
   pdl_launch_dependents();
   pdl_wait();   // the newer diffs' claims are complete
   for (uint64_t t = (uint64_t)blockIdx.x * kRT + threadIdx.x; t < ncl; t += (uint64_t)gridDim.x * kRT) {
     const uint32_t ch = __ldg(d.Cch + t);
     const unsigned long long src = __ldg(d.Csrc + t);
-    if (__ldcg(owner + ch) == 0) owner[ch] = src;
+    if (ch < n && __ldcg(owner + ch) == 0) owner[ch] = src;   // ch < n: guard against malformed plans
   }
 }
 
@@ -209,6 +209,10 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
   node_range(g, v, vlo, vhi);
   len[i] = range_bytes(g, ulo, uhi);
   d.Slo[i] = ulo;
+  // guards (malformed diffs, e.g. a corrupted import): the source checkpoint is in the chain
+  // and the source bytes lie inside one FIRST region of its data section; otherwise the
+  // plan is flagged and no restore kernel runs
+  if (c2 > d.id) { atomicExch(err, 1); d.Ssrc[i] = (unsigned long long)d.base; return; }
   const RestoreDiff& s = chain[c2];
   // FIRST region r of diff c2 with Flo[r] <= vlo (the last such): it contains v
   if (s.nF == 0 || !s.Flo) { atomicExch(err, 1); d.Ssrc[i] = (unsigned long long)s.base; return; }
@@ -217,7 +221,14 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
     const uint64_t mid = (lo + hi) >> 1;
     if (s.Flo[mid] <= vlo) lo = mid; else hi = mid;
   }
-  d.Ssrc[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + (vlo - s.Flo[lo]) * (unsigned long long)g.C);
+  const unsigned long long rel = (vlo - s.Flo[lo]) * (unsigned long long)g.C;
+  const unsigned long long rend = lo + 1 < s.nF ? s.Foff[lo + 1] : s.data_bytes;
+  if (s.Flo[lo] > vlo || s.Foff[lo] + rel + range_bytes(g, vlo, vhi) > rend) {
+    atomicExch(err, 1);
+    d.Ssrc[i] = (unsigned long long)s.base;
+    return;
+  }
+  d.Ssrc[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + rel);
 }
 
 // Basic diffs: every changed chunk is a one-chunk "FIRST region" of the plan.
@@ -231,7 +242,7 @@ __global__ void basic_expand_kernel(Geo g, RestoreDiff d, uint64_t nwords, const
   if (w >= nwords) return;
   uint32_t m = rd32(d.base + 64 + 4 * w);
   unsigned long long r = off[w];
-  for (; m; m &= m - 1, ++r) {
+  for (; m && r < d.nF; m &= m - 1, ++r) {   // r < nF: a malformed bitmap cannot overrun
     d.Flo[r] = 32ull * w + (__ffs(m) - 1);
     d.Foff[r] = r * (unsigned long long)g.C;   // only the buffer's last chunk can be short
   }
@@ -372,7 +383,7 @@ cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long
   uint64_t grid = (nx + kRT - 1) / kRT;
   const uint64_t cap = (uint64_t)num_sms * (g_claim_bps > 0 ? g_claim_bps : 4);
   if (grid > cap) grid = cap;
-  return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, d, nx, owner);
+  return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, d, nx, (uint64_t)g.n, owner);
 }
 
 cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st) {

@@ -219,6 +219,7 @@ cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
 
 // ---- restore (k_restore.cu)
 struct RestoreDiff {           // one diff of the chain, as the restore kernels see it (cached plan)
+  uint32_t id;                 // its checkpoint id (a SHIFT source must be <= id)
   const uint8_t* base;         // diff bytes (device)
   uint64_t nF, nS, meta_bytes, data_bytes;
   unsigned long long* Flo;     // per FIRST region: first chunk (sorted)

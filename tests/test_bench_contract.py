@@ -43,3 +43,17 @@ def test_our_arm_line_small():
     assert d["gpu_launches"] > 0
     assert d["restore"]["ok"] and d["restart_import"]["ok"] and d["paper_throughput"]["ok"]
     assert set(d["clocks"]) >= {"sm_mhz", "sm_max_mhz", "reasons"}
+
+
+@pytest.mark.gpu
+def test_our_arm_inplace_config5_form():
+    """The in-place form bench.py uses for config 5 (16 GiB per GPU: the lineage does not fit
+    in HBM), at a small size: one buffer mutated between steps outside the timed events."""
+    d = _run(["--config", "5", "--bytes", str(64 << 20), "--inplace", "--steps", "3", "--warmup", "3",
+              "--no-cpu-baseline"])
+    assert BASE_KEYS <= set(d)
+    assert d["value"] > 0 and d["n_gpus"] == 1 and d["config"]["buffer_bytes"] == 64 << 20
+    assert "in place" in d["config"]["l2"]
+    assert d["restore"]["ok"] and d["paper_throughput"] is None and d["restart_import"] is None
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 64 << 20
+    assert d["gpu_launches"] > 0

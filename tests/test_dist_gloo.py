@@ -53,3 +53,27 @@ def test_file_offsets_single_rank():
     import bench
     g = [[[10, 1, 9, 0], [20, 1, 19, 0]]]
     assert bench.file_offsets(g) == [[0, 0]]
+
+
+@pytest.mark.timeout(300)
+def test_bench_self_launches_ranks():
+    """`bench.py --gpus 2` without torchrun's environment re-runs itself under
+    torch.distributed.run with 2 processes; the ranks rendezvous on 127.0.0.1 and rank 0
+    prints one line with n_gpus = 2, the max-over-ranks time and the all-gathered offsets
+    (the multi-rank plumbing of run_ours, over gloo here)."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "MASTER_ADDR",
+                                                            "MASTER_PORT")}
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "3",
+                          "--bytes", "1000000000", "--dist-selftest"], cwd=root, capture_output=True, text=True,
+                         timeout=280, env=env)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["ms"] == 11.0
+    assert abs(d["value"] - 2 * 3 * 1e9 / 0.011 / 1e9) < 1e-6
+    assert d["file_offsets"] == [0, 1000]
