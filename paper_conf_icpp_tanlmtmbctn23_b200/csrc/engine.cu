@@ -287,7 +287,10 @@ int ensure_table(ckpt_ctx* h, cudaStream_t st) {
   uint64_t need = h->live + 2 * h->n - 1;   // worst case: every node inserted
   if (h->dbg & 256) need = h->live + h->n / 2;   // diagnostics only: undersized table experiment
   if (h->cap && (double)need <= kMaxLoad * (double)h->cap) return CKPT_OK;
+  // geometric growth: at least double, so a lineage whose record keeps growing pays for a
+  // (stream-ordered) reallocation and rehash only O(log) times
   uint64_t new_cap = (uint64_t)((double)need / kGrowLoad) + 1;
+  if (h->cap && new_cap < 2 * h->cap) new_cap = 2 * h->cap;
   if (new_cap < 4096) new_cap = 4096;
   if (new_cap >= (1ull << 32)) return CKPT_ENOMEM;   // slot ids are u32
   // Stream-ordered growth (no host synchronisation, ckpt.h: one sync per call): the new

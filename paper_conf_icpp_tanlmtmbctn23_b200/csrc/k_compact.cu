@@ -287,7 +287,15 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       const uint32_t x1 = x0 + kStageUnits < nunits ? x0 + kStageUnits : nunits;
       for (uint32_t x = x0 + lane; x < x1; x += 32) {
         const unsigned long long so = unit_src(x);
-        if (so < g.B) cp_async16(&gw.stage[x - x0], p.buf + so, g.B - so >= 16 ? 16u : (uint32_t)(g.B - so));
+        if (so + 16 <= g.B) {
+          cp_async16(&gw.stage[x - x0], p.buf + so, 16u);
+        } else if (so < g.B) {
+          // the buffer's last, partial unit: only its bytes are read (the caller's allocation
+          // may end at B), the rest of the staged unit is zero
+          uint32_t w4[4] = {0, 0, 0, 0};
+          for (uint32_t q = 0; q < (uint32_t)(g.B - so); ++q) w4[q >> 2] |= (uint32_t)p.buf[so + q] << (8 * (q & 3));
+          gw.stage[x - x0] = make_uint4(w4[0], w4[1], w4[2], w4[3]);
+        }
       }
       if (!entries_done) {
         // while the first round is in flight: the tile's offsets and its region entries

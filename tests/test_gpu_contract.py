@@ -83,10 +83,10 @@ def test_import_rejects_corrupt_tree_bodies(oracle_mod):
     C = 64
     bufs = _lineage_with_shifts(C)
     diffs = _take(C, bufs)
-    k = next(i for i in range(1, len(diffs)) if oracle_mod.parse_diff(diffs[i])["n_shift_regions"] > 0)
+    k = next(i for i in range(1, len(diffs)) if len(oracle_mod.parse_diff(diffs[i])["shift"]) > 0)
     d = diffs[k]
     p = oracle_mod.parse_diff(d)
-    nF, nS = p["n_first_regions"], p["n_shift_regions"]
+    nF, nS = len(p["first"]), len(p["shift"])
     n = p["n_leaves"]
     assert nF > 0 and nS > 0
     cases = []

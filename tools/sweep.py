@@ -119,6 +119,14 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=F
         # the incremental checkpoint from the GPU to the host memory" (steady checkpoints)
         rec["paper_throughput_gbs"] = round((K - 1) * B / (sum(t_st) / 1e3 + sum(d2hs[1:])) / 1e9, 1)
         rec["d2h_s_steady_mean"] = round(sum(d2hs[1:]) / max(1, K - 1), 6)
+    # where the host wall time of a call goes (library host timers, include/ckpt.h [6..9]) and
+    # how often the record table grew (capacity changes) — the wall vs device gap
+    rec["host_ms_steady_mean"] = {x: round(sum(q[x] for q in phases[1:]) / max(1, K - 1), 4)
+                                  for x in ("host_pre", "host_enqueue", "host_sync_wait", "host_post")}
+    rec["wall_ms_steady_mean"] = round(1e3 * sum(walls[1:]) / max(1, K - 1), 4)
+    rec["wall_ms_steady_median"] = round(1e3 * statistics.median(walls[1:]), 4)
+    rec["device_ms_steady_mean"] = round(sum(t_st) / max(1, K - 1), 4)
+    rec["table_growths"] = sum(1 for a, b in zip(diffs, diffs[1:]) if b["record_capacity"] != a["record_capacity"])
     if prof >= 2:   # events between every kernel (breaks PDL overlap: a breakdown, not a rate)
         rec["phase_ms_steady_mean"] = {x: round(sum(q[x] for q in phases[1:]) / max(1, K - 1), 4)
                                        for x in ("leaf_hash", "insert", "phase2", "phase3", "compact", "total")}
