@@ -7,11 +7,8 @@
 //     thread runs MurmurHash3_x64_128 over its chunk (Alg.1 l.2), compares with the
 //     persistent digest Tree(leaf) of checkpoint k-1 (l.3, R5; bulk-copied into smem in
 //     the same pipeline stage), writes one candidate bit per chunk (warp ballot) and
-//     stores the new digest of non-FIXED chunks (l.21). The hashing warps issue no
-//     atomics: at k >= 1 an INSERT WARP per CTA performs the record inserts of the tiles
-//     its CTA finished (Alg.1 l.6-19) while the CTA keeps streaming, so most inserts leave
-//     the critical path; tiles it cannot take (its queue full, the CTA's last tiles,
-//     checkpoint 0, the full-change variant) are deferred to K1b.
+//     stores the new digest of non-FIXED chunks (l.21). No atomics: the insert (which
+//     has long dependent latency) runs in K1b so the streaming loop never waits on it.
 // K1t (leaf_tail_kernel): the same for the ragged tail (< 256 chunks + a partial last
 //     chunk hashed at its true length, R4) with direct loads.
 // K1b (insert_kernel): Map.insert(digest, (leaf, chkptID)) for every candidate
@@ -113,53 +110,6 @@ __device__ __forceinline__ void insert_tile(const InsertParams& p, uint32_t tile
   __syncwarp();
 }
 
-// Map.insert(digest, (leaf, chkptID)) with the R6 tie-break for the candidates of up to
-// 32 candidate words, one per lane (`word`, whose bit b is chunk base + b), by one warp at
-// k >= 1 (K1's insert warp): the candidates are spread evenly over the lanes and each
-// inserts CAS-first (after checkpoint 0 most candidates are new keys). Equal keys meet in
-// the table, where the atomicMin gives the same result as in K1b.
-__device__ __forceinline__ void insert_words(const InsertParams& p, uint32_t word, uint64_t base, uint32_t* s_word,
-                                             uint32_t* s_excl, unsigned long long* s_base, unsigned long long& ncand) {
-  const int lane = threadIdx.x & 31;
-  const uint32_t cnt = __popc(word);
-  uint32_t incl = cnt;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += v;
-  }
-  const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  if (total == 0) return;
-  s_word[lane] = word;
-  s_excl[lane] = incl - cnt;
-  s_base[lane] = base;
-  __syncwarp();
-  const uint64_t pol = policy_evict_last();
-  for (uint32_t b0 = 0; b0 < total; b0 += 32) {
-    const uint32_t j = b0 + lane;
-    if (j < total) {
-      int lo = 0;   // source word: last w with excl[w] <= j
-#pragma unroll
-      for (int step = 16; step > 0; step >>= 1)
-        if (lo + step < 32 && s_excl[lo + step] <= j) lo += step;
-      const uint32_t bb = __fns(s_word[lo], 0, (int)(j - s_excl[lo]) + 1);
-      const uint64_t c = s_base[lo] + bb;
-      const ulonglong2 v = __ldcg(reinterpret_cast<const ulonglong2*>(p.prev) + c);
-      const Digest d{v.x, v.y};
-      bool claimed;
-      unsigned long long seen;
-      const uint32_t slot = (uint32_t)table_insert_min(p.tab, p.cap, d, pack_entry(p.g.k, node_of_chunk(p.g, c)), &claimed,
-                                                       true, &seen);
-      // an entry of an earlier checkpoint never changes again (R6): the leaf is resolved
-      // here (SHIFT to it); otherwise phase 2 reads the final value from the slot
-      const unsigned long long res = seen < ((unsigned long long)p.g.k << 32) ? seen : (kResPending | slot);
-      st_evict_last_u64(p.res_of + c, res, pol);
-    }
-  }
-  ncand += total;
-  __syncwarp();
-}
-
 // Mark the stage-0 tree tile(s) holding 256-chunk leaf tile `tile` dirty (fire-and-forget;
 // a tree tile marked without candidates is processed as all-FIXED, which is harmless).
 // bits [a, b) of a 256-bit word array
@@ -215,18 +165,8 @@ __device__ __forceinline__ void defer_tile(const InsertParams& p, uint32_t tile,
   for (uint32_t r = 0; r < rounds; ++r) p.defer[i + r] = (tile << 3) | r;
 }
 
-// shared-memory acquire / release (K1's producer -> insert-warp queue)
-__device__ __forceinline__ uint32_t ld_acquire_cta(const uint32_t* a) {
-  uint32_t v;
-  asm volatile("ld.acquire.cta.shared::cta.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(a)) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_cta(uint32_t* a, uint32_t v) {
-  asm volatile("st.release.cta.shared::cta.u32 [%0], %1;" ::"r"(smem_u32(a)), "r"(v) : "memory");
-}
-
 // ------------------------------------------------------------------ K1
-// 8 hashing (consumer) warps + 1 producer warp + 1 insert warp. The producer streams the stages with TMA
+// 8 hashing (consumer) warps + 1 producer warp. The producer streams the stages with TMA
 // (full barriers, complete_tx) and re-fills a stage as soon as all 8 consumer warps have
 // released it (empty barriers, one arrive per warp): fast warps never wait for slow ones
 // at a CTA barrier, they run ahead into the next filled stage. Tiles are handed out
@@ -236,24 +176,7 @@ __device__ __forceinline__ void st_release_cta(uint32_t* a, uint32_t v) {
 // At the end of a 256-chunk tile each consumer warp leaves its candidate ballot word in
 // the stage's slot; the producer, on the stage's release, marks the tree tile(s) dirty and
 // defers the tile's inserts to K1b, so that bookkeeping is off the hashing warps' path.
-#ifndef CKPT_K1_INSWARP
-#define CKPT_K1_INSWARP 0   // 1: insert warp in K1 (experiment: measured slower)
-#endif
-constexpr int kK1Threads = kLeafThreads + (CKPT_K1_INSWARP ? 64 : 32);
-#ifndef CKPT_K1_RING
-#define CKPT_K1_RING 32   // queued tiles per CTA for its insert warp (more: deferred to K1b)
-#endif
-constexpr uint32_t kRing = CKPT_K1_RING;
-#ifndef CKPT_K1_DBG_NOPUSH
-#define CKPT_K1_DBG_NOPUSH 0     // A/B only: the producer never queues (insert warp idles)
-#endif
-#ifndef CKPT_K1_DBG_NOINSERT
-#define CKPT_K1_DBG_NOINSERT 0   // A/B only: queued tiles are deferred to K1b, no insert here
-#endif
-#ifndef CKPT_K1_POLL_NS
-#define CKPT_K1_POLL_NS 64       // insert warp: sleep between polls of an empty queue
-#endif
-constexpr uint32_t kBatch = 4;   // queued tiles per insert-warp batch (4 x 8 candidate words = one word per lane)
+constexpr int kK1Threads = kLeafThreads + 32;
 constexpr int kMaxStagesK1 = 8;
 #ifndef CKPT_K1_CTAS
 #define CKPT_K1_CTAS 2   // resident K1 CTAs per SM when C % 128 == 0 (3 stages of 36 KB each)
@@ -269,12 +192,6 @@ struct K1Shared {
   uint32_t tile[kMaxStagesK1];       // tile streamed into the stage (kNoTile: stop)
   uint32_t tile_end[kMaxStagesK1];   // 1 if the stage holds the tile's last segment
   uint32_t words[kMaxStagesK1][8];   // candidate ballot words of the tile ending in the stage
-  // producer -> insert warp queue of finished tiles with candidates (k >= 1)
-  uint32_t ring_tile[kRing];
-  uint32_t ring_words[kRing][8];
-  uint32_t ring_head, ring_tail, ring_stop;
-  uint32_t ins_word[32], ins_excl[32];   // insert_words scratch of the insert warp
-  unsigned long long ins_base[32];
 };
 
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
@@ -298,10 +215,6 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
   const int segs = p.segs;
   const bool use_prev = p.g.k > 0;
 
-  // k >= 1, Tree / List, no full-change switch: inserts in this kernel (the insert warp);
-  // otherwise every tile's inserts go to K1b as before (checkpoint 0: hot repeated keys
-  // need K1b's warp-level de-duplication; R23: a switched checkpoint makes no record op)
-  const bool inline_ins = CKPT_K1_INSWARP && p.g.k > 0 && p.ins.mode != kModeBasic && p.ins.sw_permille < 0;
   if (tid == 0) {
     prefetch_tmap(&tmap);
     for (int s = 0; s < nst; ++s) {
@@ -309,90 +222,25 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
       mbar_init(&sh.empty[s], kLeafThreads / 32);
     }
     fence_mbar_init();
-    sh.ring_head = 0;
-    sh.ring_tail = 0;
-    sh.ring_stop = 0;
   }
   __syncthreads();
-
-  if (tid >= kLeafThreads + 32) {
-    // ---------------- insert warp: Map.insert of the tiles this CTA finished (Alg.1 l.6-19).
-    // Up to kBatch queued tiles are taken at once: their 8 x kBatch candidate words form
-    // one list whose inserts share the dependent round trips (digest load, CAS, value).
-    // When the CTA has streamed its last tile, at most one more batch is processed here;
-    // a longer backlog goes to K1b, whose many warps drain it in parallel (a single warp
-    // draining a full queue would hold the CTA, and K1, for tens of microseconds).
-    if (!inline_ins) return;
-    const int lane = tid & 31;
-    uint32_t tail = 0;
-    unsigned long long ncand = 0;
-    for (;;) {
-      // `stop` before `head`: once the producer's stop flag is seen, the head read after it
-      // is final (it queues nothing after setting the flag)
-      const bool stop = __shfl_sync(0xffffffffu, lane == 0 ? ld_acquire_cta(&sh.ring_stop) : 0u, 0) != 0;
-      const uint32_t head = __shfl_sync(0xffffffffu, lane == 0 ? ld_acquire_cta(&sh.ring_head) : 0u, 0);
-      if (stop || CKPT_K1_DBG_NOINSERT) {
-        // the CTA is streaming its last tiles: hand the queue to K1b (the tiles are already
-        // marked dirty; only their inserts are deferred)
-        for (uint32_t t = tail + lane; t < head; t += 32) {
-          const uint32_t slot = t % kRing;
-          uint32_t pc = 0;
-#pragma unroll
-          for (int q = 0; q < 8; ++q) pc += __popc(sh.ring_words[slot][q]);
-          defer_tile(p.ins, sh.ring_tile[slot], pc);
-        }
-        if (stop) break;
-        __syncwarp();
-        if (lane == 0) st_release_cta(&sh.ring_tail, head);
-        tail = head;
-        __nanosleep(CKPT_K1_POLL_NS);
-        continue;
-      }
-      if (head == tail) {
-        __nanosleep(CKPT_K1_POLL_NS);
-        continue;
-      }
-      const uint32_t E = head - tail < kBatch ? head - tail : kBatch;
-      const uint32_t e = (uint32_t)lane >> 3, q = (uint32_t)lane & 7;
-      const uint32_t slot = (tail + (e < E ? e : 0)) % kRing;
-      const uint32_t tile = sh.ring_tile[slot];
-      const uint32_t word = e < E ? sh.ring_words[slot][q] : 0u;
-      __syncwarp();
-      if (lane == 0) st_release_cta(&sh.ring_tail, tail + E);   // the entries are in registers
-      tail += E;
-      insert_words(p.ins, word, (uint64_t)tile * 256 + 32 * q, sh.ins_word, sh.ins_excl, sh.ins_base, ncand);
-    }
-    if (lane == 0 && ncand) atomicAdd(&p.ins.tot->n_cand, ncand);
-    return;
-  }
 
   if (tid >= kLeafThreads) {
     // ---------------- producer warp (lane 0)
     if (tid != kLeafThreads) return;
     const uint64_t pol_stream = policy_evict_first();
     uint32_t* cursor = &p.ins.tot->k1_next;
-    uint32_t head = 0;
-    bool ending = false;   // the stop marker is issued: nothing more is queued
-    // the tile epilogue of the step last consumed from stage s: dirty marks (fire-and-forget),
-    // then the tile's inserts are queued for the insert warp or deferred to K1b
+    // the tile epilogue of the step last consumed from stage s: dirty marks + deferral
     auto epilogue = [&](int s) {
       if (!sh.tile_end[s]) return;
       const uint32_t tile = sh.tile[s];
       uint32_t w[8], any = 0, pc = 0;
 #pragma unroll
       for (int q = 0; q < 8; ++q) { w[q] = sh.words[s][q]; any |= w[q]; pc += __popc(w[q]); }
-      if (!any) return;
-      mark_tree_dirty(p.ins, tile, w);
-      if (p.ins.mode == kModeBasic) return;   // Basic keeps no record
-      if (inline_ins && !ending && !CKPT_K1_DBG_NOPUSH && head - ld_acquire_cta(&sh.ring_tail) < kRing) {
-        const uint32_t slot = head % kRing;
-        sh.ring_tile[slot] = tile;
-#pragma unroll
-        for (int q = 0; q < 8; ++q) sh.ring_words[slot][q] = w[q];
-        st_release_cta(&sh.ring_head, ++head);
-        return;
+      if (any) {
+        mark_tree_dirty(p.ins, tile, w);
+        if (p.ins.mode != kModeBasic) defer_tile(p.ins, tile, pc);   // Basic keeps no record
       }
-      defer_tile(p.ins, tile, pc);
     };
     // tiles are handed out in groups of tpg consecutive tiles (one cursor atomic per group:
     // at small C a tile is only 256 C bytes, and one atomic per tile on one address
@@ -411,10 +259,6 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
         sh.tile[s] = kNoTile;
         sh.tile_end[s] = 0;
         mbar_arrive(&sh.full[s]);
-        // the last tiles' inserts go to K1b: an insert warp still working when the consumers
-        // finish would hold the CTA (its round trips are slow while HBM is saturated)
-        ending = true;
-        st_release_cta(&sh.ring_stop, 1u);
         break;
       }
       const bool with_prev = use_prev && (int)seg == segs - 1;
@@ -445,7 +289,6 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
       mbar_wait(&sh.empty[j % nst], (j / nst) & 1u);
       epilogue((int)(j % (uint32_t)nst));
     }
-    if (!ending) st_release_cta(&sh.ring_stop, 1u);
     return;
   }
 
@@ -702,19 +545,7 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   size_t smem;
   leaf_smem_config(p, &smem);
   const uint64_t n_tiles = p.n_main / kLeafThreads;
-  // resident CTAs per SM for this configuration's shared memory (the persistent grid is one
-  // wave; a configuration that fits fewer CTAs than the launch bound gets a smaller grid)
-  static thread_local size_t occ_smem[2] = {0, 0};
-  static thread_local int occ_val[2] = {0, 0};
-  int& occ = occ_val[p.mode3d ? 1 : 0];
-  if (occ_smem[p.mode3d ? 1 : 0] != smem) {   // queried once per configuration
-    occ = 0;
-    if (p.mode3d) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, leaf_hash_kernel<1>, kK1Threads, smem);
-    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, leaf_hash_kernel<0>, kK1Threads, smem);
-    occ_smem[p.mode3d ? 1 : 0] = smem;
-  }
-  const int want = p.mode3d ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC;
-  uint64_t grid = (uint64_t)num_sms * (occ > 0 && occ < want ? occ : want);
+  uint64_t grid = (uint64_t)num_sms * (p.mode3d ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC);
   const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
   if (grid > groups) grid = groups;
   if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
