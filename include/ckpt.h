@@ -231,8 +231,9 @@ CKPT_API int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_
  * [3] phase 3 (all stages), [4] compaction (offsets + gather), [5] whole call (first
  * kernel to last kernel; [1]..[4] are 0 at level 1); host wall times of the same call
  * (always recorded): [6] entry to first enqueue, [7] enqueue of the kernel sequence, [8]
- * wait in the one stream synchronisation, [9] bookkeeping after it.  n <= 10 values are
- * written.  ckpt_set_profiling errors: CKPT_EINVAL (level outside 0..2). */
+ * wait in the one stream synchronisation, [9] bookkeeping after it, and within [6]: [10]
+ * record-table growth (stream-ordered allocation, fill and rehash enqueued), [11] diff-arena
+ * growth (physical memory mapped).  n <= 12 values are written.  ckpt_set_profiling errors: CKPT_EINVAL (level outside 0..2). */
 CKPT_API int ckpt_set_profiling(ckpt_handle h, int enable);
 CKPT_API int ckpt_phase_times(ckpt_handle h, float* times, int n);
 /* Same for checkpoint `id` (device times kept for the latest 256 profiled checkpoints; the
@@ -247,8 +248,9 @@ CKPT_API int ckpt_kernel_launches(ckpt_handle h, uint64_t* count);
 /* Number of times this handle has blocked the host on the device so far (stream
  * synchronisations and the completion spin of ckpt_checkpoint), counted at the wait sites.
  * ckpt_checkpoint adds exactly one, including a call that grows the record table (the
- * growth is stream-ordered: allocation, rehash and release of the old table run on the
- * caller's stream).  Errors: CKPT_EINVAL. */
+ * growth enqueues the fill and rehash on the caller's stream; the replaced table is kept
+ * until ckpt_destroy, at most the size of the current one since growth doubles it).
+ * Errors: CKPT_EINVAL. */
 CKPT_API int ckpt_host_syncs(ckpt_handle h, uint64_t* count);
 
 /* Release all device memory of the handle (record, leaf digests, every diff). */

@@ -27,7 +27,7 @@ LABEL_NONE, FIRST, FIXED, SHIFT, DONE = 0, 1, 2, 3, 4
 STAT_NAMES = [
     "id", "bytes", "meta_bytes", "data_bytes", "n_first_regions", "n_shift_regions",
     "n_first", "n_fixed", "n_spatial", "n_temporal", "list_entries", "record_growth",
-    "phase2_inserts", "n_leaves",
+    "phase2_inserts", "n_leaves", "phase3_inserts",
 ]
 
 
@@ -106,7 +106,9 @@ def mmh3(data: bytes, seed: int = 0) -> bytes:
 
 MODE_TREE, MODE_LIST, MODE_BASIC = 0, 1, 2   # the methods compared in P:194 (Tree = ours)
 VAR_FULL_FIRST, VAR_FULL_SWITCH = 1, 2       # Tree-method variants (NEXT #4)
+VAR_SHIFT_INSERT = 4                         # NEXT #4(c): the SHIFT-SHIFT-insert reading of P:89 (R24)
 FLAGS_FULL = 3                               # header flags of a difference stored in full
+FLAGS_SHIFT_INSERT = 4                       # header flags of a Tree difference under VAR_SHIFT_INSERT
 
 
 class Oracle:

@@ -311,19 +311,19 @@ class Checkpointer:
             raise CkptError(rc, "ckpt_set_profiling")
 
     PHASES = ["leaf_hash", "insert", "phase2", "phase3", "compact", "total",
-              "host_pre", "host_enqueue", "host_sync_wait", "host_post"]
+              "host_pre", "host_enqueue", "host_sync_wait", "host_post", "host_table_growth", "host_arena_growth"]
 
     def phase_times(self, cid: int | None = None) -> dict:
         """Per-phase device times (ms) of checkpoint cid (default: the latest), measured with
         CUDA events on the caller's stream when profiling is on; host times for the latest."""
-        t = (ctypes.c_float * 10)()
+        t = (ctypes.c_float * 12)()
         if cid is None:
-            lib().ckpt_phase_times(self._h, t, 10)
+            lib().ckpt_phase_times(self._h, t, 12)
         else:
-            rc = lib().ckpt_phase_times_of(self._h, cid, t, 10)
+            rc = lib().ckpt_phase_times_of(self._h, cid, t, 12)
             if rc != CKPT_OK:
                 raise CkptError(rc, "ckpt_phase_times_of")
-        return {self.PHASES[i]: t[i] for i in range(10)}
+        return {self.PHASES[i]: t[i] for i in range(12)}
 
     @property
     def host_syncs(self) -> int:

@@ -104,6 +104,7 @@ struct ckpt_ctx {
   Totals* tot_host = nullptr;   // pinned + mapped: written by the gather kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
+  std::vector<void*> retired;    // record tables replaced by a growth (freed by ckpt_destroy)
   DiffArena arena;
   std::vector<DiffRec> diffs;
   uint8_t* staging = nullptr;
@@ -127,7 +128,7 @@ struct ckpt_ctx {
   int64_t ev_id[kEvRing] = {};
   int ev_level[kEvRing] = {};
   cudaEvent_t* ev = nullptr;     // event set of the current call
-  float times[12] = {};          // host times of the latest call ([6..9])
+  float times[12] = {};          // host times of the latest call ([6..11])
   PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   std::vector<void*> allocs;   // per-geometry allocations
   // diagnostics: CKPT_TRACE=<file prefix> records per-group tree timings of each call
@@ -293,18 +294,21 @@ int ensure_table(ckpt_ctx* h, cudaStream_t st) {
   if (h->cap && new_cap < 2 * h->cap) new_cap = 2 * h->cap;
   if (new_cap < 4096) new_cap = 4096;
   if (new_cap >= (1ull << 32)) return CKPT_ENOMEM;   // slot ids are u32
-  // Stream-ordered growth (no host synchronisation, ckpt.h: one sync per call): the new
-  // table is allocated, filled and rehashed on the caller's stream, and the old one is
-  // freed in stream order behind the rehash that reads it.
+  // Growth without a host synchronisation (ckpt.h: one sync per call): the new table is
+  // allocated (cudaMalloc: < 1 ms for GBs on B200, where a stream-ordered cudaMallocAsync
+  // took 6-23 ms, tools/alloc_probe.cu), filled and rehashed on the caller's stream. The
+  // old table is read by that rehash, so it is retired, not freed: cudaFree would
+  // synchronise the device. Retired tables (geometric growth: together at most the size of
+  // the current one) are released by ckpt_destroy.
   Slot* nt = nullptr;
-  if (cudaMallocAsync(reinterpret_cast<void**>(&nt), new_cap * sizeof(Slot), st) != cudaSuccess) {
+  if (cudaMalloc(reinterpret_cast<void**>(&nt), new_cap * sizeof(Slot)) != cudaSuccess) {
     cudaGetLastError();
     return CKPT_ENOMEM;
   }
   if (cudaMemsetAsync(nt, 0xFF, new_cap * sizeof(Slot), st) != cudaSuccess) return CKPT_ECUDA;
   if (h->tab) {
     if (launch_rehash(h->tab, h->cap, nt, new_cap, st) != cudaSuccess) return CKPT_ECUDA;
-    if (cudaFreeAsync(h->tab, st) != cudaSuccess) return CKPT_ECUDA;
+    h->retired.push_back(h->tab);
   }
   h->tab = nt;
   h->cap = new_cap;
@@ -514,6 +518,7 @@ int ckpt_destroy(ckpt_handle h) {
   for (void* q : {(void*)h->owner, (void*)h->rs_len, h->rs_scan, (void*)h->rs_err, (void*)h->rs_chain})
     if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
+  for (void* q : h->retired) cudaFree(q);
   if (h->tot_host) cudaFreeHost(h->tot_host);
   if (h->staging) cudaFree(h->staging);
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r)
@@ -562,7 +567,7 @@ int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const int r = (int)(id % ckpt_ctx::kEvRing);
-  float t[10] = {};
+  float t[12] = {};
   if (h->ev_id[r] == (int64_t)id) {
     cudaEvent_t* e = h->evr[r];
     if (h->ev_level[r] >= 2) {
@@ -574,15 +579,15 @@ int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
     cudaGetLastError();
   }
   if (id + 1 == h->diffs.size())
-    for (int i = 6; i < 10; ++i) t[i] = h->times[i];
-  for (int i = 0; i < n && i < 10; ++i) times[i] = t[i];
+    for (int i = 6; i < 12; ++i) t[i] = h->times[i];
+  for (int i = 0; i < n && i < 12; ++i) times[i] = t[i];
   return CKPT_OK;
 }
 
 int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
   if (h->diffs.empty()) {
-    for (int i = 0; i < n && i < 10; ++i) times[i] = 0.f;
+    for (int i = 0; i < n && i < 12; ++i) times[i] = 0.f;
     return CKPT_OK;
   }
   return ckpt_phase_times_of(h, (uint32_t)(h->diffs.size() - 1), times, n);
@@ -634,10 +639,14 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     if (r != CKPT_OK) return r;
   }
   const uint32_t k = (uint32_t)h->diffs.size();
+  const auto t_tab = clk::now();
   int r = h->mode == kModeBasic ? CKPT_OK : ensure_table(h, st);   // Basic keeps no record
   if (r != CKPT_OK) return r;
+  const auto t_arena = clk::now();
   const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
   if (!h->arena.ensure(worst)) return CKPT_ENOMEM;
+  h->times[10] = ms_since(t_tab, t_arena);
+  h->times[11] = ms_since(t_arena, clk::now());
   uint8_t* out = h->arena.top_ptr();
 
   const Geo g = make_geo(h, k);

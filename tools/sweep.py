@@ -122,7 +122,11 @@ def run_case(name, cfg, B, C, K, p, stream, host_gen=None, prof=1, mode=0, d2h=F
     # where the host wall time of a call goes (library host timers, include/ckpt.h [6..9]) and
     # how often the record table grew (capacity changes) — the wall vs device gap
     rec["host_ms_steady_mean"] = {x: round(sum(q[x] for q in phases[1:]) / max(1, K - 1), 4)
-                                  for x in ("host_pre", "host_enqueue", "host_sync_wait", "host_post")}
+                                  for x in ("host_pre", "host_enqueue", "host_sync_wait", "host_post",
+                                            "host_table_growth", "host_arena_growth")}
+    rec["host_pre_ms_max"] = round(max(q["host_pre"] for q in phases[1:]), 3) if K > 1 else None
+    rec["host_table_growth_ms_max"] = round(max(q["host_table_growth"] for q in phases[1:]), 3) if K > 1 else None
+    rec["host_arena_growth_ms_max"] = round(max(q["host_arena_growth"] for q in phases[1:]), 3) if K > 1 else None
     rec["wall_ms_steady_mean"] = round(1e3 * sum(walls[1:]) / max(1, K - 1), 4)
     rec["wall_ms_steady_median"] = round(1e3 * statistics.median(walls[1:]), 4)
     rec["device_ms_steady_mean"] = round(sum(t_st) / max(1, K - 1), 4)
