@@ -222,7 +222,7 @@ def test_variant_rejections(oracle_mod):
     with pytest.raises(ValueError):
         o.set_variant(FULL_SWITCH, 1001)
     with pytest.raises(ValueError):
-        o.set_variant(4)
+        o.set_variant(8)                 # unknown flag bit (4 is the SHIFT-insert variant)
     o.checkpoint(np.zeros(64, dtype=np.uint8))
     with pytest.raises(ValueError):
         o.set_variant(FULL_FIRST)
