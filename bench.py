@@ -456,6 +456,26 @@ def run_ours(args):
                       "note": "ckpt_import of every diff from host memory into a fresh handle"}
         ck3.close()
         del host_diffs
+    # NEXT #4(c): checkpoint 0 of the same lineage under the SHIFT-SHIFT-insert variant (R24),
+    # whose zero-heavy first checkpoint collapses into few regions (untimed, one call)
+    ck0_si = None
+    try:
+        if inplace:
+            raise RuntimeError("skipped in place (memory for a second handle at this size)")
+        cks = Checkpointer(C)
+        cks.set_variant(4)
+        e0s, e1s = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0s.record(stream)
+        dsi = cks.checkpoint(lin.get(0), nbytes=B, stream=stream)
+        e1s.record(stream)
+        stream.synchronize()
+        ck0_si = {"bytes": dsi["bytes"], "regions": dsi["n_first_regions"] + dsi["n_shift_regions"],
+                  "inserted_shifted_regions": dsi["phase3_inserts"], "ms": round(e0s.elapsed_time(e1s), 3),
+                  "default_bytes": diffs[0]["bytes"],
+                  "default_regions": diffs[0]["n_first_regions"] + diffs[0]["n_shift_regions"]}
+        cks.close()
+    except Exception as e:  # pragma: no cover
+        ck0_si = {"error": str(e)}
     check_first = ck.diff_to_host(Wm) if not inplace else None
     check_last = ck.diff_to_host(Wm + K - 1) if not inplace else None
     ck.close()
@@ -572,6 +592,7 @@ def run_ours(args):
                                         max(1, sum(d["n_first_regions"] + d["n_shift_regions"] for d in steady)), 2),
             "checkpoint0": {"ms": round(ck0["total"], 3), "gbs": round(B / (ck0["total"] / 1e3) / 1e9, 1),
                             "bytes": diffs[0]["bytes"], "note": "first touch of the lineage (untimed warm-up)"},
+            "checkpoint0_shift_insert": ck0_si,
             "restore": {"id": Wm + K - 1, "s": round(rs, 5), "gbs": round(B / rs / 1e9, 2), "ok": restore_ok,
                         "cold_s": round(rs_cold, 5), "note": "host wall time of ckpt_restore (synchronous); cold = "
                                                              "first restore, which builds the per-diff plans"},

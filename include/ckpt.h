@@ -71,6 +71,7 @@ typedef struct {
   uint64_t record_size;     /* entries in the historical record after this checkpoint */
   uint64_t record_capacity; /* slots of the device record table                              */
   uint64_t phase2_inserts;  /* FIRST internal nodes inserted (Alg.1 l.29)                    */
+  uint64_t phase3_inserts;  /* CKPT_VARIANT_SHIFT_INSERT: shifted regions inserted (R24)*/
 } ckpt_diff;
 
 /* De-duplication methods compared in the paper; the diff header's u16 `flags`
@@ -104,11 +105,24 @@ enum { CKPT_MODE_TREE = 0, CKPT_MODE_LIST = 1, CKPT_MODE_BASIC = 2 };
  *                             leaf digests are still updated, l.21). Its statistics count the
  *                             changed chunks as n_first (n_spatial = n_temporal = 0) and
  *                             phase2_inserts = 0; record_size is unchanged.
+ *   CKPT_VARIANT_SHIFT_INSERT "If this is the case, the new region is added to the historical
+ *                             record of unique hashes", reading R24: after phase 2,
+ *                             every internal node whose leaves are all shifted duplicates and
+ *                             whose hash is new enters the record (minimum node id among
+ *                             equal hashes, as R6); in phase 3 a parent of two shifted
+ *                             children that finds ITS OWN entry is the first occurrence of
+ *                             that content: its children are saved and it is not a region.
+ *                             Repeated content then collapses into few regions (an all-zero
+ *                             buffer of n = 2^h chunks: 2h regions instead of n). Such a node
+ *                             can be the source of a later region although its bytes are no
+ *                             first-occurrence data: restore resolves those sources chunk by
+ *                             chunk through the source checkpoint's own regions (R25). Its
+ *                             Tree differences carry header flags CKPT_FLAGS_SHIFT_INSERT.
  * A difference stored in full has header flags CKPT_FLAGS_FULL and the Tree layout with
  * n_first_regions = 1 (the root, node 0), n_shift_regions = 0 and the whole buffer as data
  * (meta_bytes = 80, data_bytes = B); ckpt_restore and ckpt_import accept it. */
-enum { CKPT_VARIANT_FULL_FIRST = 1, CKPT_VARIANT_FULL_SWITCH = 2 };
-enum { CKPT_FLAGS_FULL = 3 };
+enum { CKPT_VARIANT_FULL_FIRST = 1, CKPT_VARIANT_FULL_SWITCH = 2, CKPT_VARIANT_SHIFT_INSERT = 4 };
+enum { CKPT_FLAGS_FULL = 3, CKPT_FLAGS_SHIFT_INSERT = 4 };
 
 /* Create a handle.  P:77: fixed-size chunks of "tens or hundreds of bytes".
  *   chunk_bytes  C, a multiple of 16 with 32 <= C <= 65536 (C > 2 x 16-B digest).

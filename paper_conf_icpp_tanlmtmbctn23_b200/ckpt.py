@@ -20,7 +20,9 @@ CKPT_OK, CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ERANGE, CKPT_ESTATE, CKPT_EC
 
 CKPT_MODE_TREE, CKPT_MODE_LIST, CKPT_MODE_BASIC = 0, 1, 2   # methods of P:194 (include/ckpt.h)
 CKPT_VARIANT_FULL_FIRST, CKPT_VARIANT_FULL_SWITCH = 1, 2      # Tree variants
+CKPT_VARIANT_SHIFT_INSERT = 4                                 # Tree variant: P:89's insert reading (R24)
 CKPT_FLAGS_FULL = 3                                           # header flags of a full difference
+CKPT_FLAGS_SHIFT_INSERT = 4                                   # header flags under the SHIFT-insert variant
 
 ABI_FUNCTIONS = [
     "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore",
@@ -51,6 +53,7 @@ class CkptDiff(ctypes.Structure):
         ("record_size", ctypes.c_uint64),
         ("record_capacity", ctypes.c_uint64),
         ("phase2_inserts", ctypes.c_uint64),
+        ("phase3_inserts", ctypes.c_uint64),
     ]
 
     def as_dict(self) -> dict:

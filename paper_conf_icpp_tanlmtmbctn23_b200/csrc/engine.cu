@@ -83,9 +83,11 @@ struct ckpt_ctx {
   unsigned long long* tsrc[kMaxStages] = {};
   uint32_t* arr2[kMaxStages] = {};
   uint32_t* arr3[kMaxStages] = {};
+  uint32_t* arr4[kMaxStages] = {};
   uint32_t* dcnt[kMaxStages] = {};
   uint32_t* gm2[kMaxStages] = {};
   uint32_t* gm3[kMaxStages] = {};
+  uint32_t* gm4[kMaxStages] = {};
   uint32_t* wl0 = nullptr;
   uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
   uint32_t* tcc = nullptr;       // candidate leaves per stage-0 tree tile (inside ctr)
@@ -238,7 +240,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
     size_t off[kMaxStages] = {};
     for (int s = 1; s < h->S; ++s) {
       off[s] = bytes;
-      bytes += (3 + 32 + 64) * h->ngroups[s] * sizeof(uint32_t);   // arr2 arr3 dcnt, gm2, gm3
+      bytes += (4 + 32 + 64 + 32) * h->ngroups[s] * sizeof(uint32_t);   // arr2 arr3 arr4 dcnt, gm2, gm3, gm4
     }
     AL(h->ctr2[0], bytes);
     AL(h->ctr2[1], bytes);
@@ -358,6 +360,7 @@ void fill_diff(const ckpt_ctx* h, uint32_t id, const Totals& t, uint8_t* ptr, ck
   d->record_size = h->live;
   d->record_capacity = h->cap;
   d->phase2_inserts = t.p2_inserts;
+  d->phase3_inserts = t.p3_inserts;
 }
 
 // ---- host twins of dev.cuh's tree geometry (R3), used only to validate imported diffs
@@ -550,7 +553,7 @@ int ckpt_host_syncs(ckpt_handle h, uint64_t* count) {
 int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_permille) {
   if (!h) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
-  if (h->mode != kModeTree || !h->diffs.empty() || (flags & ~3u) || switch_permille > 1000) return CKPT_EINVAL;
+  if (h->mode != kModeTree || !h->diffs.empty() || (flags & ~7u) || switch_permille > 1000) return CKPT_EINVAL;
   h->variant = flags;
   h->switch_permille = switch_permille;
   return CKPT_OK;
@@ -612,9 +615,11 @@ static void select_ctr(ckpt_ctx* h, int parity) {
   for (int s = 1; s < h->S; ++s) {
     h->arr2[s] = reinterpret_cast<uint32_t*>(c + h->ctr_stage_off[s]);
     h->arr3[s] = h->arr2[s] + h->ngroups[s];
-    h->dcnt[s] = h->arr3[s] + h->ngroups[s];
+    h->arr4[s] = h->arr3[s] + h->ngroups[s];
+    h->dcnt[s] = h->arr4[s] + h->ngroups[s];
     h->gm2[s] = h->dcnt[s] + h->ngroups[s];
     h->gm3[s] = h->gm2[s] + 32 * h->ngroups[s];
+    h->gm4[s] = h->gm3[s] + 64 * h->ngroups[s];
   }
 }
 
@@ -751,15 +756,19 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     sp.tsrc = h->tsrc[s];
     sp.arr2 = h->arr2[s];
     sp.arr3 = h->arr3[s];
+    sp.arr4 = h->arr4[s];
     sp.dcnt = h->dcnt[s];
     sp.gm2 = h->gm2[s];
     sp.gm3 = h->gm3[s];
+    sp.gm4 = h->gm4[s];
   }
   tp.list = h->mode == kModeList;
+  tp.shift_insert = h->mode == kModeTree && (h->variant & CKPT_VARIANT_SHIFT_INSERT);
   tp.sw_permille = ip.sw_permille;
   if (h->mode != kModeBasic) {   // Basic: no record, no tree
     CK(launch_tree(tp, 2, h->num_sms, st));
     if (pe) CK(cudaEventRecord(h->ev[3], st));
+    if (tp.shift_insert) CK(launch_tree(tp, 4, h->num_sms, st));   // R24 inserts, before any lookup
     CK(launch_tree(tp, 3, h->num_sms, st));
     if (pe) CK(cudaEventRecord(h->ev[4], st));
   } else if (pe) {
@@ -781,6 +790,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.ctr_next = reinterpret_cast<uint4*>(h->ctr2[(k + 1) & 1]);
   cp.ctr_next_words = h->ctr_bytes / 16;
   cp.mode = h->mode;
+  cp.flags = tp.shift_insert ? CKPT_FLAGS_SHIFT_INSERT : h->mode;
   cp.cand = h->cand;
   cp.nwords = h->nwords;
   cp.tcc = h->tcc;
@@ -830,7 +840,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
     if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), f); fclose(f); }
   }
-  if (h->mode != kModeBasic && t.full_kind != 2) h->live += t.n_first + t.p2_inserts;   // R23: no record op
+  if (h->mode != kModeBasic && t.full_kind != 2) h->live += t.n_first + t.p2_inserts + t.p3_inserts;   // R23: no record op
   DiffRec rec;
   rec.ptr = out;
   fill_diff(h, k, t, out, &rec.info);
@@ -942,6 +952,7 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     DiffRec& d = h->diffs[c];
     RestoreDiff& r = rd[c];
     r.id = c;
+    r.composite = (h->variant & CKPT_VARIANT_SHIFT_INSERT) ? 1u : 0u;   // R25
     r.base = d.ptr;
     r.nF = d.info.n_first_regions;
     r.nS = d.info.n_shift_regions;
@@ -959,6 +970,7 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     }
     r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
     r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
+    r.Cch = d.Cch; r.Csrc = d.Csrc;
     if (!d.planned && r.nF &&
         (basic ? restore_prepare_basic(g, r, h->nwords, h->rs_len, h->rs_scan, h->rs_scan_bytes, st)
                : restore_prepare_first(g, r, h->rs_len, h->rs_scan, h->rs_scan_bytes, st)) != cudaSuccess)
@@ -1004,6 +1016,22 @@ static int ensure_plans(ckpt_ctx* h, uint32_t id, const Geo& g, cudaStream_t st)
     rd[c].Cch = d.Cch;
     rd[c].Csrc = d.Csrc;
     if (restore_claimlist(g, rd[c], h->num_sms, st) != cudaSuccess) return CKPT_ECUDA;
+    if (rd[c].composite && rd[c].nS) {
+      // R25: SHIFT chunks whose source lies outside the source diff's FIRST data take the
+      // address of that chunk in the source checkpoint (its own claim list, complete for
+      // older diffs; for this diff, one level per pass since a source node's bytes are
+      // regions of smaller levels)
+      if (cudaMemcpyAsync(h->rs_chain + c, &rd[c], sizeof(RestoreDiff), cudaMemcpyHostToDevice, st) != cudaSuccess ||
+          restore_resolve(g, rd[c], h->rs_chain, h->h + 2, h->rs_err, h->num_sms, st) != cudaSuccess)
+        return CKPT_ECUDA;
+    }
+  }
+  {
+    int herr2 = 0;
+    if (cudaMemcpyAsync(&herr2, h->rs_err, sizeof(int), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        sync_stream(h, st) != cudaSuccess)
+      return CKPT_ECUDA;
+    if (herr2) return CKPT_EINVAL;   // a source chunk no diff covers (malformed chain)
   }
   if (sync_stream(h, st) != cudaSuccess) return CKPT_ECUDA;
   for (uint32_t c = 0; c <= id; ++c) h->diffs[c].planned = true;
@@ -1031,8 +1059,10 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
   std::memcpy(&flags, hd + 6, 2);
   const uint32_t id = (uint32_t)h->diffs.size();
   const uint64_t B = rd64h(16), n = rd64h(24), nF = rd64h(32), nS = rd64h(40), data = rd64h(48);
-  const bool full_form = flags == CKPT_FLAGS_FULL && h->mode == kModeTree && h->variant != 0;   // R22 / R23
-  if (rd32h(0) != 0x44504B43u || ver != 1 || (flags != (uint16_t)h->mode && !full_form) || rd32h(8) != id ||
+  const bool full_form = flags == CKPT_FLAGS_FULL && h->mode == kModeTree && (h->variant & 3);   // R22 / R23
+  const bool shift_insert = h->mode == kModeTree && (h->variant & CKPT_VARIANT_SHIFT_INSERT);      // R24
+  const uint16_t want_flags = shift_insert ? (uint16_t)CKPT_FLAGS_SHIFT_INSERT : (uint16_t)h->mode;
+  if (rd32h(0) != 0x44504B43u || ver != 1 || (flags != want_flags && !full_form) || rd32h(8) != id ||
       rd32h(12) != h->C)
     return CKPT_EINVAL;
   if (B == 0 || n != (B + h->C - 1) / h->C || n > (1ull << 31) || (h->geo_set && B != h->B)) return CKPT_EINVAL;
@@ -1139,7 +1169,7 @@ int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream)
   uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
   for (int64_t c = id; c >= 0; --c) {
     const DiffRec& d = h->diffs[c];
-    RestoreDiff r;
+    RestoreDiff r = {};
     r.id = (uint32_t)c;
     r.base = d.ptr;
     r.nF = d.info.n_first_regions;

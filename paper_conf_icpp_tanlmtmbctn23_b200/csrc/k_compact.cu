@@ -165,7 +165,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     uint8_t* o = p.out;
     *reinterpret_cast<uint32_t*>(o + 0) = 0x44504B43u;   // 'CKPD'
     *reinterpret_cast<uint16_t*>(o + 4) = 1;             // version
-    *reinterpret_cast<uint16_t*>(o + 6) = (uint16_t)p.mode;   // flags: the method
+    *reinterpret_cast<uint16_t*>(o + 6) = (uint16_t)p.flags;  // flags: the method, 4 under R24
     *reinterpret_cast<uint32_t*>(o + 8) = g.k;
     *reinterpret_cast<uint32_t*>(o + 12) = g.C;
     *reinterpret_cast<unsigned long long*>(o + 16) = g.B;

@@ -123,7 +123,63 @@ __global__ void __launch_bounds__(kRT) claimlist_kernel(Geo g, RestoreDiff d) {
     }
     const unsigned long long rel = o - __ldg(off + lo);
     d.Cch[t] = (uint32_t)((first ? __ldg(d.Flo + lo) : __ldg(d.Slo + lo)) + rel / C);
-    d.Csrc[t] = first ? (unsigned long long)(data + o) : __ldg(d.Ssrc + lo) + rel;
+    // Ssrc == 0: a source node whose bytes are no first-occurrence data (R25), resolved
+    // chunk by chunk by resolve_kernel
+    const unsigned long long ss = first ? 0ull : __ldg(d.Ssrc + lo);
+    d.Csrc[t] = first ? (unsigned long long)(data + o) : (ss ? ss + rel : 0ull);
+  }
+}
+
+// resolve_kernel (R25, plan building of a SHIFT-insert lineage): a SHIFT claim step whose
+// source node v of checkpoint c' holds no first-occurrence data takes the address of the
+// corresponding chunk x of checkpoint c': inside a FIRST region of diff c', its data; inside
+// a SHIFT region of diff c', that step's own resolved address in c''s claim list. v's range
+// is non-FIXED in c' (every leaf below v was a shifted duplicate), so one of the two holds.
+// For c' = this diff the source's steps belong to smaller regions: one pass resolves one
+// more level; steps still unresolved after the last pass flag the chain as malformed.
+__device__ __forceinline__ uint64_t last_le(const unsigned long long* a, uint64_t n, unsigned long long x) {
+  uint64_t lo = 0, hi = n;   // last index with a[i] <= x (a[0] <= x assumed by the caller)
+  while (hi - lo > 1) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (a[mid] <= x) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__global__ void __launch_bounds__(kRT) resolve_kernel(Geo g, RestoreDiff d, const RestoreDiff* chain, int last, int* err) {
+  const unsigned long long C = g.C;
+  const uint64_t nxF = (d.data_bytes + C - 1) / C, nxS = (d.shift_bytes + C - 1) / C;
+  for (uint64_t t = nxF + (uint64_t)blockIdx.x * kRT + threadIdx.x; t < nxF + nxS; t += (uint64_t)gridDim.x * kRT) {
+    if (d.Csrc[t]) continue;
+    const unsigned long long o = (t - nxF) * C;
+    const uint64_t r = region_at(d.Soff, d.nS, o);
+    const uint8_t* e = d.base + 64 + 4 * d.nF + 12 * r;
+    const uint32_t u = rd32(e), v = rd32(e + 4), c2 = rd32(e + 8);
+    uint64_t ulo, uhi, vlo, vhi;
+    node_range(g, u, ulo, uhi);
+    node_range(g, v, vlo, vhi);
+    const uint64_t x = vlo + (d.Cch[t] - ulo);
+    const RestoreDiff& s = chain[c2 <= d.id ? c2 : d.id];
+    unsigned long long addr = 0;
+    bool found = false;
+    if (s.nF && s.Flo[0] <= x) {
+      const uint64_t f = last_le(s.Flo, s.nF, x);
+      const unsigned long long fend = f + 1 < s.nF ? s.Foff[f + 1] : s.data_bytes;
+      if ((x - s.Flo[f]) * C < fend - s.Foff[f]) {
+        addr = (unsigned long long)(s.base + s.meta_bytes + s.Foff[f]) + (x - s.Flo[f]) * C;
+        found = true;
+      }
+    }
+    if (!found && s.nS && s.Slo[0] <= x) {
+      const uint64_t q = last_le(s.Slo, s.nS, x);
+      if ((x - s.Slo[q]) * C < s.Soff[q + 1] - s.Soff[q]) {
+        const uint64_t sxF = (s.data_bytes + C - 1) / C;
+        addr = s.Csrc[sxF + s.Soff[q] / C + (x - s.Slo[q])];   // 0 while not yet resolved
+        found = true;
+      }
+    }
+    if (addr) d.Csrc[t] = addr;
+    else if (last || !found || c2 > d.id) atomicExch(err, 1);
   }
 }
 
@@ -214,8 +270,14 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
   // plan is flagged and no restore kernel runs
   if (c2 > d.id) { atomicExch(err, 1); d.Ssrc[i] = (unsigned long long)d.base; return; }
   const RestoreDiff& s = chain[c2];
-  // FIRST region r of diff c2 with Flo[r] <= vlo (the last such): it contains v
-  if (s.nF == 0 || !s.Flo) { atomicExch(err, 1); d.Ssrc[i] = (unsigned long long)s.base; return; }
+  // FIRST region r of diff c2 with Flo[r] <= vlo (the last such): it contains v. Under the
+  // SHIFT-insert variant (R25) v may instead be a node of c2 whose bytes are c2's own
+  // regions below it: Ssrc = 0, resolved per chunk after the claim list is built.
+  if (s.nF == 0 || !s.Flo) {
+    if (!d.composite) atomicExch(err, 1);
+    d.Ssrc[i] = d.composite ? 0ull : (unsigned long long)s.base;
+    return;
+  }
   uint64_t lo = 0, hi = s.nF;
   while (hi - lo > 1) {
     const uint64_t mid = (lo + hi) >> 1;
@@ -224,8 +286,8 @@ __global__ void prepare_shift_kernel(Geo g, RestoreDiff d, const RestoreDiff* ch
   const unsigned long long rel = (vlo - s.Flo[lo]) * (unsigned long long)g.C;
   const unsigned long long rend = lo + 1 < s.nF ? s.Foff[lo + 1] : s.data_bytes;
   if (s.Flo[lo] > vlo || s.Foff[lo] + rel + range_bytes(g, vlo, vhi) > rend) {
-    atomicExch(err, 1);
-    d.Ssrc[i] = (unsigned long long)s.base;
+    if (!d.composite) atomicExch(err, 1);
+    d.Ssrc[i] = d.composite ? 0ull : (unsigned long long)s.base;
     return;
   }
   d.Ssrc[i] = (unsigned long long)(s.base + s.meta_bytes + s.Foff[lo] + rel);
@@ -377,6 +439,19 @@ cudaError_t restore_claimlist(const Geo& g, const RestoreDiff& d, int num_sms, c
   return cudaGetLastError();
 }
 
+cudaError_t restore_resolve(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, int passes, int* err,
+                            int num_sms, cudaStream_t st) {
+  const uint64_t nx = (d.shift_bytes + g.C - 1) / g.C;
+  if (nx == 0) return cudaSuccess;
+  uint64_t grid = (nx + kRT - 1) / kRT;
+  if (grid > (uint64_t)num_sms * 8) grid = (uint64_t)num_sms * 8;
+  for (int i = 0; i < passes; ++i) {
+    resolve_kernel<<<(unsigned)grid, kRT, 0, st>>>(g, d, chain_dev, i + 1 == passes ? 1 : 0, err);
+    note_launch();
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st) {
   const uint64_t nx = claim_count(g, d);
   if (nx == 0) return cudaSuccess;
@@ -417,6 +492,7 @@ cudaError_t preload_restore() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_count_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, basic_expand_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, compare_kernel);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, resolve_kernel);
   return e;
 }
 

@@ -29,6 +29,12 @@
 // order (FIRST list, then SHIFT list); an upper-stage region starts at a tile boundary
 // and is recorded in the tile holding its first leaf, so the per-tile lists in tile
 // order are the regions sorted by first chunk (R13) — k_compact.cu relies on it.
+//
+// PHASE 4 (CKPT_VARIANT_SHIFT_INSERT, reading R24 of P:89) runs between the two: pass 1 as
+// phase 3 (the hashes of every POTENTIAL shifted node, i.e. every node whose leaves are all
+// SHIFT), pass 2 inserts them (find-or-claim, then atomicMin over ckpt<<32|node: the
+// minimum node id wins among equal new hashes, an existing entry is never changed, R6).
+// Phase 3 then finds every SHIFT-SHIFT parent; one that finds its own entry is a miss.
 #include "kernels.h"
 #include "tma.cuh"
 
@@ -509,6 +515,9 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
     if (PHASE == 2) {
       F = __ldcg(sp.gm2 + c.G * 32 + lane);
       S = 0;
+    } else if (PHASE == 4) {
+      F = 0;
+      S = __ldcg(sp.gm4 + c.G * 32 + lane);
     } else {
       const uint32_t* gm = sp.gm3 + c.G * 64;
       F = __ldcg(gm + lane);
@@ -547,6 +556,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   ws.W[lane] = 0;
   ws.K[lane] = 0;
   __syncwarp();
+  uint32_t Ptop = 0;   // PHASE 4: potential shifted nodes at the group's top level
   if (__any_sync(0xffffffffu, ((PHASE == 2 ? F : S) | (PHASE == 2 ? lF1 : lS1)) != 0)) {
     uint32_t P = PHASE == 2 ? F : S;
     for (int lv = 1; lv <= gsz; ++lv) {
@@ -596,6 +606,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
       });
       P = work | inj;
     }
+    Ptop = P;
   }
   __syncwarp();
   if (p.trace && lane == 0) ws.tp[1] = gtimer();
@@ -604,7 +615,26 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   // pass 1 resolved from their children's sources)
   ws.H[lane] = PHASE == 3 ? ws.K[lane] : 0u;
   __syncwarp();
-  {
+  if (PHASE == 4) {
+    // R24: every potential shifted node's hash enters the record unless present; the
+    // minimum node id wins among equal new hashes (read first: hot repeated keys, e.g. the
+    // all-zero subtrees of a first checkpoint, meet on one slot)
+    const uint32_t total = batch_begin(ws, ws.W[lane]);
+    for (uint32_t j = lane; j < total; j += 32) {
+      uint32_t iw, ib;
+      batch_item(ws, j, iw, ib);
+      int lv;
+      uint32_t r;
+      lay_decode(iw, ib, lv, r);
+      const Digest d = dig_load(ws, c.tdig, ws.WP[iw] + __popc(ws.W[iw] & ((1u << ib) - 1u)));
+      const uint64_t gpos = (c.G << (gsz - lv)) + rev_n(r, gsz - lv);
+      bool claimed;
+      unsigned long long seen;
+      table_insert_min(p.tab, p.cap, d, pack_entry(g.k, node_id(g, c.Lin + lv, gpos)), &claimed, false, &seen);
+      if (claimed) ++ins_cnt;
+    }
+    __syncwarp();
+  } else {
     constexpr int kB2 = CKPT_TREE_KB2;
     const uint32_t total = batch_begin(ws, PHASE == 3 ? (ws.W[lane] & ~ws.K[lane]) : ws.W[lane]);
     for (uint32_t base = 0; base < total; base += 32 * kB2) {
@@ -665,6 +695,10 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
           if (olo[t] == d[t].lo && ohi[t] == d[t].hi) v = oval[t];
           else if (olo[t] == kEmpty && ohi[t] == kEmpty) v = kEmpty;
           else v = table_lookup_from(p.tab, p.cap, d[t], sl[t] + 1 == p.cap ? 0 : sl[t] + 1);
+          // R24: a node that finds its own entry is the first occurrence of its content
+          if (v != kEmpty && p.shift_insert &&
+              v == pack_entry(g.k, node_id(g, c.Lin + lv, (c.G << (gsz - lv)) + rev_n(r, gsz - lv))))
+            v = kEmpty;
           if (v != kEmpty) {
             atomicOr(&ws.H[iw[t]], 1u << ib[t]);
             c.tsrc[P0 + lvl_off(P0, lv) + r] = v;
@@ -676,7 +710,10 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   }
   if (p.trace && lane == 0) ws.tp[2] = gtimer();
 
-  if (PHASE == 2) {
+  if (PHASE == 4) {
+    F = 0;
+    S = Ptop;   // the group root is a potential shifted node iff bit 0 of lane 0 is set
+  } else if (PHASE == 2) {
     // the FIRST label chain up to the group root (stops once no FIRST node is left)
     for (int lv = 1; lv <= gsz; ++lv) {
       const uint64_t Nc = P0 >> (lv - 1), Np = Nc >> 1;
@@ -735,7 +772,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
   const uint32_t rF = __shfl_sync(0xffffffffu, F, 0) & 1u;
   const uint32_t rS = __shfl_sync(0xffffffffu, S, 0) & 1u;
   const bool last = (c.s == p.S - 1);
-  c.pub = !last && (rF || (PHASE == 3 && rS));
+  c.pub = !last && (rF || (PHASE != 2 && rS));
   if (last) {
     if (PHASE == 3 && lane == 0 && (rF | rS))
       emit_region(c, ws, gsz, 0, rF != 0, rS ? child_src(c, gsz, 0) : 0ull);   // R10
@@ -749,6 +786,12 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
         const Digest d = child_digest(c, ws, gsz, 0);
         reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
         atomicOr(nx.gm2 + Pg * 32 + (rr >> 5), 1u << (rr & 31));
+      }
+    } else if (PHASE == 4) {
+      if (rS) {
+        const Digest d = child_digest(c, ws, gsz, 0);
+        reinterpret_cast<ulonglong2*>(nx.in.dig)[c.G] = make_ulonglong2(d.lo, d.hi);
+        atomicOr(nx.gm4 + Pg * 32 + (rr >> 5), 1u << (rr & 31));
       }
     } else {
       if (rS) {
@@ -857,7 +900,7 @@ __global__ void __launch_bounds__(kTreeThreads, CKPT_TREE_BPS) tree_kernel(const
       // release: only a group that published a root label / digest to the parent has
       // writes the parent's processor reads (nothing else it wrote is read in this kernel)
       if (c.pub) __threadfence();
-      if (lane == 0) old = atomicAdd((PHASE == 2 ? up.arr2 : up.arr3) + P, 1u);
+      if (lane == 0) old = atomicAdd((PHASE == 2 ? up.arr2 : PHASE == 3 ? up.arr3 : up.arr4) + P, 1u);
       old = __shfl_sync(0xffffffffu, old, 0);
       if (old + 1 != target) return;   // not the last full child
       __threadfence();
@@ -924,6 +967,12 @@ __global__ void __launch_bounds__(kTreeThreads, CKPT_TREE_BPS) tree_kernel(const
     w = !CKPT_TREE_CURSOR ? w + nwarps : nwarps < count ? nwarps + __shfl_sync(0xffffffffu, nx, 0) : count;
   }
   const unsigned long long ta = p.trace ? gtime_ns() : 0;
+  if (PHASE == 4) {
+    unsigned long long v = ins;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0 && v) atomicAdd(&s_cnt[3], v);
+  }
   if (PHASE == 2) {
     // warp sums first: 64-bit shared atomics are CAS loops, 256 contending threads serialise
     unsigned long long v[5] = {ins, coll, lc.f, lc.s, lc.t};
@@ -941,6 +990,7 @@ __global__ void __launch_bounds__(kTreeThreads, CKPT_TREE_BPS) tree_kernel(const
   }
   __syncthreads();
   const unsigned long long tb = p.trace ? gtime_ns() : 0;
+  if (threadIdx.x == 0 && PHASE == 4 && s_cnt[3]) atomicAdd(&p.tot->p3_inserts, s_cnt[3]);
   if (threadIdx.x == 0 && PHASE == 2) {
     if (s_cnt[3]) atomicAdd(&p.tot->p2_inserts, s_cnt[3]);
     if (s_cnt[0]) atomicAdd(&p.tot->n_first, s_cnt[0]);
@@ -952,7 +1002,7 @@ __global__ void __launch_bounds__(kTreeThreads, CKPT_TREE_BPS) tree_kernel(const
   trace_block(p.trace, p.trace_n, bt0, bt1, PHASE);
 }
 
-static int g_tree_blocks_per_sm[2] = {0, 0};
+static int g_tree_blocks_per_sm[3] = {0, 0, 0};
 
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st) {
   // all CTAs resident at once (static tile striding relies on it): occupancy-sized grid
@@ -961,6 +1011,7 @@ cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_
   if (grid > p.n_tiles) grid = p.n_tiles ? p.n_tiles : 1;   // worklist spread over blocks first
   const size_t smem = kWarps * sizeof(WarpSmem);
   if (phase == 2) return launch_pdl(tree_kernel<2>, (unsigned)grid, kTreeThreads, smem, st, p);
+  if (phase == 4) return launch_pdl(tree_kernel<4>, (unsigned)grid, kTreeThreads, smem, st, p);
   return launch_pdl(tree_kernel<3>, (unsigned)grid, kTreeThreads, smem, st, p);
 }
 
@@ -968,10 +1019,13 @@ cudaError_t tree_setup_attributes() {
   const int smem = (int)(kWarps * sizeof(WarpSmem));
   cudaError_t e = cudaFuncSetAttribute(tree_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(tree_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(tree_kernel<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess)
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_tree_blocks_per_sm[0], tree_kernel<2>, kTreeThreads, smem);
   if (e == cudaSuccess)
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_tree_blocks_per_sm[1], tree_kernel<3>, kTreeThreads, smem);
+  if (e == cudaSuccess)
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_tree_blocks_per_sm[2], tree_kernel<4>, kTreeThreads, smem);
   return e;
 }
 
@@ -985,6 +1039,7 @@ cudaError_t preload_tree() {
   cudaError_t e = cudaSuccess;
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, tree_kernel<2>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, tree_kernel<3>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, tree_kernel<4>);
   return e;
 }
 

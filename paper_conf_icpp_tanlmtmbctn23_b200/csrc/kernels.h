@@ -34,11 +34,12 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   unsigned long long nF, nS, data_bytes, meta_bytes;
   unsigned long long n_first, n_spatial, n_temporal, p2_inserts;
   unsigned long long collisions, n_cand;
+  unsigned long long p3_inserts;     // CKPT_VARIANT_SHIFT_INSERT: new potential shifted regions (R24)
   unsigned long long full_kind;      // 0, or the difference is stored in full: 1 = full first
                                      // checkpoint, 2 = switched (gather kernel, R22 / R23)
   unsigned long long n_nonfixed;     // non-FIXED leaves (K1/K1t, counted only for the switch)
   uint32_t wl_count[kMaxStages];
-  uint32_t tree_next[2];             // work-stealing cursors of the phase-2 / phase-3 kernels
+  uint32_t tree_next[3];             // work-stealing cursors of the phase-2 / phase-3 / phase-3a kernels
   uint32_t gather_next;              // work-stealing cursor of the gather kernel
   uint32_t k1_next;                  // K1 tile cursor (tiles handed out beyond the first wave)
   uint32_t defer_count;              // 256-chunk leaf tiles whose inserts K1 left to K1b
@@ -101,9 +102,11 @@ struct StageParams {
   unsigned long long* tsrc;    // per group: sources of SHIFT nodes (2 * 2^gsz entries)
   uint32_t* arr2;              // s >= 1: arrivals of dirty children, phase 2
   uint32_t* arr3;              //                                     phase 3
+  uint32_t* arr4;              //                                     phase 3a (R24 inserts)
   const uint32_t* dcnt;        // s >= 1: full children per group (K1b)
   uint32_t* gm2;               // s >= 1: per group, 32 words: FIRST children (bit-reversed), phase 2
   uint32_t* gm3;               // s >= 1: per group, 64 words: FIRST / SHIFT children, phase 3
+  uint32_t* gm4;               // s >= 1: per group, 32 words: all-SHIFT children, phase 3a
 };
 
 struct TreeParams {
@@ -126,6 +129,7 @@ struct TreeParams {
   Totals* tot;
   int dbg;                     // diagnostics only (CKPT_DBG bits; 0 in production)
   int list;                    // CKPT_MODE_LIST: no compaction, every FIRST/SHIFT leaf is an entry
+  int shift_insert;            // CKPT_VARIANT_SHIFT_INSERT (R24): a lookup finding its own entry is a miss
   int sw_permille;             // full-change switch threshold (R23), -1 = off
   ulonglong4* trace;           // optional diagnostics (CKPT_TRACE): {t_start, t_end, stage|G, phase}
   uint32_t* trace_n;
@@ -151,6 +155,7 @@ struct CompactParams {
   uint4* ctr_next;               // the next call's counter block, zeroed by the gather kernel
   uint64_t ctr_next_words;
   int mode;                      // CKPT_MODE_*: header flags; Basic writes the bitmap instead of entries
+  int flags;                     // header flags of a Tree / List / Basic difference (= mode, or 4, R24)
   const uint32_t* cand;          // Basic: the changed-chunk bitmap (K1)
   uint64_t nwords;               // Basic: its u32 words
   const uint32_t* tcc;           // Basic: changed chunks per tree tile (K1)
@@ -220,6 +225,7 @@ cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes);
 // ---- restore (k_restore.cu)
 struct RestoreDiff {           // one diff of the chain, as the restore kernels see it (cached plan)
   uint32_t id;                 // its checkpoint id (a SHIFT source must be <= id)
+  uint32_t composite;          // R25: a SHIFT source may lie outside its diff's FIRST regions
   const uint8_t* base;         // diff bytes (device)
   uint64_t nF, nS, meta_bytes, data_bytes;
   unsigned long long* Flo;     // per FIRST region: first chunk (sorted)
@@ -243,6 +249,8 @@ cudaError_t restore_segmaps(RestoreDiff& d, cudaStream_t st);
 cudaError_t device_compare(const void* a, const void* b, uint64_t bytes, int* diff, int num_sms, cudaStream_t st);
 uint64_t restore_segments(uint64_t bytes);
 cudaError_t restore_claimlist(const Geo& g, const RestoreDiff& d, int num_sms, cudaStream_t st);
+cudaError_t restore_resolve(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, int passes, int* err,
+                            int num_sms, cudaStream_t st);
 cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st);
 cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st);
 size_t scan_tmp_bytes_for(uint64_t count);

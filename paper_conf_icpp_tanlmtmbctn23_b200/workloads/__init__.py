@@ -8,7 +8,7 @@ GDV workloads). Every random draw is the counter-based hash
     H(s, a, b, ...) = H(H(s, a), b, ...)
 
 so the host (numpy, this module) and the device (``gen.cu`` → ``libckptgen.so``)
-produce identical bytes independently; ``tests/test_gpu_workloads.py`` checks that.
+produce identical bytes independently; ``tests/test_gpu_api.py::test_device_generators_match_host`` checks that.
 
 Configs (BASELINE.json ``configs``):
   1  sparse random: B=1 MiB, C=128, K=10, 1 % Bernoulli chunk updates

@@ -20,7 +20,7 @@ def _dev(buf: np.ndarray):
 
 
 STAT_KEYS = ["n_first_regions", "n_shift_regions", "n_first", "n_fixed", "n_spatial", "n_temporal",
-             "list_entries", "meta_bytes", "data_bytes", "bytes", "phase2_inserts"]
+             "list_entries", "meta_bytes", "data_bytes", "bytes", "phase2_inserts", "phase3_inserts"]
 
 
 def run_parity(oracle_mod, bufs, C, check_record=True, check_digests=True, check_restore=True, mode=0,

@@ -179,6 +179,8 @@ def main():
             ("var_switch30_cfg2_p0.05", 2, GiB // s, 128, 20, 0.05, None, 0, False, (2, 30)),
             ("var_none_cfg4_dup_heavy", 4, GiB // s, 128, 20, 0.0, "dup", 0, False, None),
             ("var_switch850_cfg4_dup_heavy", 4, GiB // s, 128, 20, 0.0, "dup", 0, False, (2, 850)),
+            ("var_shift_insert_cfg2_p0.01", 2, GiB // s, 128, 20, 0.01, None, 0, False, (4, 1000)),
+            ("var_shift_insert_cfg4_dup_heavy", 4, GiB // s, 128, 20, 0.0, "dup", 0, False, (4, 1000)),
         ]
     recs = []
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
