@@ -158,7 +158,10 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
   // Basic: the changed-chunk bitmap replaces the entry lists (nF_tot = changed chunks)
   const unsigned long long raw = basic ? 64 + 4ull * p.nwords : 64 + 4 * nF_tot + 12 * nS_tot;
   const unsigned long long meta = (raw + 15) & ~15ull;
-  if (blockIdx.x == 0 && wid == 0 && lane == 0 && !full) {
+  // the header is written by a warp without a tile when there is one (the last warp):
+  // the mapped-memory totals and their system-scope fence would otherwise delay a tile
+  const uint64_t hdr_warp = (uint64_t)count * parts < nwarps ? nwarps - 1 : 0;
+  if ((uint64_t)wid * gridDim.x + blockIdx.x == hdr_warp && lane == 0 && !full) {
     // totals and the 64-byte header (R13)
     p.tot->nF = nF_tot; p.tot->nS = nS_tot; p.tot->data_bytes = data_tot; p.tot->meta_bytes = meta;
     if (basic) p.tot->n_first = nF_tot;   // every changed chunk is stored (no record)
