@@ -198,7 +198,12 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <int MODE3D>
+// UNITS: the 16-byte blocks of a thread's chunk per stage as a compile-time constant (8 for
+// C >= 128; C / 16 for the small chunk sizes C = 32 and 64), 0 = read from p at run time.
+// With it known, each thread's swizzled shared-memory offsets are computed once, outside
+// the stage loop (at C = 32 the per-stage address arithmetic and the generic unit loop were
+// as many instructions as a block of the hash, and K1 is issue-bound there).
+template <int MODE3D, int UNITS>
 __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
@@ -294,9 +299,16 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
 
   // ---------------- consumer (hashing) warps
   const uint64_t pol_keep = policy_evict_last();
-  const int units = MODE3D ? 8 : (int)(p.g.C / 16);   // 16-byte blocks of this thread per stage
+  const int units = UNITS ? UNITS : (int)(p.g.C / 16);   // 16-byte blocks of this thread per stage
   const uint32_t ubase = (uint32_t)tid * (uint32_t)units;
   const int lane = tid & 31, wid = tid >> 5;
+  constexpr int kOffs = UNITS ? UNITS : 1;
+  uint32_t offs[kOffs];   // SWIZZLE_128B offsets of this thread's units within a stage
+#pragma unroll
+  for (int j = 0; j < kOffs; ++j) {
+    const uint32_t u = ubase + j, row = u >> 3;
+    offs[j] = (row << 7) | ((((u & 7) ^ (row & 7))) << 4);
+  }
   uint64_t h1 = 0, h2 = 0;
   int st = 0, seg = 0;
   uint32_t phase = 0;
@@ -306,17 +318,29 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
     if (tile == kNoTile) break;
     if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
     const uint8_t* sd = data + (size_t)st * stage_bytes;
-#pragma unroll 8
-    for (int j = 0; j < units; ++j) {
-      const uint32_t u = ubase + j;
-      const uint32_t row = u >> 3;
-      const uint32_t off = (row << 7) | ((((u & 7) ^ (row & 7))) << 4);   // SWIZZLE_128B
-      const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + off);
+    if (UNITS) {
+#pragma unroll
+      for (int j = 0; j < kOffs; ++j) {
+        const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + offs[j]);
 #ifdef CKPT_K1_NOHASH   // timing experiment only: data movement without the hash
-      h1 ^= v.x; h2 ^= v.y;
+        h1 ^= v.x; h2 ^= v.y;
 #else
-      mm::block(h1, h2, v.x, v.y);
+        mm::block(h1, h2, v.x, v.y);
 #endif
+      }
+    } else {
+#pragma unroll 8
+      for (int j = 0; j < units; ++j) {
+        const uint32_t u = ubase + j;
+        const uint32_t row = u >> 3;
+        const uint32_t off = (row << 7) | ((((u & 7) ^ (row & 7))) << 4);   // SWIZZLE_128B
+        const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + off);
+#ifdef CKPT_K1_NOHASH
+        h1 ^= v.x; h2 ^= v.y;
+#else
+        mm::block(h1, h2, v.x, v.y);
+#endif
+      }
     }
     if (seg == segs - 1) {
       const Digest d = mm::finish(h1, h2, p.g.C);
@@ -548,8 +572,10 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   uint64_t grid = (uint64_t)num_sms * (p.mode3d ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC);
   const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
   if (grid > groups) grid = groups;
-  if (p.mode3d) leaf_hash_kernel<1><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
-  else leaf_hash_kernel<0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  if (p.mode3d) leaf_hash_kernel<1, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  else if (p.g.C == 32) leaf_hash_kernel<0, 2><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  else if (p.g.C == 64) leaf_hash_kernel<0, 4><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  else leaf_hash_kernel<0, 0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   note_launch();
   return cudaGetLastError();
 }
@@ -580,8 +606,10 @@ cudaError_t leaf_setup_attributes() {
   // the largest leaf configuration: kLeafStages3d x (32 KB + 4 KB) when C % 128 == 0, <= 96 KB of stages below
   const int stages = kLeafStages3d * (32768 + 4096) > 98304 + 8 * 4096 ? kLeafStages3d * (32768 + 4096) : 98304 + 8 * 4096;
   const int smem = 1008 + stages + (int)sizeof(K1Shared);
-  cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;
 }
 
@@ -601,8 +629,10 @@ cudaError_t launch_rehash(const Slot* old_tab, uint64_t old_cap, Slot* new_tab, 
 cudaError_t preload_leaf() {
   cudaFuncAttributes a;
   cudaError_t e = cudaSuccess;
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0>);
-  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<1>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0, 2>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0, 4>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0, 0>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<1, 8>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_tail_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, insert_kernel);
   if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_insert_blocks_per_sm, insert_kernel, 256, 0);
