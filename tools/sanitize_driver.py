@@ -4,7 +4,7 @@
     compute-sanitizer --tool {memcheck,racecheck,synccheck} python tools/sanitize_driver.py
 
 config 1 (1 MiB, 10 checkpoints), duplicate-heavy lineages in the Tree / List / Basic
-methods (C = 64, ragged n), the two variants (full first checkpoint, full-change switch),
+methods (C = 64, ragged n), the variants (full first checkpoint, full-change switch, SHIFT-SHIFT insertion),
 a multi-stage tree (n > 2^20 at C = 32), every restore, and a lineage import. Each diff
 is compared with the CPU oracle so a sanitizer run is also a parity run.
 """
@@ -60,6 +60,9 @@ def main():
         run(f"dup_mode{mode}", dup_lineage(11, 3000 * 64 - 5, 64, K=6), 64, mode=mode, check_import=True)
     run("full_first", dup_lineage(12, 2000 * 64, 64, K=4), 64, variant=(1, 1000))
     run("switch", dup_lineage(13, 2000 * 64, 64, K=4, p_change=0.9), 64, variant=(2, 300), check_import=True)
+    run("shift_insert", dup_lineage(14, 2000 * 64 - 3, 64, K=4, alphabet=2), 64, variant=(4, 1000), check_import=True)
+    run("shift_insert_zero", [np.zeros(4096 * 32, dtype=np.uint8), np.full(4096 * 32, 3, dtype=np.uint8)], 32,
+        variant=(4, 1000))
     run("config2_small", list(W.lineage(2, (1 << 22) + 100, 128, 4, p=0.05)), 128)
     if os.environ.get("SAN_BIG", "1") == "1":
         run("multistage_C32", list(W.lineage(1, (1 << 25) + 100, 32, 3, p=0.01)), 32)
