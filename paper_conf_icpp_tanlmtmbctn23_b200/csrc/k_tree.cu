@@ -88,6 +88,7 @@ struct WarpSmem {
   uint32_t H[32];       // pass-2 lookup hits (same layout)
   uint32_t K[32];       // phase 3: level-1 pairs resolved without a lookup (same layout)
   uint16_t items[1 << kTileLog];   // the set bits of the current work mask as a list (word << 5 | bit)
+  uint32_t dense;                  // list_bits: the set bits were exactly 0 .. total-1 (no list written)
   Digest dig[kDigCap];  // compact on-chip digests of pass-1 nodes (rank < kDigCap; others: global)
   uint8_t lvl[1 << kTileLog];   // level of the region starting at each slot
   unsigned long long tp[8];     // diagnostics: intra-group timestamps
@@ -149,8 +150,17 @@ __device__ __forceinline__ uint32_t list_bits(WarpSmem& ws, uint32_t m) {
     if (lane >= o) incl += v;
   }
   const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-  uint32_t r = incl - cnt;
-  for (uint32_t x = m; x; x &= x - 1) ws.items[r++] = (uint16_t)(lane * 32 + (__ffs(x) - 1));
+  // dense masks (every position 0 .. total-1 set, e.g. every level of a fully changed
+  // tile): item j is position j, and the serial per-bit list (12 % of phase 3's
+  // instructions on the duplicate-heavy config) is skipped
+  const uint32_t q0 = (uint32_t)lane * 32;
+  const uint32_t want = q0 < total ? low_mask(total - q0) : 0u;
+  const bool dense = __all_sync(0xffffffffu, m == want);
+  if (!dense) {
+    uint32_t r = incl - cnt;
+    for (uint32_t x = m; x; x &= x - 1) ws.items[r++] = (uint16_t)(lane * 32 + (__ffs(x) - 1));
+  }
+  if (lane == 0) ws.dense = dense ? 1u : 0u;
   __syncwarp();
   return total;
 }
@@ -163,7 +173,7 @@ __device__ __forceinline__ void for_each_bit_balanced(WarpSmem& ws, uint32_t m, 
   if (!__any_sync(0xffffffffu, m != 0)) return;   // most levels have no work: one vote, no scan
   const uint32_t total = list_bits(ws, m);
   for (uint32_t j = lane; j < total; j += 32) {
-    const uint32_t q = ws.items[j];
+    const uint32_t q = ws.dense ? j : ws.items[j];
     f(q >> 5, q & 31u, q);
   }
   __syncwarp();
@@ -178,7 +188,7 @@ __device__ __forceinline__ uint32_t batch_begin(WarpSmem& ws, uint32_t m) {
 }
 // item j (< total) -> (word, bit)
 __device__ __forceinline__ void batch_item(const WarpSmem& ws, uint32_t j, uint32_t& w, uint32_t& b) {
-  const uint32_t q = ws.items[j];
+  const uint32_t q = ws.dense ? j : ws.items[j];
   w = q >> 5;
   b = q & 31u;
 }
