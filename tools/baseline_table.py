@@ -1,6 +1,7 @@
 #!/usr/bin/env python
-"""Regenerates BASELINE.md §3's results rows from profiles/ (sweep_r1.json, bench_r1.json,
-bench_cfg1_r1.json, oracle_time_r1.json) and MEASURED_PEAKS.json:
+"""Regenerates BASELINE.md §3's results rows from profiles/ (sweep_rN.json, bench_rN.json,
+bench_cfg1_rN.json, oracle_time_rN.json of the latest round that has each file) and
+MEASURED_PEAKS.json:
     python tools/baseline_table.py            # rewrites the table rows in place"""
 import json
 import os
@@ -9,11 +10,19 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 P = lambda *a: os.path.join(ROOT, *a)
 
 
+def latest(stem):
+    for r in (3, 2, 1):
+        f = P("profiles", f"{stem}_r{r}.json")
+        if os.path.exists(f):
+            return f
+    raise FileNotFoundError(stem)
+
+
 def main():
-    sw = {r["case"]: r for r in json.load(open(P("profiles", "sweep_r1.json")))}
-    bench = json.loads(open(P("profiles", "bench_r1.json")).read())
-    c1 = json.loads(open(P("profiles", "bench_cfg1_r1.json")).read())
-    ot = {c["case"]: c for c in json.load(open(P("profiles", "oracle_time_r1.json")))["cases"]}
+    sw = {r["case"]: r for r in json.load(open(latest("sweep")))}
+    bench = json.loads(open(latest("bench")).read())
+    c1 = json.loads(open(latest("bench_cfg1")).read())
+    ot = {c["case"]: c for c in json.load(open(latest("oracle_time")))["cases"]}
     try:
         meas = json.load(open(P("MEASURED_PEAKS.json")))["hbm_gbs"]
     except Exception:
