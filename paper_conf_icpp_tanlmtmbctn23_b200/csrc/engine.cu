@@ -43,8 +43,11 @@ struct DiffRec {
   bool planned = false;
 };
 
+#ifndef CKPT_K1_C32_SMEM
+#define CKPT_K1_C32_SMEM 49152      // K1 stage budget per CTA when C = 32 (data + digests; 4 CTAs per SM)
+#endif
 #ifndef CKPT_K1_SMALLC_SMEM
-#define CKPT_K1_SMALLC_SMEM 65536   // K1 stage budget per CTA when C < 128 (data + digests; 3 CTAs per SM)
+#define CKPT_K1_SMALLC_SMEM 65536   // K1 stage budget per CTA when 32 < C < 128 (3 CTAs per SM)
 #endif
 #ifndef CKPT_K1_GRAB_BYTES
 #define CKPT_K1_GRAB_BYTES 32768
@@ -699,7 +702,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     lp.mode3d = 0;
     lp.segs = 1;
     lp.stage_bytes = kLeafThreads * h->C;
-    lp.nst = (int)std::min<uint64_t>(8, std::max<uint64_t>(2, CKPT_K1_SMALLC_SMEM / (lp.stage_bytes + kLeafThreads * 16)));
+    const uint64_t budget = h->C == 32 ? CKPT_K1_C32_SMEM : CKPT_K1_SMALLC_SMEM;
+    lp.nst = (int)std::min<uint64_t>(8, std::max<uint64_t>(2, budget / (lp.stage_bytes + kLeafThreads * 16)));
     lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
   } else {
     lp.n_main = 0;   // odd chunk sizes above 128 B: direct-load pass only

@@ -181,6 +181,9 @@ constexpr int kMaxStagesK1 = 8;
 #ifndef CKPT_K1_CTAS
 #define CKPT_K1_CTAS 2   // resident K1 CTAs per SM when C % 128 == 0 (3 stages of 36 KB each)
 #endif
+#ifndef CKPT_K1_CTAS_C32
+#define CKPT_K1_CTAS_C32 4      // C = 32: 4 CTAs per SM with 48 KB of stages each (issue-bound: one
+#endif                          // more CTA of hashing warps, 274 -> 255 us per GiB; neutral at C = 64)
 #ifndef CKPT_K1_CTAS_SMALLC
 #define CKPT_K1_CTAS_SMALLC 3   // C < 128: a tile is only 256 C bytes and one producer thread per
 #endif                          // CTA bounds the rate (C = 32: 2 CTAs 320 us, 3 CTAs 288 us / GiB)
@@ -204,7 +207,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 // the stage loop (at C = 32 the per-stage address arithmetic and the generic unit loop were
 // as many instructions as a block of the hash, and K1 is issue-bound there).
 template <int MODE3D, int UNITS>
-__global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
+__global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : (UNITS == 2 ? CKPT_K1_CTAS_C32 : CKPT_K1_CTAS_SMALLC)) leaf_hash_kernel(const __grid_constant__ CUtensorMap tmap, LeafParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-B alignment for the 128B swizzle atom, kept as a shared-space pointer (LDS, not LD)
   const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -316,7 +319,7 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
     mbar_wait(&sh.full[st], phase);
     const uint32_t tile = sh.tile[st];
     if (tile == kNoTile) break;
-    if (seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1)
+    if (!MODE3D || seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1); C < 128: one stage per chunk
     const uint8_t* sd = data + (size_t)st * stage_bytes;
     if (UNITS) {
 #pragma unroll
@@ -342,7 +345,7 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : CKPT_K1_CT
 #endif
       }
     }
-    if (seg == segs - 1) {
+    if (!MODE3D || seg == segs - 1) {
       const Digest d = mm::finish(h1, h2, p.g.C);
       const uint64_t c = (uint64_t)tile * kLeafThreads + tid;
       Digest pd{0, 0};
@@ -559,6 +562,10 @@ __global__ void rehash_kernel(const Slot* old_tab, uint64_t old_cap, Slot* new_t
 }
 
 // ------------------------------------------------------------------ launchers
+int leaf_ctas_per_sm(int mode3d, uint32_t C) {
+  return mode3d ? CKPT_K1_CTAS : (C == 32 ? CKPT_K1_CTAS_C32 : CKPT_K1_CTAS_SMALLC);
+}
+
 cudaError_t leaf_smem_config(const LeafParams& p, size_t* smem_bytes) {
   *smem_bytes = 1008 + (size_t)p.nst * p.stage_bytes + (size_t)p.nst * kLeafThreads * 16 + sizeof(K1Shared);
   return cudaSuccess;
@@ -569,7 +576,7 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   size_t smem;
   leaf_smem_config(p, &smem);
   const uint64_t n_tiles = p.n_main / kLeafThreads;
-  uint64_t grid = (uint64_t)num_sms * (p.mode3d ? CKPT_K1_CTAS : CKPT_K1_CTAS_SMALLC);
+  uint64_t grid = (uint64_t)num_sms * leaf_ctas_per_sm(p.mode3d, p.g.C);
   const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
   if (grid > groups) grid = groups;
   if (p.mode3d) leaf_hash_kernel<1, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);

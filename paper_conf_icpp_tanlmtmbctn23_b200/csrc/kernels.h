@@ -214,6 +214,7 @@ cudaError_t preload_tree();
 cudaError_t preload_compact();
 cudaError_t preload_restore();
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
+int leaf_ctas_per_sm(int mode3d, uint32_t C);   // resident K1 CTAs per SM for chunk size C
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
 cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st);
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st);
