@@ -147,16 +147,22 @@ CKPT_API int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out);
 CKPT_API int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_permille);
 
 /* De-duplicate one checkpoint (Alg.1; serialization P:81).
- *   dev_ptr  device buffer of `bytes` bytes, 16-byte aligned, BORROWED for the call; the
- *            caller must not modify it until the call returns.
+ *   dev_ptr  device buffer of `bytes` bytes, 16-byte aligned, BORROWED: the call's kernels on
+ *            `stream` read it; modify it only with work ordered after them (later work on
+ *            `stream`, or after synchronising `stream`).
  *   bytes    B >= 1 with ceil(B / C) <= 2^31; every checkpoint of a handle must have the
  *            same B (R17: the fixed-duplicate test is positional).
  *   stream   cudaStream_t (as void*) all GPU work is enqueued on, in order.
  *   diff     receives the statistics and the device pointer of the new diff.
- * The call returns after exactly one host synchronisation with `stream` (a spin on the
- * completion the last kernel publishes to mapped host memory; the process
- * "stops during checkpointing"); a call that grows the record table does so in
- * stream order on `stream` and still synchronises once (ckpt_host_syncs). Capacity for the
+ * The call returns after exactly one host wait (ckpt_host_syncs): a spin on the flag the last
+ * kernel publishes to mapped host memory as soon as the checkpoint's statistics are final —
+ * after phases 2 and 3, when the gather kernel has summed the region counts (the process
+ * "stops during checkpointing"). The rest of that kernel (writing the entries and data
+ * of the diff) completes in stream order on `stream`: every later call of this library that
+ * reads the lineage (the next ckpt_checkpoint on any stream, ckpt_diff_to_host[_async],
+ * ckpt_restore[_stream], ckpt_import, the introspection calls) first waits on it (a stream
+ * wait on an event, not a host wait); other readers of diff->dev_ptr order themselves after
+ * `stream`. A call that grows the record table does so in stream order on `stream`. Capacity for the
  * record table and the diff is reserved before the first kernel, so an error leaves the
  * lineage unchanged (CKPT_ECOLLIDE is a committed checkpoint, see above).
  * Errors: CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ESTATE, CKPT_ECOLLIDE. */

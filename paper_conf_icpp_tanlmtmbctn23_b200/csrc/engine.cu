@@ -124,6 +124,11 @@ struct ckpt_ctx {
   RestoreDiff* rs_chain = nullptr;
   uint64_t rs_chain_cap = 0;
   cudaStream_t internal = nullptr;
+  // completion of the latest ckpt_checkpoint's work (its gather kernel finishes writing the
+  // diff after the call has returned on the statistics): every later consumer of the lineage
+  // (the next checkpoint on any stream, D2H copies, restores, introspection) waits on it
+  cudaEvent_t done_ev = nullptr;
+  bool done_ev_valid = false;
   uint64_t launches = 0;         // kernels this handle has enqueued (all calls)
   uint64_t host_syncs = 0;       // host waits on the device this handle has performed (all calls)
   int prof = 0;                  // 0 off, 1 K1 + whole call, 2 every phase
@@ -160,6 +165,11 @@ namespace {
 cudaError_t sync_stream(ckpt_ctx* h, cudaStream_t st) {
   ++h->host_syncs;
   return cudaStreamSynchronize(st);
+}
+
+// Order `st` after the latest checkpoint's kernels (no host wait).
+cudaError_t after_last_checkpoint(ckpt_ctx* h, cudaStream_t st) {
+  return h->done_ev_valid ? cudaStreamWaitEvent(st, h->done_ev, 0) : cudaSuccess;
 }
 
 template <class T>
@@ -503,6 +513,7 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
   // ckpt_leaf_digests touch memory on it (ckpt.h ordering contract).
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamDefault) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaHostAlloc(&h->tot_host, sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  if (cudaEventCreateWithFlags(&h->done_ev, cudaEventDisableTiming) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   std::memset(h->tot_host, 0, sizeof(Totals));   // done = 0: no call completed yet (epochs start at 1)
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
     h->ev_id[r] = -1;
@@ -530,6 +541,7 @@ int ckpt_destroy(ckpt_handle h) {
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r)
     for (int i = 0; i < 6; ++i) if (h->evr[r][i]) cudaEventDestroy(h->evr[r][i]);
   if (h->internal) cudaStreamDestroy(h->internal);
+  if (h->done_ev) cudaEventDestroy(h->done_ev);
   cudaGetLastError();
   delete h;
   return CKPT_OK;
@@ -576,6 +588,7 @@ int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
   float t[12] = {};
   if (h->ev_id[r] == (int64_t)id) {
     cudaEvent_t* e = h->evr[r];
+    cudaEventSynchronize(e[5]);   // the call returned on its statistics; its kernels may still run
     if (h->ev_level[r] >= 2) {
       for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], e[i], e[i + 1]);   // K1, K1b, phase 2, phase 3, compaction
     } else {
@@ -724,6 +737,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   // keeps only the events around K1 (the first kernel) and at the end of the call
   const bool pe = h->prof >= 2;
   const auto t_pre = clk::now();
+  CK(after_last_checkpoint(h, st));   // the previous call's gather may still be finishing
   if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 32 * kTraceLanes, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
@@ -803,6 +817,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.full_first = (h->variant & CKPT_VARIANT_FULL_FIRST) && k == 0;   // R22
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
+  CK(cudaEventRecord(h->done_ev, st));
+  h->done_ev_valid = true;
   const auto t_launched = clk::now();
   // The one host synchronisation of the call: spin on the completion epoch the last gather
   // block writes to mapped memory (measured ~8 us per call sooner than
@@ -831,6 +847,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
 
   const Totals t = *h->tot_host;   // written by the gather kernel (mapped host memory)
   if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
+    CK(sync_stream(h, st));
     std::vector<uint32_t> cnt(8 * kTraceLanes);
     cudaMemcpy(cnt.data(), h->trace_n, cnt.size() * 4, cudaMemcpyDeviceToHost);
     std::vector<ulonglong4> tr;
@@ -873,6 +890,7 @@ int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capac
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
+  CK(after_last_checkpoint(h, h->internal));
   CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, h->internal));   // one D2H
   CK(sync_stream(h, h->internal));
   return CKPT_OK;
@@ -884,6 +902,7 @@ int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
+  CK(after_last_checkpoint(h, static_cast<cudaStream_t>(stream)));
   CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, static_cast<cudaStream_t>(stream)));
   return CKPT_OK;
 }
@@ -901,6 +920,7 @@ int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, vo
     h->staging_size = bytes;
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  CK(after_last_checkpoint(h, st));   // the previous call's kernels may still read the staging buffer
   CK(cudaMemcpyAsync(h->staging, host_ptr, bytes, cudaMemcpyHostToDevice, st));
   int r = ckpt_checkpoint(h, h->staging, bytes, stream, diff);
   if (r != CKPT_OK) return r;
@@ -1131,7 +1151,7 @@ int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stre
   int mismatch = d.bytes != bytes;
   if (!mismatch) {
     int hf = 0;
-    if (cudaMemsetAsync(flag, 0, sizeof(int), in) != cudaSuccess ||
+    if (after_last_checkpoint(h, in) != cudaSuccess || cudaMemsetAsync(flag, 0, sizeof(int), in) != cudaSuccess ||
         device_compare(d.dev_ptr, tmp, bytes, flag, h->num_sms, in) != cudaSuccess ||
         cudaMemcpyAsync(&hf, flag, sizeof(int), cudaMemcpyDeviceToHost, in) != cudaSuccess ||
         sync_stream(h, in) != cudaSuccess) {
@@ -1160,6 +1180,7 @@ int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream)
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   LaunchCount lc(h);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  CK(after_last_checkpoint(h, st));
   const Geo g = make_geo(h, id);
   int rc = ensure_plans(h, id, g, st);
   if (rc != CKPT_OK) {
@@ -1194,6 +1215,7 @@ int ckpt_leaf_digests(ckpt_handle h, void* dev_out) {
   if (!h || !dev_out) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
   if (!h->geo_set) return CKPT_ERANGE;
+  CK(after_last_checkpoint(h, h->internal));
   CK(cudaMemcpyAsync(dev_out, h->prev, h->n * 16, cudaMemcpyDeviceToDevice, h->internal));
   CK(sync_stream(h, h->internal));
   return CKPT_OK;
@@ -1206,6 +1228,7 @@ int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_nodes, ui
   *count = h->live;
   if (!h->tab || cap == 0) return CKPT_OK;
   std::vector<Slot> all(h->cap);
+  CK(after_last_checkpoint(h, h->internal));
   CK(cudaMemcpyAsync(all.data(), h->tab, h->cap * sizeof(Slot), cudaMemcpyDeviceToHost, h->internal));
   CK(sync_stream(h, h->internal));
   uint64_t i = 0;

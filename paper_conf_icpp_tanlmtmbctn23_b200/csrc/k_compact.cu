@@ -46,6 +46,13 @@ __device__ __forceinline__ void host_totals(const CompactParams& p) {
   __threadfence_system();
 }
 
+// The call's statistics are final here (phases 2-3 are complete, the totals are summed): the
+// host may return (one host wait per call, include/ckpt.h). The rest of this kernel (entries,
+// data) completes in stream order; the library's diff consumers wait for it on an event.
+__device__ __forceinline__ void publish_done(const CompactParams& p) {
+  *reinterpret_cast<volatile uint32_t*>(&p.tot_host->done) = p.g.epoch;   // after host_totals' fence
+}
+
 // KG: one WARP per dirty tile (worklist of the phase-2 kernel). Writes the tile's metadata
 // entries (its region records from phase 3) and copies its FIRST bytes. The data section
 // is the FIRST chunks in chunk order (every FIRST leaf lies in exactly one FIRST region,
@@ -117,6 +124,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
       *reinterpret_cast<unsigned long long*>(o + 56) = 0;  // hash seed, reserved
       *reinterpret_cast<uint4*>(o + 64) = make_uint4(0, 0, 0, 0);   // root entry (node 0) + pad
       host_totals(p);
+      publish_done(p);
     }
     // the whole buffer, 16-byte units, kFullUnroll loads in flight per thread before the
     // stores (2 CTAs x 256 threads per SM: 64 KB in flight per SM covers HBM latency)
@@ -180,6 +188,7 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     *reinterpret_cast<uint32_t*>(o + 60) = 0;            // reserved
     for (unsigned long long x = raw; x < meta; ++x) o[x] = 0;
     host_totals(p);
+    publish_done(p);
   }
   if (basic) {   // the bitmap: K1's candidate words, all n bits
     uint32_t* bm = reinterpret_cast<uint32_t*>(p.out + 64);
@@ -334,18 +343,6 @@ __global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
     }
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
-    // The last block to finish publishes completion to the host: every byte of the diff is
-    // written and every read of the caller's buffer is done. Blocks arrive with a gpu-scope
-    // fence (cumulative through the arrival counter); only the last one issues the system-
-    // scope fence before the epoch.
-    __threadfence();
-    if (atomicAdd(&p.tot->blocks_done, 1u) + 1 == gridDim.x) {
-      __threadfence();
-      __threadfence_system();   // block 0's mapped totals (written early) before the epoch
-      *reinterpret_cast<volatile uint32_t*>(&p.tot_host->done) = g.epoch;
-    }
-  }
   trace_block(p.trace, p.trace_n, bt0, bt1, 5);
 }
 

@@ -44,7 +44,7 @@ struct Totals {                      // per-checkpoint device counters (zeroed e
   uint32_t k1_next;                  // K1 tile cursor (tiles handed out beyond the first wave)
   uint32_t defer_count;              // 256-chunk leaf tiles whose inserts K1 left to K1b
   uint32_t insert_next;              // work-stealing cursor of K1b
-  uint32_t blocks_done;              // gather blocks finished (the last one publishes `done`)
+  uint32_t spare;
   uint32_t done;                     // host copy: epoch of the last completed call (spin-wait target)
 };
 

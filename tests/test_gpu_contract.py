@@ -161,3 +161,34 @@ def test_restore_ordered_after_caller_stream_work():
         assert rc == 0
         assert torch.equal(out, devs[k]), k
     ck.close()
+
+
+def test_calls_ordered_across_streams_after_early_return(oracle_mod):
+    """ckpt_checkpoint returns once the statistics are final while its last kernel may still
+    write the diff: consecutive checkpoints on different streams, the D2H copies and a restore
+    issued right after each call must still see complete diffs (the library orders them after
+    the call's completion event)."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    B, C = (1 << 22) + 48, 128
+    bufs = list(W.lineage(2, B, C, 6, p=0.05))
+    devs = [torch.from_numpy(b).cuda() for b in bufs]
+    torch.cuda.synchronize()
+    o = oracle_mod.Oracle(C)
+    ck = Checkpointer(C)
+    streams = [torch.cuda.Stream() for _ in range(3)]
+    pinned = torch.empty(B + 64 + 12 * ((B + C - 1) // C) + 16, dtype=torch.uint8).pin_memory()
+    out = torch.empty(B, dtype=torch.uint8, device="cuda")
+    for k, t in enumerate(devs):
+        o.checkpoint(bufs[k])
+        s = streams[k % 3]
+        d = ck.checkpoint(t, stream=s)
+        side = streams[(k + 1) % 3]
+        ck.diff_to_host_async(k, pinned, side, nbytes=d["bytes"])   # another stream, right away
+        side.synchronize()
+        assert bytes(pinned[: d["bytes"]].numpy()) == o.diff(k), k
+        assert ck.diff_to_host(k) == o.diff(k), k
+    for k in range(len(devs)):
+        ck.restore(k, out)
+        assert torch.equal(out, devs[k]), k
+    ck.close()
