@@ -181,6 +181,9 @@ constexpr int kMaxStagesK1 = 8;
 #ifndef CKPT_K1_CTAS
 #define CKPT_K1_CTAS 2   // resident K1 CTAs per SM when C % 128 == 0 (3 stages of 36 KB each)
 #endif
+#ifndef CKPT_K1_PDL
+#define CKPT_K1_PDL 1           // K1 launched with programmatic stream serialization (see pdl_wait)
+#endif
 #ifndef CKPT_K1_CTAS_C32
 #define CKPT_K1_CTAS_C32 4      // C = 32: 4 CTAs per SM with 48 KB of stages each (issue-bound: one
 #endif                          // more CTA of hashing warps, 274 -> 255 us per GiB; neutral at C = 64)
@@ -232,6 +235,10 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : (UNITS == 
     fence_mbar_init();
   }
   __syncthreads();
+  // K1 is launched with programmatic stream serialization: its CTAs may be set up while the
+  // previous call's gather kernel drains (that call has already returned on its statistics);
+  // nothing of the previous call's memory is touched before this wait
+  pdl_wait();
 
   if (tid >= kLeafThreads) {
     // ---------------- producer warp (lane 0)
@@ -579,12 +586,20 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   uint64_t grid = (uint64_t)num_sms * leaf_ctas_per_sm(p.mode3d, p.g.C);
   const uint64_t groups = (n_tiles + p.tpg - 1) / p.tpg;
   if (grid > groups) grid = groups;
+#if CKPT_K1_PDL
+  const CUtensorMap tm = *tmap;
+  if (p.mode3d) return launch_pdl(leaf_hash_kernel<1, 8>, (unsigned)grid, kK1Threads, smem, st, tm, p);
+  if (p.g.C == 32) return launch_pdl(leaf_hash_kernel<0, 2>, (unsigned)grid, kK1Threads, smem, st, tm, p);
+  if (p.g.C == 64) return launch_pdl(leaf_hash_kernel<0, 4>, (unsigned)grid, kK1Threads, smem, st, tm, p);
+  return launch_pdl(leaf_hash_kernel<0, 0>, (unsigned)grid, kK1Threads, smem, st, tm, p);
+#else
   if (p.mode3d) leaf_hash_kernel<1, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else if (p.g.C == 32) leaf_hash_kernel<0, 2><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else if (p.g.C == 64) leaf_hash_kernel<0, 4><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else leaf_hash_kernel<0, 0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   note_launch();
   return cudaGetLastError();
+#endif
 }
 
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
