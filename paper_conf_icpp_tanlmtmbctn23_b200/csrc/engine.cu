@@ -126,9 +126,13 @@ struct ckpt_ctx {
   cudaStream_t internal = nullptr;
   // completion of the latest ckpt_checkpoint's work (its gather kernel finishes writing the
   // diff after the call has returned on the statistics): every later consumer of the lineage
-  // (the next checkpoint on any stream, D2H copies, restores, introspection) waits on it
+  // on another stream (the next checkpoint, D2H copies, restores, introspection) waits for
+  // the stream the call ran on. The event is recorded lazily, when such a consumer comes:
+  // an event between the gather and the next call's K1 on the same stream would stop K1's
+  // programmatic early launch
   cudaEvent_t done_ev = nullptr;
-  bool done_ev_valid = false;
+  cudaStream_t last_stream = nullptr;
+  bool pending = false;
   uint64_t launches = 0;         // kernels this handle has enqueued (all calls)
   uint64_t host_syncs = 0;       // host waits on the device this handle has performed (all calls)
   int prof = 0;                  // 0 off, 1 K1 + whole call, 2 every phase
@@ -167,9 +171,14 @@ cudaError_t sync_stream(ckpt_ctx* h, cudaStream_t st) {
   return cudaStreamSynchronize(st);
 }
 
-// Order `st` after the latest checkpoint's kernels (no host wait).
+// Order `st` after the latest checkpoint's kernels (no host wait). On the stream that call
+// ran on, stream order does it; elsewhere an event recorded now on that stream (it follows
+// the call's kernels, and possibly later work of the caller there: correct, at worst early).
 cudaError_t after_last_checkpoint(ckpt_ctx* h, cudaStream_t st) {
-  return h->done_ev_valid ? cudaStreamWaitEvent(st, h->done_ev, 0) : cudaSuccess;
+  if (!h->pending || st == h->last_stream) return cudaSuccess;
+  cudaError_t e = cudaEventRecord(h->done_ev, h->last_stream);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(st, h->done_ev, 0);
+  return e;
 }
 
 template <class T>
@@ -817,8 +826,8 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.full_first = (h->variant & CKPT_VARIANT_FULL_FIRST) && k == 0;   // R22
   CK(launch_compact(cp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[5], st));
-  CK(cudaEventRecord(h->done_ev, st));
-  h->done_ev_valid = true;
+  h->last_stream = st;
+  h->pending = true;
   const auto t_launched = clk::now();
   // The one host synchronisation of the call: spin on the completion epoch the last gather
   // block writes to mapped memory (measured ~8 us per call sooner than
