@@ -345,7 +345,12 @@ int make_tmap(ckpt_ctx* h, const void* buf, const LeafParams& lp, CUtensorMap* m
   cuuint32_t box[3];
   cuuint32_t es[3] = {1, 1, 1};
   cuuint32_t rank;
-  if (lp.mode3d) {
+  if (lp.mode3d == 2) {   // rows of C bytes; a box past C is zero-filled (not read)
+    rank = 2;
+    dims[0] = h->C; dims[1] = lp.n_main;
+    strides[0] = h->C;
+    box[0] = 128; box[1] = kLeafThreads;
+  } else if (lp.mode3d) {
     rank = 3;
     dims[0] = 128; dims[1] = h->C / 128; dims[2] = lp.n_main;
     strides[0] = 128; strides[1] = h->C;
@@ -356,8 +361,12 @@ int make_tmap(ckpt_ctx* h, const void* buf, const LeafParams& lp, CUtensorMap* m
     strides[0] = 128;
     box[0] = 128; box[1] = lp.stage_bytes / 128;
   }
+  // MODE3D 2: a chunk row starts anywhere in a 128-B line, and 256-B promotion fetched lines of
+  // the neighbouring rows early (K1 at C = 176: 0.265 ms/GiB with 256-B, 0.221 with 128-B promotion)
+  const CUtensorMapL2promotion promo =
+      lp.mode3d == 2 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B;
   CUresult r = h->encode(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, rank, const_cast<void*>(buf), dims, strides, box, es,
-                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, promo,
                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? CKPT_OK : CKPT_ECUDA;
 }
@@ -727,8 +736,18 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     const uint64_t budget = h->C == 32 ? CKPT_K1_C32_SMEM : CKPT_K1_SMALLC_SMEM;
     lp.nst = (int)std::min<uint64_t>(8, std::max<uint64_t>(2, budget / (lp.stage_bytes + kLeafThreads * 16)));
     lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
+  } else if (h->C < 1024 && h->C % 128 >= 32) {
+    // C > 128, not a multiple of 128: ceil(C / 128) segments, the last one partial. Not kept
+    // when that segment is a single 16-B unit (a pipeline step for 16 bytes: slower than the
+    // direct-load pass, e.g. C = 144, 1040) nor at C > 1024 (the direct pass was as fast);
+    // DESIGN.md §5, K1 design
+    lp.mode3d = 2;
+    lp.segs = (int)((h->C + 127) / 128);
+    lp.stage_bytes = 128 * kLeafThreads;
+    lp.nst = kLeafStages3d;
+    lp.n_main = (n_full / kLeafThreads) * kLeafThreads;
   } else {
-    lp.n_main = 0;   // odd chunk sizes above 128 B: direct-load pass only
+    lp.n_main = 0;   // the direct-load pass only
   }
   lp.tail_begin = lp.n_main;
   // one cursor grab per >= 32 KB of input (CKPT_K1_GRAB_BYTES): a tile is 256 C bytes

@@ -204,6 +204,10 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
+// MODE3D: 1 = C % 128 == 0 (3-D map: 128-B row r of 256 chunks per stage); 2 = C > 128 not a
+// multiple of 128 (2-D map of C-byte rows, the same 128-B boxes; the last one runs past the
+// chunk's end, which TMA fills with zeros without reading, and hashes only its C mod 128 bytes);
+// 0 = C < 128 (whole chunks in 2-D rows).
 // UNITS: the 16-byte blocks of a thread's chunk per stage as a compile-time constant (8 for
 // C >= 128; C / 16 for the small chunk sizes C = 32 and 64), 0 = read from p at run time.
 // With it known, each thread's swizzled shared-memory offsets are computed once, outside
@@ -280,8 +284,11 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : (UNITS == 
       sh.tile[s] = tile;
       sh.tile_end[s] = (int)seg == segs - 1;
       mbar_arrive_expect_tx(&sh.full[s], stage_bytes + (with_prev ? kLeafThreads * 16u : 0u));
-      if (MODE3D)
+      if (MODE3D == 1)
         tma_load_3d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, (int)seg, (int)(tile * kLeafThreads), pol_stream);
+      else if (MODE3D == 2)   // box (128 B, 256 chunks) at byte seg * 128 of each chunk row; past C: zero fill
+        tma_load_2d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], (int)(seg * 128), (int)(tile * kLeafThreads),
+                    pol_stream);
       else
         tma_load_2d(data + (size_t)s * stage_bytes, &tmap, &sh.full[s], 0, (int)(tile * (stage_bytes / 128)), pol_stream);
       if (with_prev)
@@ -329,8 +336,11 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : (UNITS == 
     if (!MODE3D || seg == 0) { h1 = 0; h2 = 0; }   // seed 0 (R1); C < 128: one stage per chunk
     const uint8_t* sd = data + (size_t)st * stage_bytes;
     if (UNITS) {
+      // MODE3D 2: the chunk's last segment holds (C mod 128) / 16 units
+      const int nu = (MODE3D == 2 && seg == segs - 1) ? (int)((p.g.C & 127u) >> 4) : kOffs;
 #pragma unroll
       for (int j = 0; j < kOffs; ++j) {
+        if (MODE3D == 2 && j >= nu) break;
         const ulonglong2 v = *reinterpret_cast<const ulonglong2*>(sd + offs[j]);
 #ifdef CKPT_K1_NOHASH   // timing experiment only: data movement without the hash
         h1 ^= v.x; h2 ^= v.y;
@@ -588,12 +598,14 @@ cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sm
   if (grid > groups) grid = groups;
 #if CKPT_K1_PDL
   const CUtensorMap tm = *tmap;
+  if (p.mode3d == 2) return launch_pdl(leaf_hash_kernel<2, 8>, (unsigned)grid, kK1Threads, smem, st, tm, p);
   if (p.mode3d) return launch_pdl(leaf_hash_kernel<1, 8>, (unsigned)grid, kK1Threads, smem, st, tm, p);
   if (p.g.C == 32) return launch_pdl(leaf_hash_kernel<0, 2>, (unsigned)grid, kK1Threads, smem, st, tm, p);
   if (p.g.C == 64) return launch_pdl(leaf_hash_kernel<0, 4>, (unsigned)grid, kK1Threads, smem, st, tm, p);
   return launch_pdl(leaf_hash_kernel<0, 0>, (unsigned)grid, kK1Threads, smem, st, tm, p);
 #else
-  if (p.mode3d) leaf_hash_kernel<1, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  if (p.mode3d == 2) leaf_hash_kernel<2, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
+  else if (p.mode3d) leaf_hash_kernel<1, 8><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else if (p.g.C == 32) leaf_hash_kernel<0, 2><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else if (p.g.C == 64) leaf_hash_kernel<0, 4><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
   else leaf_hash_kernel<0, 0><<<(unsigned)grid, kK1Threads, smem, st>>>(*tmap, p);
@@ -629,6 +641,7 @@ cudaError_t leaf_setup_attributes() {
   const int stages = kLeafStages3d * (32768 + 4096) > 98304 + 8 * 4096 ? kLeafStages3d * (32768 + 4096) : 98304 + 8 * 4096;
   const int smem = 1008 + stages + (int)sizeof(K1Shared);
   cudaError_t e = cudaFuncSetAttribute(leaf_hash_kernel<1, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<2, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(leaf_hash_kernel<0, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -655,6 +668,7 @@ cudaError_t preload_leaf() {
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0, 4>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<0, 0>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<1, 8>);
+  if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_hash_kernel<2, 8>);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, leaf_tail_kernel);
   if (e == cudaSuccess) e = cudaFuncGetAttributes(&a, insert_kernel);
   if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&g_insert_blocks_per_sm, insert_kernel, 256, 0);

@@ -80,7 +80,8 @@ struct LeafParams {
   uint64_t n_main;       // chunks handled by the TMA pipeline (multiple of 256)
   uint64_t tail_begin;   // first chunk of the direct-load tail pass
   int segs;              // 128-B rows per chunk (C >= 128) or 1
-  int mode3d;            // 1: C % 128 == 0 (3-D map: row r of 256 chunks); 0: C < 128 (2-D rows)
+  int mode3d;            // 1: C % 128 == 0 (3-D map: row r of 256 chunks); 2: other C > 128 (2-D map of
+                         // chunk rows, 128-B boxes, zero-filled past C); 0: C < 128 (2-D rows)
   uint32_t stage_bytes;  // TMA bytes per pipeline stage
   int nst;               // pipeline stages
   uint32_t tpg;          // tiles per cursor grab (>= 1; more at small C, see the K1 producer)

@@ -111,6 +111,26 @@ def test_random_dup_lineages_odd_sizes(oracle_mod, seed):
     run_parity(oracle_mod, bufs, C)
 
 
+@pytest.mark.parametrize("C", [144, 160, 192, 240, 272, 400, 1040, 2064])
+def test_partial_segment_chunk_sizes(oracle_mod, C):
+    """C > 128 and not a multiple of 128 (K1 MODE3D 2: a 2-D map of C-byte rows read in 128-B
+    boxes, the last one zero-filled past C and hashed over C mod 128 bytes only): many
+    256-chunk tiles through the TMA pipeline, a ragged tail tile and a short last chunk."""
+    rng = np.random.default_rng(C)
+    n = 256 * (37 if C < 1024 else 9) + 101
+    nbytes = n * C - int(rng.integers(1, C))
+    bufs = dup_lineage(C, nbytes, C, K=4, alphabet=6)
+    run_parity(oracle_mod, bufs, C)
+
+
+@pytest.mark.parametrize("C", [160, 400])
+def test_partial_segment_config2(oracle_mod, C):
+    """The config-2 recipe (GDV-like, p = 1 %) at 32 MiB with a partial-segment chunk size."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    bufs = list(W.lineage(2, 1 << 25, C, 4))
+    run_parity(oracle_mod, bufs, C)
+
+
 def test_all_zero_and_unchanged(oracle_mod):
     C = 64
     z = np.zeros(1000 * C, dtype=np.uint8)
