@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--inplace", action="store_true",
                     help="one buffer mutated between steps (automatic when the lineage does not fit)")
+    ap.add_argument("--sync", action="store_true",
+                    help="time one ckpt_checkpoint at a time (default for resident lineages: pipelined "
+                         "ckpt_checkpoint_submit / _wait, two checkpoints in flight)")
     ap.add_argument("--dist-selftest", action="store_true", help=argparse.SUPPRESS)
     return ap.parse_args()
 
@@ -339,10 +342,26 @@ def run_ours(args):
     # the timed handle records no library events: an event after K1 stops K1b's programmatic
     # early launch (PDL) and cost ~6 us per step; K1's duration for the roofline comes from a
     # replay of the same steps with events around K1 and the whole call only (level 1)
+    pipe = not inplace and not args.sync
+
+    def run_steps(h, ks, out, raw_out):
+        """Checkpoints ks of the lineage on handle h: pipelined (submit k, then collect k - 1)
+        or one call at a time."""
+        if not pipe:
+            for k in ks:
+                out.append(h.checkpoint(lin.get(k), nbytes=B, stream=stream, raw=raw_out))
+            return
+        pend = None
+        for k in ks:
+            cid = h.submit(lin.get(k), nbytes=B, stream=stream)
+            if pend is not None:
+                out.append(h.wait(pend, stream=stream, raw=raw_out))
+            pend = cid
+        out.append(h.wait(pend, stream=stream, raw=raw_out))
+
     diffs = []
     ck0 = None
-    for k in range(Wm):
-        diffs.append(ck.checkpoint(lin.get(k), nbytes=B, stream=stream))
+    run_steps(ck, range(Wm), diffs, False)
     n = (B + C - 1) // C
     k1_ms, phase = [], []
     raw = []
@@ -353,9 +372,8 @@ def run_ours(args):
         if not inplace:
             ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             ev0.record(stream)
-            for k in range(Wm, Wm + K):
-                raw.append(ck.checkpoint(lin.get(k), nbytes=B, stream=stream, raw=True))
-            ev1.record(stream)
+            run_steps(ck, range(Wm, Wm + K), raw, True)
+            ev1.record(stream)   # after the last wait: `stream` follows every call's work
             stream.synchronize()
             ms_local = ev0.elapsed_time(ev1)
         else:
@@ -377,6 +395,24 @@ def run_ours(args):
     ms = max_over_ranks(ms_local, ws)
     total_bytes = sum_over_ranks(float(K * B), ws)
     value = total_bytes / (ms / 1e3) / 1e9
+    # the same K steps one call at a time (a fresh handle replaying the lineage), for comparison
+    sync_res = None
+    if pipe:
+        cks1 = Checkpointer(C)
+        for k in range(Wm):
+            cks1.checkpoint(lin.get(k), nbytes=B, stream=stream)
+        barrier(ws)
+        torch.cuda.synchronize()
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        for k in range(Wm, Wm + K):
+            cks1.checkpoint(lin.get(k), nbytes=B, stream=stream, raw=True)
+        s1.record(stream)
+        stream.synchronize()
+        sms = max_over_ranks(s0.elapsed_time(s1), ws)
+        sync_res = {"value": round(total_bytes / (sms / 1e3) / 1e9, 3), "ms_per_step": round(sms / K, 4),
+                    "note": "the same steps through ckpt_checkpoint, one call at a time"}
+        cks1.close()
     # K1 and whole-call device times: the same lineage replayed on a second handle at
     # profiling level 1 (CUDA events around K1 and around the whole call, on `stream`),
     # timed like the main region (W untimed warm-up checkpoints, then the K steps)
@@ -580,6 +616,10 @@ def run_ours(args):
             "steps": K, "warmup": Wm, "ms_per_step": round(ms / K, 4), "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
             "config": workload_config(args, ws, inplace),
+            "calls": ("pipelined: ckpt_checkpoint_submit of step k+1, then ckpt_checkpoint_wait of step k "
+                      "(two checkpoints in flight; the diffs are bit-identical to one call at a time)"
+                      if pipe else "one ckpt_checkpoint at a time (returns on the checkpoint's statistics)"),
+            "sync": sync_res,
             "per_gpu_gbs": round(value / ws, 3),
             "hbm_frac_of_measured": round((value / ws) * (1 + 16 / C) / peak, 4),
             "roofline": {"bound": "hbm", "kernel": "leaf_hash_kernel (K1)", "achieved": round(achieved, 1),

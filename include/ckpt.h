@@ -168,6 +168,34 @@ CKPT_API int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_per
  * Errors: CKPT_EINVAL, CKPT_ENOMEM, CKPT_ECUDA, CKPT_ESTATE, CKPT_ECOLLIDE. */
 CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff);
 
+/* Pipelined de-duplication of a lineage: the same checkpoint as ckpt_checkpoint, enqueued
+ * without waiting for its statistics, so that checkpoint k + 1's leaf pass (K1, HBM-bound)
+ * runs while checkpoint k's record and tree phases (latency-bound, "waves") do. The
+ * method's arithmetic and every result are those of ckpt_checkpoint (the diffs are
+ * bit-identical); only the overlap of consecutive calls differs.
+ *   dev_ptr, bytes  as ckpt_checkpoint. BORROWED until ckpt_checkpoint_wait(id) returns AND
+ *                   the caller's later work is ordered after the stream passed to it.
+ *   stream          cudaStream_t (as void*) the leaf pass is enqueued on; the record and tree
+ *                   phases and the gather run on an internal non-blocking stream of the handle,
+ *                   ordered after it by events.
+ *   id              receives the checkpoint id (= the number of checkpoints before it).
+ * At most two calls are in flight: a submit with two outstanding first collects the older
+ * (a host wait). Every other call of this library (ckpt_checkpoint, diff access, restore,
+ * import, introspection) first collects all outstanding calls, oldest first.
+ * Errors: as ckpt_checkpoint (an error of the collected older call is returned here). */
+CKPT_API int ckpt_checkpoint_submit(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, uint32_t* id);
+
+/* Collect checkpoint `id` (and every older outstanding one): returns its statistics once they
+ * are final (one host wait per collected call, ckpt_host_syncs), like ckpt_checkpoint.
+ *   stream  cudaStream_t (as void*) made to wait (an event, not a host wait) for the rest of
+ *           call id's work (the gather of its entries and data, which reads the buffer);
+ *           enqueue reuse of the buffer or reads of diff->dev_ptr after it. May be the
+ *           stream of a later submit: that call's leaf pass is already enqueued before it.
+ *   diff    receives the statistics and the device pointer of diff `id`.
+ * Errors: CKPT_ERANGE (id not submitted), CKPT_EINVAL, CKPT_ECUDA, CKPT_ESTATE,
+ * CKPT_ECOLLIDE (committed, R14). */
+CKPT_API int ckpt_checkpoint_wait(ckpt_handle h, uint32_t id, void* stream, ckpt_diff* diff);
+
 /* Rebuild checkpoint `id` into the caller's device buffer ("start from the
  * first-time occurrences, then fill the fixed duplicates and finally assemble the shifted
  * duplicates from the corresponding checkpoint ID"). Equivalent to replaying diffs 0..id

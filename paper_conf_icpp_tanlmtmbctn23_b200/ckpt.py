@@ -25,7 +25,8 @@ CKPT_FLAGS_FULL = 3                                           # header flags of 
 CKPT_FLAGS_SHIFT_INSERT = 4                                   # header flags under the SHIFT-insert variant
 
 ABI_FUNCTIONS = [
-    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_restore",
+    "ckpt_create", "ckpt_create_mode", "ckpt_set_variant", "ckpt_checkpoint", "ckpt_checkpoint_submit",
+    "ckpt_checkpoint_wait", "ckpt_restore",
     "ckpt_restore_stream", "ckpt_diff_info", "ckpt_diff_to_host", "ckpt_diff_to_host_async",
     "ckpt_checkpoint_host", "ckpt_import", "ckpt_num_checkpoints", "ckpt_leaf_digests", "ckpt_record_dump",
     "ckpt_set_profiling", "ckpt_phase_times", "ckpt_phase_times_of", "ckpt_kernel_launches",
@@ -85,6 +86,8 @@ def lib() -> ctypes.CDLL:
             "ckpt_create_mode": ([u32, i32, P(vp)], i32),
             "ckpt_set_variant": ([vp, u32, u32], i32),
             "ckpt_checkpoint": ([vp, vp, u64, vp, P(CkptDiff)], i32),
+            "ckpt_checkpoint_submit": ([vp, vp, u64, vp, P(u32)], i32),
+            "ckpt_checkpoint_wait": ([vp, u32, vp, P(CkptDiff)], i32),
             "ckpt_restore": ([vp, u32, vp], i32),
             "ckpt_restore_stream": ([vp, u32, vp, vp], i32),
             "ckpt_diff_info": ([vp, u32, P(CkptDiff)], i32),
@@ -158,6 +161,8 @@ class Checkpointer:
         self.chunk_bytes = chunk_bytes
         self.mode = mode
         self._ckpt_fn = lib().ckpt_checkpoint   # bound once: the per-call path is marshalling only
+        self._submit_fn = lib().ckpt_checkpoint_submit
+        self._wait_fn = lib().ckpt_checkpoint_wait
 
     def set_variant(self, flags: int, switch_permille: int = 1000) -> None:
         """CKPT_VARIANT_FULL_FIRST / CKPT_VARIANT_FULL_SWITCH (Tree mode, before the first
@@ -175,6 +180,27 @@ class Checkpointer:
             if rc == CKPT_ECOLLIDE:   # committed with a warning (include/ckpt.h, R14)
                 return self._collided(d, raw)
             raise CkptError(rc, "ckpt_checkpoint")
+        return d if raw else d.as_dict()
+
+    def submit(self, buf, nbytes: int | None = None, stream=None) -> int:
+        """Pipelined checkpoint (include/ckpt.h ckpt_checkpoint_submit): enqueue and return the
+        id; collect it with wait(). The buffer stays borrowed until wait(id) returns."""
+        cid = ctypes.c_uint32()
+        n = _nbytes(buf) if nbytes is None else nbytes
+        rc = self._submit_fn(self._h, _ptr(buf), n, _stream_handle(stream), ctypes.byref(cid))
+        if rc != CKPT_OK:
+            raise CkptError(rc, "ckpt_checkpoint_submit")
+        return cid.value
+
+    def wait(self, cid: int, stream=None, raw: bool = False):
+        """Statistics of submitted checkpoint `cid` (ckpt_checkpoint_wait); `stream` (default:
+        torch's current stream) is ordered after the rest of that call's work."""
+        d = CkptDiff()
+        rc = self._wait_fn(self._h, cid, _stream_handle(stream), ctypes.byref(d))
+        if rc != CKPT_OK:
+            if rc == CKPT_ECOLLIDE:
+                return self._collided(d, raw)
+            raise CkptError(rc, "ckpt_checkpoint_wait")
         return d if raw else d.as_dict()
 
     @staticmethod

@@ -15,6 +15,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <deque>
 #include <new>
 #include <vector>
 
@@ -41,6 +42,17 @@ struct DiffRec {
   unsigned long long* Csrc = nullptr;
   unsigned long long shift_bytes = 0;
   bool planned = false;
+  bool collided = false;                // CKPT_ECOLLIDE: committed with a skipped insert (R14)
+};
+
+// A checkpoint whose kernels are enqueued and whose statistics the host has not collected
+// (ckpt_checkpoint_submit; ckpt_checkpoint collects its own before returning).
+struct Inflight {
+  uint32_t k = 0;
+  uint8_t* out = nullptr;            // the diff's place in arena[arena]
+  int arena = 0;
+  cudaStream_t wait_st = nullptr;    // queried while waiting (a failed kernel never publishes)
+  std::chrono::steady_clock::time_point t_entry, t_pre, t_launched;
 };
 
 #ifndef CKPT_K1_C32_SMEM
@@ -78,7 +90,11 @@ struct ckpt_ctx {
   uint64_t ngroups[kMaxStages] = {};
   // device state
   Digest* prev = nullptr;
-  uint32_t* cand = nullptr;
+  uint32_t* cand = nullptr;       // = cand2[k & 1] of the current call
+  uint32_t* cand2[2] = {};        // candidate bits per call parity: a pipelined call's K1 writes its own
+                                  // while the previous call's tree phases read theirs
+  Digest* cdig2[2] = {};          // pipelined calls: the candidates' digests of call k (parity k & 1), read
+                                  // by its K1b / tree kernels while the next call's K1 updates prev in place
   uint64_t nwords = 0;
   unsigned long long* res_of = nullptr;   // per chunk (candidates only): K1b's resolution
   LevelIO lvl[kMaxStages] = {};
@@ -94,24 +110,32 @@ struct ckpt_ctx {
   uint32_t* wl0 = nullptr;
   uint32_t* dbits = nullptr;     // dirty bit per stage-0 tree tile (inside ctr: zeroed per call)
   uint32_t* tcc = nullptr;       // candidate leaves per stage-0 tree tile (inside ctr)
-  // Totals + per-stage counters, double-buffered: call k uses ctr2[k & 1] and its last
-  // kernel zeroes ctr2[(k + 1) & 1] for the next call, so no memset precedes K1.
-  uint8_t* ctr2[2] = {};
+  // Totals + per-stage counters, triple-buffered: call k uses ctr3[k % 3] and its last kernel
+  // zeroes ctr3[(k + 2) % 3] (the previous call's, complete by then) for call k + 2, so no
+  // memset precedes K1 and a pipelined call's K1 never meets a buffer still being zeroed.
+  uint8_t* ctr3[3] = {};
   size_t ctr_bytes = 0;
   size_t ctr_dbits_off = 0, ctr_tcc_off = 0, ctr_bsum_off = 0, ctr_gsum_off = 0, ctr_stage_off[kMaxStages] = {};
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
-  uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b
+  uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b (= defer2[k & 1])
+  uint32_t* defer2[2] = {};
   unsigned long long* blocksum = nullptr;
   unsigned long long* gsum = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
-  Totals* tot_host = nullptr;   // pinned + mapped: written by the gather kernel
+  Totals* tot_host2[2] = {};    // pinned + mapped, per call parity: written by the gather kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
   std::vector<void*> retired;    // record tables replaced by a growth (freed by ckpt_destroy)
-  DiffArena arena;
+  DiffArena arena[2];            // diffs; pipelined calls alternate (call k: arena[k & 1])
+  bool arena1_ready = false;
   std::vector<DiffRec> diffs;
+  // pipelining (ckpt_checkpoint_submit): K1 on the caller's stream, K1b .. gather on `cs`
+  std::deque<Inflight> inflight;
+  bool call_pipe[4] = {};        // call k was submitted pipelined (index k & 3)
+  cudaStream_t cs = nullptr;
+  cudaEvent_t ev_k1[2] = {}, ev_chain[2] = {};   // after K1(k) / after gather(k), parity k & 1
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
   // restore state (lazy): chunk owners, plan scratch, the chain's plans on device
@@ -160,6 +184,17 @@ struct ckpt_ctx {
       h->poisoned = true;                                                                   \
       return CKPT_ECUDA;                                                                    \
     }                                                                                       \
+  } while (0)
+
+// Any host thread may call the library: each entry point that touches the device makes the
+// handle's device (its primary context) current first. A thread that has made no CUDA
+// runtime call has no current context, and the driver-API tensor-map encode then fails.
+#define BIND(h)                                                                  \
+  do {                                                                           \
+    if (cudaSetDevice((h)->device) != cudaSuccess) {                             \
+      cudaGetLastError();                                                        \
+      return CKPT_ECUDA;                                                         \
+    }                                                                            \
   } while (0)
 
 namespace {
@@ -232,7 +267,9 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
     if (e != cudaSuccess) return CKPT_ENOMEM; \
   } while (0)
   AL(h->prev, n);
-  AL(h->cand, h->nwords + 32);
+  AL(h->cand2[0], h->nwords + 32);
+  AL(h->cand2[1], h->nwords + 32);
+  h->cand = h->cand2[0];
   AL(h->res_of, n);
   for (int s = 0; s < h->S; ++s) {
     if (s >= 1) {
@@ -264,10 +301,10 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
       off[s] = bytes;
       bytes += (4 + 32 + 64 + 32) * h->ngroups[s] * sizeof(uint32_t);   // arr2 arr3 arr4 dcnt, gm2, gm3, gm4
     }
-    AL(h->ctr2[0], bytes);
-    AL(h->ctr2[1], bytes);
-    if (cudaMemsetAsync(h->ctr2[0], 0, bytes, st) != cudaSuccess || cudaMemsetAsync(h->ctr2[1], 0, bytes, st) != cudaSuccess)
-      return CKPT_ECUDA;
+    for (int i = 0; i < 3; ++i) {
+      AL(h->ctr3[i], bytes);
+      if (cudaMemsetAsync(h->ctr3[i], 0, bytes, st) != cudaSuccess) return CKPT_ECUDA;
+    }
     h->ctr_bytes = bytes;
     h->ctr_dbits_off = dbits_off;
     h->ctr_tcc_off = tcc_off;
@@ -279,7 +316,9 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
   AL(h->tilecnt, n_tiles);
   AL(h->wl0, n_tiles);
   AL(h->lmask, n_tiles * kLmWords);
-  AL(h->defer, n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
+  AL(h->defer2[0], n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
+  AL(h->defer2[1], n / 32 + 16);
+  h->defer = h->defer2[0];
 #undef AL
   if (cudaMemsetAsync(h->tilecnt, 0, n_tiles * sizeof(uint4), st) != cudaSuccess) return CKPT_ECUDA;
   if (h->trace_path) {
@@ -289,7 +328,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
   }
   bool reserved = false;
   for (uint64_t va : kArenaVA)
-    if (va >= 4 * (h->B + 12 * n + 1024) && h->arena.reserve(va)) { reserved = true; break; }
+    if (va >= 4 * (h->B + 12 * n + 1024) && h->arena[0].reserve(va)) { reserved = true; break; }
   if (!reserved) return CKPT_ENOMEM;
   h->geo_set = true;
   return CKPT_OK;
@@ -308,8 +347,11 @@ Geo make_geo(const ckpt_ctx* h, uint32_t k) {
   return g;
 }
 
-int ensure_table(ckpt_ctx* h, cudaStream_t st) {
-  uint64_t need = h->live + 2 * h->n - 1;   // worst case: every node inserted
+int ensure_table(ckpt_ctx* h, cudaStream_t st, bool pipe) {
+  // worst case: every node inserted, by this call and, for pipelined calls, by
+  // the call that may still be in flight (its inserts are not counted in `live` yet); sized
+  // for two from the first pipelined call on, so the growth happens there and not later
+  uint64_t need = h->live + (pipe ? 2 : 1) * (2 * h->n - 1);
   if (h->dbg & 256) need = h->live + h->n / 2;   // diagnostics only: undersized table experiment
   if (h->cap && (double)need <= kMaxLoad * (double)h->cap) return CKPT_OK;
   // geometric growth: at least double, so a lineage whose record keeps growing pays for a
@@ -368,6 +410,7 @@ int make_tmap(ckpt_ctx* h, const void* buf, const LeafParams& lp, CUtensorMap* m
   CUresult r = h->encode(map, CU_TENSOR_MAP_DATA_TYPE_UINT8, rank, const_cast<void*>(buf), dims, strides, box, es,
                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, promo,
                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) fprintf(stderr, "libckpt: cuTensorMapEncodeTiled failed (%d)\n", (int)r);
   return r == CUDA_SUCCESS ? CKPT_OK : CKPT_ECUDA;
 }
 
@@ -476,6 +519,8 @@ bool validate_import_body(const HostGeo& g, const uint8_t* hd, uint32_t id, int 
 
 extern "C" {
 
+static int drain(ckpt_ctx* h);   // collects the calls in flight (ckpt_checkpoint_submit)
+
 const char* ckpt_strerror(int status) {
   switch (status) {
     case CKPT_OK: return "ok";
@@ -522,7 +567,7 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
     delete h;
     return CKPT_ECUDA;
   }
-  if (!h->arena.init(dev)) {
+  if (!h->arena[0].init(dev)) {
     delete h;
     return CKPT_ECUDA;
   }
@@ -530,9 +575,10 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
   // default stream (torch's default) completes before ckpt_restore / ckpt_import /
   // ckpt_leaf_digests touch memory on it (ckpt.h ordering contract).
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamDefault) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  if (cudaHostAlloc(&h->tot_host, sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
+  for (int i = 0; i < 2; ++i)
+    if (cudaHostAlloc(&h->tot_host2[i], sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaEventCreateWithFlags(&h->done_ev, cudaEventDisableTiming) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  std::memset(h->tot_host, 0, sizeof(Totals));   // done = 0: no call completed yet (epochs start at 1)
+  for (int i = 0; i < 2; ++i) std::memset(h->tot_host2[i], 0, sizeof(Totals));   // done = 0: epochs start at 1
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
     h->ev_id[r] = -1;
     for (int i = 0; i < 6; ++i) cudaEventCreate(&h->evr[r][i]);
@@ -543,9 +589,11 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
 
 int ckpt_destroy(ckpt_handle h) {
   if (!h) return CKPT_EINVAL;
+  cudaSetDevice(h->device);
   cudaDeviceSynchronize();
   for (void* p : h->allocs) cudaFree(p);
-  h->arena.release_all();
+  h->arena[0].release_all();
+  if (h->arena1_ready) h->arena[1].release_all();
   for (auto& d : h->diffs)
     for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg,
                     (void*)d.Cch, (void*)d.Csrc})
@@ -554,7 +602,13 @@ int ckpt_destroy(ckpt_handle h) {
     if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
   for (void* q : h->retired) cudaFree(q);
-  if (h->tot_host) cudaFreeHost(h->tot_host);
+  for (int i = 0; i < 2; ++i)
+    if (h->tot_host2[i]) cudaFreeHost(h->tot_host2[i]);
+  for (int i = 0; i < 2; ++i) {
+    if (h->ev_k1[i]) cudaEventDestroy(h->ev_k1[i]);
+    if (h->ev_chain[i]) cudaEventDestroy(h->ev_chain[i]);
+  }
+  if (h->cs) cudaStreamDestroy(h->cs);
   if (h->staging) cudaFree(h->staging);
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r)
     for (int i = 0; i < 6; ++i) if (h->evr[r][i]) cudaEventDestroy(h->evr[r][i]);
@@ -567,7 +621,7 @@ int ckpt_destroy(ckpt_handle h) {
 
 int ckpt_num_checkpoints(ckpt_handle h, uint32_t* count) {
   if (!h || !count) return CKPT_EINVAL;
-  *count = (uint32_t)h->diffs.size();
+  *count = (uint32_t)(h->diffs.size() + h->inflight.size());   // submitted, collected or not
   return CKPT_OK;
 }
 
@@ -586,7 +640,9 @@ int ckpt_host_syncs(ckpt_handle h, uint64_t* count) {
 int ckpt_set_variant(ckpt_handle h, uint32_t flags, uint32_t switch_permille) {
   if (!h) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
-  if (h->mode != kModeTree || !h->diffs.empty() || (flags & ~7u) || switch_permille > 1000) return CKPT_EINVAL;
+  BIND(h);
+  if (h->mode != kModeTree || !h->diffs.empty() || !h->inflight.empty() || (flags & ~7u) || switch_permille > 1000)
+    return CKPT_EINVAL;
   h->variant = flags;
   h->switch_permille = switch_permille;
   return CKPT_OK;
@@ -601,6 +657,8 @@ int ckpt_set_profiling(ckpt_handle h, int enable) {
 
 int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const int r = (int)(id % ckpt_ctx::kEvRing);
   float t[12] = {};
@@ -623,6 +681,8 @@ int ckpt_phase_times_of(ckpt_handle h, uint32_t id, float* times, int n) {
 
 int ckpt_phase_times(ckpt_handle h, float* times, int n) {
   if (!h || !times) return CKPT_EINVAL;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;
   if (h->diffs.empty()) {
     for (int i = 0; i < n && i < 12; ++i) times[i] = 0.f;
     return CKPT_OK;
@@ -638,9 +698,12 @@ struct LaunchCount {
   ~LaunchCount() { h->launches += g_kernel_launches - start; }
 };
 
-// Point the per-call counter views at ctr2[parity].
-static void select_ctr(ckpt_ctx* h, int parity) {
-  uint8_t* c = h->ctr2[parity];
+// Point the per-call views at call k's buffers: counters ctr3[k % 3], candidate bits and
+// deferred tiles of parity k & 1.
+static void select_ctr(ckpt_ctx* h, uint32_t k) {
+  h->cand = h->cand2[k & 1];
+  h->defer = h->defer2[k & 1];
+  uint8_t* c = h->ctr3[k % 3];
   h->tot = reinterpret_cast<Totals*>(c);
   h->dbits = reinterpret_cast<uint32_t*>(c + h->ctr_dbits_off);
   h->tcc = reinterpret_cast<uint32_t*>(c + h->ctr_tcc_off);
@@ -657,45 +720,104 @@ static void select_ctr(ckpt_ctx* h, int parity) {
   }
 }
 
-int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
-  using clk = std::chrono::steady_clock;
+using clk = std::chrono::steady_clock;
+static float ms_since(clk::time_point a, clk::time_point b) { return std::chrono::duration<float, std::milli>(b - a).count(); }
+
+// Pipelined calls only: the chain stream, the events and the second arena (created once).
+static int ensure_pipe_state(ckpt_ctx* h) {
+  if (h->cs) return CKPT_OK;
+  // non-blocking: work on the legacy default stream must not serialise against the chain.
+  // Highest priority: when K1 of the next call and this chain's kernels both wait for SM
+  // resources, the (short, latency-bound) chain kernels are placed first and K1's persistent
+  // CTAs fill the rest, growing back as the chain's CTAs exit
+  int lo = 0, hi = 0;   // numerically lowest = highest priority
+  if (cudaDeviceGetStreamPriorityRange(&lo, &hi) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
+  // (measured: with default priority, config 2 steps were 0.220 ms when the chain won the
+  // race and 0.4-2.4 ms when K1's CTAs starved the chain's statically partitioned K1b and
+  // gather; with the highest priority 0.226-0.228 ms, every run)
+  if (cudaStreamCreateWithPriority(&h->cs, cudaStreamNonBlocking, hi) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
+  for (int i = 0; i < 2; ++i)
+    if (cudaEventCreateWithFlags(&h->ev_k1[i], cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&h->ev_chain[i], cudaEventDisableTiming) != cudaSuccess) {
+      cudaGetLastError();
+      return CKPT_ECUDA;
+    }
+  return CKPT_OK;
+}
+
+// Enqueue checkpoint k = (calls so far) of dev_ptr. Synchronous form: every kernel on `st`,
+// PDL-chained. Pipelined form (pipe): K1 (+ K1t) on `st`, then K1b .. gather on the chain
+// stream h->cs. There K1(k) waits only for K1(k - 1) (the digests it compares with) and for
+// the tree phases of call k - 2 (whose candidate bits, candidate digests, deferred tiles and
+// counters it reuses), so it runs while call k - 1's tree phases do.
+static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStream_t st, bool pipe, Inflight* f) {
   const auto t_entry = clk::now();
-  auto ms_since = [](clk::time_point a, clk::time_point b) { return std::chrono::duration<float, std::milli>(b - a).count(); };
-  if (!h) return CKPT_EINVAL;
-  if (h->poisoned) return CKPT_ESTATE;
-  LaunchCount lc(h);
-  if (!dev_ptr || !diff || bytes == 0 || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
-  if ((bytes + h->C - 1) / h->C > (1ull << 31)) return CKPT_EINVAL;
-  if (h->geo_set && bytes != h->B) return CKPT_EINVAL;   // R17
-  {
-    cudaPointerAttributes pa;
-    if (cudaPointerGetAttributes(&pa, dev_ptr) != cudaSuccess) { cudaGetLastError(); return CKPT_EINVAL; }
-    if (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged) return CKPT_EINVAL;
-  }
-  cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (!h->geo_set) {
     const int r = setup_geometry(h, bytes, st);
     if (r != CKPT_OK) return r;
   }
-  const uint32_t k = (uint32_t)h->diffs.size();
+  const uint32_t k = (uint32_t)(h->diffs.size() + h->inflight.size());
+  int r = CKPT_OK;
+  // the stream of the tree phases and the gather
+  const cudaStream_t cst = pipe ? h->cs : st;
+  if (pipe) {
+    if (!h->cdig2[0]) {
+      if (dalloc(h, &h->cdig2[0], h->n) != cudaSuccess || dalloc(h, &h->cdig2[1], h->n) != cudaSuccess) return CKPT_ENOMEM;
+    }
+    const bool prev_pipe = k > 0 && h->call_pipe[(k - 1) & 3];
+    if (!prev_pipe) {
+      // after a synchronous call (or the first call: the setup memsets on st): both streams
+      // follow everything enqueued so far
+      if (h->pending || k == 0) {
+        const cudaStream_t ls = h->pending ? h->last_stream : st;
+        CK(cudaEventRecord(h->done_ev, ls));
+        if (st != ls) CK(cudaStreamWaitEvent(st, h->done_ev, 0));
+        if (cst != ls) CK(cudaStreamWaitEvent(cst, h->done_ev, 0));
+      }
+    } else {
+      // K1(k) after K1(k - 1) (prev digests, possibly another stream) and after the chain of
+      // call k - 2 (this parity's buffers); the chain follows call k - 1's on h->cs
+      CK(cudaStreamWaitEvent(st, h->ev_k1[(k - 1) & 1], 0));
+      if (k >= 2 && h->call_pipe[(k - 2) & 3]) CK(cudaStreamWaitEvent(st, h->ev_chain[k & 1], 0));
+    }
+  }
   const auto t_tab = clk::now();
-  int r = h->mode == kModeBasic ? CKPT_OK : ensure_table(h, st);   // Basic keeps no record
+  // a growth's rehash runs on the chain stream: after the inserts of a call still in flight
+  r = h->mode == kModeBasic ? CKPT_OK : ensure_table(h, cst, pipe);   // Basic keeps no record
   if (r != CKPT_OK) return r;
   const auto t_arena = clk::now();
   const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
-  if (!h->arena.ensure(worst)) return CKPT_ENOMEM;
+  // pipelined calls alternate between two arenas, so a call's place is known while the
+  // previous call's diff size is not yet; the other arena's last diff (call k - 2) is final
+  const int ai = pipe ? (int)(k & 1) : 0;
+  if (ai == 1 && !h->arena1_ready) {
+    if (!h->arena[1].init(h->device)) return CKPT_ECUDA;
+    bool reserved = false;
+    for (uint64_t va : kArenaVA)
+      if (va >= 4 * (h->B + 12 * h->n + 1024) && h->arena[1].reserve(va)) { reserved = true; break; }
+    if (!reserved) return CKPT_ENOMEM;
+    h->arena1_ready = true;
+  }
+  // pipelined: an arena's first mapping covers two diffs' worst case, so that its next
+  // physical growth (a host cost of 0.5-2 ms, during which a pipelined lineage starves) comes
+  // only after about a buffer's worth of diffs, not at its second call
+  const bool first_map = pipe && h->arena[ai].mapped() == 0 && worst <= (8ull << 30);
+  if (!h->arena[ai].ensure(first_map ? 2 * worst : worst)) return CKPT_ENOMEM;
   h->times[10] = ms_since(t_tab, t_arena);
   h->times[11] = ms_since(t_arena, clk::now());
-  uint8_t* out = h->arena.top_ptr();
+  uint8_t* out = h->arena[ai].top_ptr();
 
   const Geo g = make_geo(h, k);
   const uint8_t* buf = static_cast<const uint8_t*>(dev_ptr);
-  select_ctr(h, (int)(k & 1));
+  select_ctr(h, k);
+  // the leaf digests the chain reads: prev itself, or (pipelined) this call's copy of its
+  // candidates' digests, since the next call's K1 rewrites prev meanwhile
+  Digest* const ldig = pipe ? h->cdig2[k & 1] : h->prev;
 
   // ---- record-insert state (K1's insert warp and K1b)
   InsertParams ip;
   std::memset(&ip, 0, sizeof(ip));
-  ip.g = g; ip.prev = h->prev; ip.cand = h->cand; ip.nwords = h->nwords;
+  ip.g = g; ip.prev = ldig; ip.cand = h->cand; ip.nwords = h->nwords;
   ip.tab = h->tab; ip.cap = h->cap; ip.res_of = h->res_of;
   ip.tot = h->tot;
   ip.defer = h->defer;
@@ -720,6 +842,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   lp.g = g;
   lp.buf = buf;
   lp.prev = h->prev;
+  lp.cdig = pipe ? ldig : nullptr;
   lp.cand = h->cand;
   lp.ins = ip;
   const uint64_t n_full = h->B / h->C;
@@ -765,16 +888,20 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   // keeps only the events around K1 (the first kernel) and at the end of the call
   const bool pe = h->prof >= 2;
   const auto t_pre = clk::now();
-  CK(after_last_checkpoint(h, st));   // the previous call's gather may still be finishing
+  if (!pipe) CK(after_last_checkpoint(h, st));   // the previous call's gather may still be finishing
   if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 32 * kTraceLanes, st));
   if (h->prof) CK(cudaEventRecord(h->ev[0], st));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
   CK(launch_leaf_tail(lp, st));
   CK(launch_leaf(&tmap, lp, h->num_sms, st));
   if (h->prof) CK(cudaEventRecord(h->ev[1], st));
+  if (pipe) {
+    CK(cudaEventRecord(h->ev_k1[k & 1], st));
+    CK(cudaStreamWaitEvent(cst, h->ev_k1[k & 1], 0));
+  }
   // K1b: record insert + tie-break (l.6-19), dirty tiles
-  CK(launch_insert(ip, h->num_sms, st));
-  if (pe) CK(cudaEventRecord(h->ev[2], st));
+  CK(launch_insert(ip, h->num_sms, cst));
+  if (pe) CK(cudaEventRecord(h->ev[2], cst));
 
   // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11
   TreeParams tp;
@@ -785,7 +912,7 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.wl0 = h->wl0;
   tp.buf = buf;
   tp.tcc = h->tcc;
-  tp.cand = h->cand; tp.res_of = h->res_of; tp.prev = h->prev;
+  tp.cand = h->cand; tp.res_of = h->res_of; tp.prev = ldig;
   tp.tab = h->tab; tp.cap = h->cap;
   tp.scratch = h->scratch; tp.tilecnt = h->tilecnt; tp.lmask = h->lmask; tp.tot = h->tot;
   tp.blocksum = h->blocksum;
@@ -812,14 +939,14 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   tp.shift_insert = h->mode == kModeTree && (h->variant & CKPT_VARIANT_SHIFT_INSERT);
   tp.sw_permille = ip.sw_permille;
   if (h->mode != kModeBasic) {   // Basic: no record, no tree
-    CK(launch_tree(tp, 2, h->num_sms, st));
-    if (pe) CK(cudaEventRecord(h->ev[3], st));
-    if (tp.shift_insert) CK(launch_tree(tp, 4, h->num_sms, st));   // R24 inserts, before any lookup
-    CK(launch_tree(tp, 3, h->num_sms, st));
-    if (pe) CK(cudaEventRecord(h->ev[4], st));
+    CK(launch_tree(tp, 2, h->num_sms, cst));
+    if (pe) CK(cudaEventRecord(h->ev[3], cst));
+    if (tp.shift_insert) CK(launch_tree(tp, 4, h->num_sms, cst));   // R24 inserts, before any lookup
+    CK(launch_tree(tp, 3, h->num_sms, cst));
+    if (pe) CK(cudaEventRecord(h->ev[4], cst));
   } else if (pe) {
-    CK(cudaEventRecord(h->ev[3], st));
-    CK(cudaEventRecord(h->ev[4], st));
+    CK(cudaEventRecord(h->ev[3], cst));
+    CK(cudaEventRecord(h->ev[4], cst));
   }
 
   // ---- compaction + serialisation
@@ -831,9 +958,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.lmask = h->lmask;
   cp.out = out; cp.buf = buf;
   cp.trace = h->trace; cp.trace_n = h->trace_n;
-  cp.tot_host = h->tot_host;
+  cp.tot_host = h->tot_host2[k & 1];
   cp.dbg = h->dbg;
-  cp.ctr_next = reinterpret_cast<uint4*>(h->ctr2[(k + 1) & 1]);
+  cp.ctr_next = reinterpret_cast<uint4*>(h->ctr3[(k + 2) % 3]);   // call k - 1's: complete
   cp.ctr_next_words = h->ctr_bytes / 16;
   cp.mode = h->mode;
   cp.flags = tp.shift_insert ? CKPT_FLAGS_SHIFT_INSERT : h->mode;
@@ -843,24 +970,39 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   cp.parts = gather_parts(h->ngroups[0], h->C, h->num_sms);
   cp.sw_permille = ip.sw_permille;
   cp.full_first = (h->variant & CKPT_VARIANT_FULL_FIRST) && k == 0;   // R22
-  CK(launch_compact(cp, h->num_sms, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[5], st));
-  h->last_stream = st;
+  CK(launch_compact(cp, h->num_sms, cst));
+  if (h->prof) CK(cudaEventRecord(h->ev[5], cst));
+  if (pipe) CK(cudaEventRecord(h->ev_chain[k & 1], cst));
+  h->last_stream = cst;
   h->pending = true;
-  const auto t_launched = clk::now();
-  // The one host synchronisation of the call: spin on the completion epoch the last gather
-  // block writes to mapped memory (measured ~8 us per call sooner than
-  // cudaStreamSynchronize). The stream is queried now and then, so a failed kernel (which
-  // never publishes) surfaces as an error instead of a hang.
+  h->call_pipe[k & 3] = pipe;
+  f->k = k;
+  f->out = out;
+  f->arena = ai;
+  f->wait_st = cst;
+  f->t_entry = t_entry;
+  f->t_pre = t_pre;
+  f->t_launched = clk::now();
+  return CKPT_OK;
+}
+
+// Collect a launched call: the one host synchronisation of a call is a spin on the
+// completion epoch the gather kernel writes to mapped memory once the statistics are final
+// (measured ~8 us per call sooner than cudaStreamSynchronize). The stream is queried now and
+// then, so a failed kernel (which never publishes) surfaces as an error instead of a hang.
+static int finish_call(ckpt_ctx* h, const Inflight& f, ckpt_diff* diff) {
+  const uint32_t k = f.k;
+  const uint32_t epoch = k + 1;
+  Totals* const th = h->tot_host2[k & 1];
   {
     ++h->host_syncs;
-    volatile uint32_t* done = &h->tot_host->done;
+    volatile uint32_t* done = &th->done;
     for (uint32_t it = 1;; ++it) {
-      if (*done == g.epoch) break;
+      if (*done == epoch) break;
       if ((it & 1023) == 0) {
-        const cudaError_t q = cudaStreamQuery(st);
+        const cudaError_t q = cudaStreamQuery(f.wait_st);
         if (q == cudaSuccess) {
-          if (*done == g.epoch) break;
+          if (*done == epoch) break;
           fprintf(stderr, "libckpt: stream idle without completion\n");
           h->poisoned = true;
           return CKPT_ECUDA;
@@ -873,9 +1015,9 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
   std::atomic_thread_fence(std::memory_order_acquire);   // the totals after the epoch
   const auto t_synced = clk::now();
 
-  const Totals t = *h->tot_host;   // written by the gather kernel (mapped host memory)
+  const Totals t = *th;   // written by the gather kernel (mapped host memory)
   if (h->trace) {   // diagnostics only: dump {t0, t1, stage<<32|G, phase} records
-    CK(sync_stream(h, st));
+    CK(sync_stream(h, f.wait_st));
     std::vector<uint32_t> cnt(8 * kTraceLanes);
     cudaMemcpy(cnt.data(), h->trace_n, cnt.size() * 4, cudaMemcpyDeviceToHost);
     std::vector<ulonglong4> tr;
@@ -887,26 +1029,107 @@ int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* st
     }
     char path[512];
     snprintf(path, sizeof(path), "%s.%u.bin", h->trace_path, k);
-    if (FILE* f = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), f); fclose(f); }
+    if (FILE* fp = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), fp); fclose(fp); }
   }
   if (h->mode != kModeBasic && t.full_kind != 2) h->live += t.n_first + t.p2_inserts + t.p3_inserts;   // R23: no record op
   DiffRec rec;
-  rec.ptr = out;
-  fill_diff(h, k, t, out, &rec.info);
-  h->arena.commit(rec.info.bytes);
+  rec.ptr = f.out;
+  fill_diff(h, k, t, f.out, &rec.info);
+  rec.collided = t.collisions != 0;
+  h->arena[f.arena].commit(rec.info.bytes);
   h->diffs.push_back(rec);
-  *diff = rec.info;
+  if (diff) *diff = rec.info;
   // host-side timings: [6] entry->first enqueue, [7] enqueue of the sequence, [8] sync wait, [9] post
   const auto t_exit = clk::now();
-  h->times[6] = ms_since(t_entry, t_pre);
-  h->times[7] = ms_since(t_pre, t_launched);
-  h->times[8] = ms_since(t_launched, t_synced);
+  h->times[6] = ms_since(f.t_entry, f.t_pre);
+  h->times[7] = ms_since(f.t_pre, f.t_launched);
+  h->times[8] = ms_since(f.t_launched, t_synced);
   h->times[9] = ms_since(t_synced, t_exit);
-  return t.collisions ? CKPT_ECOLLIDE : CKPT_OK;
+  return rec.collided ? CKPT_ECOLLIDE : CKPT_OK;
+}
+
+// Collect every call still in flight (oldest first). Collisions are committed warnings
+// (kept per diff for ckpt_checkpoint_wait), not errors.
+static int drain(ckpt_ctx* h) {
+  while (!h->inflight.empty()) {
+    const Inflight f = h->inflight.front();
+    h->inflight.pop_front();
+    const int r = finish_call(h, f, nullptr);
+    if (r != CKPT_OK && r != CKPT_ECOLLIDE) return r;
+  }
+  return CKPT_OK;
+}
+
+static int check_buffer(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes) {
+  if (!dev_ptr || bytes == 0 || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
+  if ((bytes + h->C - 1) / h->C > (1ull << 31)) return CKPT_EINVAL;
+  if (h->geo_set && bytes != h->B) return CKPT_EINVAL;   // R17
+  cudaPointerAttributes pa;
+  if (cudaPointerGetAttributes(&pa, dev_ptr) != cudaSuccess) { cudaGetLastError(); return CKPT_EINVAL; }
+  if (pa.type != cudaMemoryTypeDevice && pa.type != cudaMemoryTypeManaged) return CKPT_EINVAL;
+  return CKPT_OK;
+}
+
+int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, ckpt_diff* diff) {
+  if (!h || !diff) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  LaunchCount lc(h);
+  int r = check_buffer(h, dev_ptr, bytes);
+  if (r != CKPT_OK) return r;
+  if ((r = drain(h)) != CKPT_OK) return r;
+  Inflight f;
+  if ((r = launch_call(h, dev_ptr, bytes, static_cast<cudaStream_t>(stream), false, &f)) != CKPT_OK) return r;
+  return finish_call(h, f, diff);
+}
+
+int ckpt_checkpoint_submit(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, uint32_t* id) {
+  if (!h || !id) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  LaunchCount lc(h);
+  int r = check_buffer(h, dev_ptr, bytes);
+  if (r != CKPT_OK) return r;
+  // at most two calls in flight: collect the oldest first
+  while (h->inflight.size() >= 2) {
+    const Inflight f = h->inflight.front();
+    h->inflight.pop_front();
+    r = finish_call(h, f, nullptr);
+    if (r != CKPT_OK && r != CKPT_ECOLLIDE) return r;
+  }
+  if ((r = ensure_pipe_state(h)) != CKPT_OK) return r;
+  Inflight f;
+  if ((r = launch_call(h, dev_ptr, bytes, static_cast<cudaStream_t>(stream), true, &f)) != CKPT_OK) return r;
+  h->inflight.push_back(f);
+  *id = f.k;
+  return CKPT_OK;
+}
+
+int ckpt_checkpoint_wait(ckpt_handle h, uint32_t id, void* stream, ckpt_diff* diff) {
+  if (!h || !diff) return CKPT_EINVAL;
+  if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (id >= h->diffs.size() + h->inflight.size()) return CKPT_ERANGE;
+  while (h->diffs.size() <= id) {
+    const Inflight f = h->inflight.front();
+    h->inflight.pop_front();
+    const int r = finish_call(h, f, nullptr);
+    if (r != CKPT_OK && r != CKPT_ECOLLIDE) return r;
+  }
+  // the rest of call id (its gather) before the caller's later work on `stream`: the event
+  // of this parity follows call id's gather (or a later call's, at worst late)
+  const cudaStream_t ws = static_cast<cudaStream_t>(stream);
+  if (h->call_pipe[id & 3] && ws != h->cs) CK(cudaStreamWaitEvent(ws, h->ev_chain[id & 1], 0));
+  *diff = h->diffs[id].info;
+  return h->diffs[id].collided ? CKPT_ECOLLIDE : CKPT_OK;
 }
 
 int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff) {
   if (!h || !diff) return CKPT_EINVAL;
+  if (!h->inflight.empty()) {
+    BIND(h);
+    if (const int rd = drain(h)) return rd;
+  }
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   *diff = h->diffs[id].info;
   return CKPT_OK;
@@ -915,6 +1138,8 @@ int ckpt_diff_info(ckpt_handle h, uint32_t id, ckpt_diff* diff) {
 int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity) {
   if (!h || !host_ptr) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
@@ -927,6 +1152,8 @@ int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capac
 int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t capacity, void* stream) {
   if (!h || !host_ptr) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
@@ -939,6 +1166,8 @@ int ckpt_checkpoint_host(ckpt_handle h, const void* host_ptr, uint64_t bytes, vo
                          uint64_t host_diff_cap, ckpt_diff* diff) {
   if (!h || !host_ptr || !diff || bytes == 0) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   if (h->geo_set && bytes != h->B) return CKPT_EINVAL;
   if (h->staging_size < bytes) {
     if (h->staging) cudaFree(h->staging);
@@ -1103,6 +1332,8 @@ static void free_plan(DiffRec& d) {
 int ckpt_import(ckpt_handle h, const void* host_diff, uint64_t bytes, void* stream) {
   if (!h || !host_diff || bytes < 64) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   const uint8_t* hd = static_cast<const uint8_t*>(host_diff);
   auto rd32h = [&](size_t o) { uint32_t v; std::memcpy(&v, hd + o, 4); return v; };
   auto rd64h = [&](size_t o) { uint64_t v; std::memcpy(&v, hd + o, 8); return v; };
@@ -1205,6 +1436,8 @@ int ckpt_restore(ckpt_handle h, uint32_t id, void* dev_ptr) {
 int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream) {
   if (!h || !dev_ptr || (reinterpret_cast<uintptr_t>(dev_ptr) & 15)) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   LaunchCount lc(h);
   cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -1242,6 +1475,8 @@ int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream)
 int ckpt_leaf_digests(ckpt_handle h, void* dev_out) {
   if (!h || !dev_out) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   if (!h->geo_set) return CKPT_ERANGE;
   CK(after_last_checkpoint(h, h->internal));
   CK(cudaMemcpyAsync(dev_out, h->prev, h->n * 16, cudaMemcpyDeviceToDevice, h->internal));
@@ -1253,6 +1488,8 @@ int ckpt_record_dump(ckpt_handle h, uint8_t* host_keys, uint32_t* host_nodes, ui
                      uint64_t* count) {
   if (!h || !count) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
+  BIND(h);
+  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
   *count = h->live;
   if (!h->tab || cap == 0) return CKPT_OK;
   std::vector<Slot> all(h->cap);

@@ -377,6 +377,7 @@ __global__ void __launch_bounds__(kK1Threads, MODE3D ? CKPT_K1_CTAS : (UNITS == 
         // (raising the L2 priority of the candidate chunk's own lines for the gather kernel
         // was measured neutral on configs 2 and 4 and is not done)
         st_evict_last_v2(p.prev + c, d.lo, d.hi, pol_keep);   // K1b / the tree kernels re-read it
+        if (p.cdig) st_evict_last_v2(p.cdig + c, d.lo, d.hi, pol_keep);   // pipelined: the chain reads this copy
       }
     }
     __syncwarp();
@@ -429,7 +430,10 @@ __global__ void __launch_bounds__(256) leaf_tail_kernel(LeafParams p) {
     s_w[threadIdx.x >> 5] = mask;
     if (c < p.g.n) p.cand[c >> 5] = mask;
   }
-  if (cand) reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
+  if (cand) {
+    reinterpret_cast<ulonglong2*>(p.prev)[c] = make_ulonglong2(d.lo, d.hi);
+    if (p.cdig) reinterpret_cast<ulonglong2*>(p.cdig)[c] = make_ulonglong2(d.lo, d.hi);
+  }
   const int pc = __syncthreads_count(cand);
   if (pc && threadIdx.x == 0) {
     const uint32_t tile = (uint32_t)((p.tail_begin >> 8) + blockIdx.x);

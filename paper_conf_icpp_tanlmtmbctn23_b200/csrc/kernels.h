@@ -86,6 +86,7 @@ struct LeafParams {
   int nst;               // pipeline stages
   uint32_t tpg;          // tiles per cursor grab (>= 1; more at small C, see the K1 producer)
   Digest* prev;          // persistent leaf digests Tree(leaf), 16 n bytes
+  Digest* cdig;          // pipelined calls: this call's candidate digests (also written here), or null
   uint32_t* cand;        // candidate (non-FIXED) bit per chunk
   InsertParams ins;      // record insert state (K1's producer warp marks/defers, K1b inserts)
 };

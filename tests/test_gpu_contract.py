@@ -192,3 +192,38 @@ def test_calls_ordered_across_streams_after_early_return(oracle_mod):
         ck.restore(k, out)
         assert torch.equal(out, devs[k]), k
     ck.close()
+
+
+def test_calls_from_another_host_thread():
+    """Any host thread may drive a handle (the library binds the handle's device per call): a
+    checkpoint and a restore issued from a fresh thread match the same lineage run inline."""
+    import threading
+    import numpy as np
+    import torch
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    C = 128
+    bufs = [torch.from_numpy(b).cuda() for b in W.lineage(2, 1 << 22, C, 3)]
+    a, b = Checkpointer(C), Checkpointer(C)
+    for x in bufs:
+        a.checkpoint(x)
+    out, err = {}, []
+
+    def work():
+        try:
+            st = torch.cuda.Stream()
+            for x in bufs:
+                b.checkpoint(x, stream=st)
+            r = torch.empty_like(bufs[-1])
+            b.restore(2, r)
+            torch.cuda.synchronize()
+            out["r"] = r.cpu().numpy()
+        except Exception as e:   # surfaced in the main thread
+            err.append(e)
+    t = threading.Thread(target=work)
+    t.start()
+    t.join()
+    assert not err, err
+    for k in range(3):
+        assert a.diff_to_host(k) == b.diff_to_host(k), k
+    assert np.array_equal(out["r"], bufs[-1].cpu().numpy())
