@@ -1,5 +1,6 @@
 #!/bin/bash
-# Round-2 measurement pass: GPU tests, smoke, bench (config 2, config 5 in place, config 1, reference arm),
+# Round-2 measurement pass: GPU tests, smoke, bench (config 2 pipelined and --sync, config 5 in place, config 1,
+# reference arm), pipelined vs synchronous lineages (tools/pipe_probe.py),
 # ncu launch list and full captures (config 2 steady + per-config), sweep (configs 2-5, variants, methods),
 # oracle timing, in-kernel trace, sanitizers.
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu,power.draw --format=csv,noheader
@@ -19,6 +20,10 @@ bash tools/ncu_configs.sh > gpurun_out/ncu_configs.log 2>&1; echo "ncu configs r
 timeout 2400 python tools/sweep.py --out gpurun_out/sweep.json > gpurun_out/sweep.log 2>&1; echo "sweep rc=$?"
 timeout 1500 python tools/sweep.py --variants --out gpurun_out/variants.json > gpurun_out/variants.log 2>&1; echo "variants rc=$?"
 timeout 1500 python tools/sweep.py --methods --out gpurun_out/methods.json > gpurun_out/methods.log 2>&1; echo "methods rc=$?"
+for a in "" "P=0.05" "P=0.001" "C=32 B=4294967296 K=8" "C=4096 B=4294967296 K=8" "CFG=4 K=12"; do
+  env $a STEPS=1 REPS=1 timeout 600 python tools/pipe_probe.py 2>&1 | head -2 | cut -c1-300
+done > gpurun_out/pipeline.txt 2>&1; echo "pipeline rc=$?"; cat gpurun_out/pipeline.txt | grep "sync"
+timeout 600 python bench.py --sync --no-cpu-baseline > gpurun_out/bench_sync.log 2>&1; echo "bench sync rc=$?"
 timeout 900 python tools/oracle_time.py --out gpurun_out/oracle_time.json > gpurun_out/oracle_time.log 2>&1; echo "oracle_time rc=$?"
 CKPT_TRACE=gpurun_out/tr K=6 timeout 300 python tools/profile_step.py > gpurun_out/trace_step.log 2>&1; echo "trace rc=$?"
 python tools/trace_kernels.py gpurun_out/tr > gpurun_out/trace_kernels.txt 2>&1; cat gpurun_out/trace_kernels.txt

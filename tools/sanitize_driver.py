@@ -23,7 +23,7 @@ from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W  # noqa: E402
 from tests._lineages import dup_lineage  # noqa: E402
 
 
-def run(name, bufs, C, mode=0, variant=None, check_import=False):
+def run(name, bufs, C, mode=0, variant=None, check_import=False, pipe=False):
     B = bufs[0].size
     o = oracle.Oracle(C, mode=mode)
     ck = Checkpointer(C, mode)
@@ -31,11 +31,21 @@ def run(name, bufs, C, mode=0, variant=None, check_import=False):
         o.set_variant(*variant)
         ck.set_variant(*variant)
     devs = []
+    pend = None
     for k, b in enumerate(bufs):
         o.checkpoint(b)
         t = torch.from_numpy(np.ascontiguousarray(b)).cuda()
         devs.append(t)
-        ck.checkpoint(t, nbytes=B)
+        if pipe:   # ckpt_checkpoint_submit / _wait, two calls in flight
+            cid = ck.submit(t, nbytes=B)
+            if pend is not None:
+                ck.wait(pend)
+            pend = cid
+        else:
+            ck.checkpoint(t, nbytes=B)
+    if pend is not None:
+        ck.wait(pend)
+    for k in range(len(bufs)):
         assert ck.diff_to_host(k) == o.diff(k), (name, k)
     out = torch.empty(B, dtype=torch.uint8, device="cuda")
     for k in range(len(bufs)):
@@ -64,6 +74,8 @@ def main():
     run("shift_insert_zero", [np.zeros(4096 * 32, dtype=np.uint8), np.full(4096 * 32, 3, dtype=np.uint8)], 32,
         variant=(4, 1000))
     run("config2_small", list(W.lineage(2, (1 << 22) + 100, 128, 4, p=0.05)), 128)
+    run("pipelined_config2", list(W.lineage(2, (1 << 22) + 100, 128, 5, p=0.05)), 128, pipe=True)
+    run("pipelined_dup", dup_lineage(15, 3000 * 64 - 5, 64, K=6, p_change=0.8), 64, pipe=True, check_import=True)
     if os.environ.get("SAN_BIG", "1") == "1":
         run("multistage_C32", list(W.lineage(1, (1 << 25) + 100, 32, 3, p=0.01)), 32)
     print("sanitize driver done", flush=True)
