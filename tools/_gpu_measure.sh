@@ -20,7 +20,7 @@ bash tools/ncu_configs.sh > gpurun_out/ncu_configs.log 2>&1; echo "ncu configs r
 timeout 2400 python tools/sweep.py --out gpurun_out/sweep.json > gpurun_out/sweep.log 2>&1; echo "sweep rc=$?"
 timeout 1500 python tools/sweep.py --variants --out gpurun_out/variants.json > gpurun_out/variants.log 2>&1; echo "variants rc=$?"
 timeout 1500 python tools/sweep.py --methods --out gpurun_out/methods.json > gpurun_out/methods.log 2>&1; echo "methods rc=$?"
-for a in "" "P=0.05" "P=0.001" "C=32 B=4294967296 K=8" "C=4096 B=4294967296 K=8" "CFG=4 K=12"; do
+for a in "" "P=0.05" "P=0.001" "CFG=3 C=32 B=4294967296 K=8" "CFG=3 C=4096 B=4294967296 K=8" "CFG=3 C=128 B=4294967296 K=8" "CFG=4 K=12"; do
   env $a STEPS=1 REPS=1 timeout 600 python tools/pipe_probe.py 2>&1 | head -2 | cut -c1-300
 done > gpurun_out/pipeline.txt 2>&1; echo "pipeline rc=$?"; cat gpurun_out/pipeline.txt | grep "sync"
 timeout 600 python bench.py --sync --no-cpu-baseline > gpurun_out/bench_sync.log 2>&1; echo "bench sync rc=$?"
