@@ -900,7 +900,9 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
     CK(cudaStreamWaitEvent(cst, h->ev_k1[k & 1], 0));
   }
   // K1b: record insert + tie-break (l.6-19), dirty tiles
-  CK(launch_insert(ip, h->num_sms, cst));
+  // pipelined: a plain launch (the chain stream's previous kernel is the last call's gather,
+  // which triggers early; see launch_insert)
+  CK(launch_insert(ip, h->num_sms, cst, !pipe));
   if (pe) CK(cudaEventRecord(h->ev[2], cst));
 
   // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11

@@ -628,15 +628,18 @@ cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st) {
 
 static int g_insert_blocks_per_sm = 0;
 
-cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st) {
+cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st, bool pdl) {
   const uint64_t tiles = (p.nwords + 7) / 8;
   uint64_t blocks = (tiles + 7) / 8 + 1;   // + block 0: tree work description
   if (p.mode == kModeBasic) blocks = 1;    // Basic: no record; only the dirty-tile worklist
   // one resident wave: the deferred work is strided statically over the warps
   const uint64_t wave = (uint64_t)num_sms * (g_insert_blocks_per_sm > 0 ? g_insert_blocks_per_sm : 4);
   if (blocks > wave) blocks = wave;
-  if (blocks) return launch_pdl(insert_kernel, (unsigned)blocks, 256, 0, st, p);
-  return cudaSuccess;
+  if (!blocks) return cudaSuccess;
+  if (pdl) return launch_pdl(insert_kernel, (unsigned)blocks, 256, 0, st, p);
+  insert_kernel<<<(unsigned)blocks, 256, 0, st>>>(p);
+  note_launch();
+  return cudaGetLastError();
 }
 
 cudaError_t leaf_setup_attributes() {

@@ -218,7 +218,11 @@ cudaError_t preload_restore();
 cudaError_t launch_leaf(const CUtensorMap* tmap, const LeafParams& p, int num_sms, cudaStream_t st);
 int leaf_ctas_per_sm(int mode3d, uint32_t C);   // resident K1 CTAs per SM for chunk size C
 cudaError_t launch_leaf_tail(const LeafParams& p, cudaStream_t st);
-cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st);
+// pdl: launched with programmatic stream serialization. Only after K1 / K1t, which never
+// trigger their dependents early: after a gather (the chain stream of pipelined calls) an
+// early launch would let the next call's chain start, and its gather zero the previous
+// call's counters (pre-wait), while that call's phase 3 and gather still run.
+cudaError_t launch_insert(const InsertParams& p, int num_sms, cudaStream_t st, bool pdl);
 cudaError_t launch_tree(const TreeParams& p, int phase, int num_sms, cudaStream_t st);
 cudaError_t launch_compact(const CompactParams& p, int num_sms, cudaStream_t st);
 uint32_t gather_parts(uint64_t n_tiles, uint32_t C, int num_sms);

@@ -221,3 +221,28 @@ def test_pipelined_equals_synchronous_at_1gib():
     assert torch.equal(out, bufs[-1])
     a.close()
     b.close()
+
+
+def test_pipelined_stress_tiny_lineages(oracle_mod):
+    """A 255-chunk lineage (one leaf-tail kernel, microsecond kernels) pipelined 150 times:
+    with K1b launched programmatically after the previous call's gather, the next call's
+    chain could start early and its gather zero the previous call's counters before that
+    call's phase 3 had read them (1 failure in 200 runs before the fix)."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    bufs = dup_lineage(13, 255 * 128 - 116, 128, K=5, alphabet=4, p_change=0.9)
+    o = oracle_mod.Oracle(128)
+    for b in bufs:
+        o.checkpoint(b)
+    want = [o.stats(k) for k in range(len(bufs))]
+    devs = [_dev(b) for b in bufs]
+    torch.cuda.synchronize()
+    for it in range(150):
+        ck = Checkpointer(128)
+        ds = pipelined(ck, devs, bufs[0].size)
+        for k in range(len(bufs)):
+            for key in STAT_KEYS:
+                assert ds[k][key] == want[k][key], (it, k, key)
+        if it % 50 == 0:
+            for k in range(len(bufs)):
+                assert ck.diff_to_host(k) == o.diff(k), (it, k)
+        ck.close()
