@@ -27,7 +27,10 @@ __device__ __forceinline__ void warp_sum3(unsigned long long& a, unsigned long l
 }
 
 
-constexpr int kCT = 256;
+#ifndef CKPT_GATHER_THREADS
+#define CKPT_GATHER_THREADS 256
+#endif
+constexpr int kCT = CKPT_GATHER_THREADS;
 
 // Every counter the host reports is final once the gather kernel runs (tree kernels done,
 // pdl_wait): block 0 copies them to mapped host memory early, in 16-byte stores, and
@@ -82,7 +85,7 @@ __device__ __forceinline__ void cp_async_wait_all() {
   asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
 }
 
-__global__ void __launch_bounds__(kCT, 2) gather_kernel(CompactParams p) {
+__global__ void __launch_bounds__(kCT, 512 / kCT) gather_kernel(CompactParams p) {
   extern __shared__ __align__(16) uint8_t gather_smem[];
   GatherWarp* gsm = reinterpret_cast<GatherWarp*>(gather_smem);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;

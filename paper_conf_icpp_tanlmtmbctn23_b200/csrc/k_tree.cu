@@ -44,7 +44,7 @@ namespace {
 
 constexpr int kWarps = kTreeThreads / 32;
 #ifndef CKPT_TREE_BPS
-#define CKPT_TREE_BPS 2   // tree-kernel launch bound: resident CTAs per SM (register budget)
+#define CKPT_TREE_BPS (512 / CKPT_TREE_THREADS)   // launch bound: 512 threads per SM (<= 128 registers)
 #endif
 #ifndef CKPT_TREE_KB2
 #define CKPT_TREE_KB2 2   // pass-2 record operations per lane in flight (3 and 4 spill: config 4 phase 3 +40-55 %)

@@ -20,7 +20,10 @@ constexpr int kMaxStages = 8;
 constexpr int kTileLog = 10;    // stage-0 tile: 1024 virtual leaf slots
 constexpr int kGroupLog = 10;   // upper stages: 1024 positions per group
 constexpr int kLeafThreads = 256;
-constexpr int kTreeThreads = 256;
+#ifndef CKPT_TREE_THREADS
+#define CKPT_TREE_THREADS 256   // tree-kernel CTA size (experiments: 128 lets a tree CTA sit beside K1's)
+#endif
+constexpr int kTreeThreads = CKPT_TREE_THREADS;
 constexpr int kTilesPerBlock = 1024;  // compaction: tiles per reduce/offsets CTA
 constexpr unsigned long long kResPending = 1ull << 63;   // res_of: value not final after K1b
 constexpr int kModeTree = 0, kModeList = 1, kModeBasic = 2;   // = CKPT_MODE_* (include/ckpt.h)

@@ -43,6 +43,15 @@ def test_our_arm_line_small():
     assert d["gpu_launches"] > 0
     assert d["restore"]["ok"] and d["restart_import"]["ok"] and d["paper_throughput"]["ok"]
     assert set(d["clocks"]) >= {"sm_mhz", "sm_max_mhz", "reasons"}
+    # resident lineage: pipelined calls timed, the one-call-at-a-time value beside them
+    assert d["calls"].startswith("pipelined") and d["sync"]["value"] > 0 and d["sync"]["ms_per_step"] > 0
+
+
+@pytest.mark.gpu
+def test_our_arm_sync_flag():
+    d = _run(["--config", "1", "--bytes", str(1 << 20), "--steps", "4", "--warmup", "3", "--no-cpu-baseline",
+              "--e2e-steps", "1", "--sync"])
+    assert d["calls"].startswith("one ckpt_checkpoint") and d["sync"] is None and d["value"] > 0
 
 
 @pytest.mark.gpu
@@ -53,7 +62,7 @@ def test_our_arm_inplace_config5_form():
               "--no-cpu-baseline"])
     assert BASE_KEYS <= set(d)
     assert d["value"] > 0 and d["n_gpus"] == 1 and d["config"]["buffer_bytes"] == 64 << 20
-    assert "in place" in d["config"]["l2"]
+    assert "in place" in d["config"]["l2"] and d["calls"].startswith("one ckpt_checkpoint")
     assert d["restore"]["ok"] and d["paper_throughput"] is None and d["restart_import"] is None
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 64 << 20
     assert d["gpu_launches"] > 0
