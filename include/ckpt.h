@@ -12,8 +12,9 @@
  * General rules for every function:
  *  - Return value: a CKPT_* status; 0 (CKPT_OK) on success. Nothing is silently degraded
  *    and there is no CPU fallback: without a usable sm_100a GPU, calls fail.
- *  - A handle is bound to the CUDA device current at ckpt_create and is not thread-safe;
- *    different handles (one per GPU / process) are independent.
+ *  - A handle is bound to the CUDA device current at ckpt_create (every call makes that
+ *    device current in the calling thread) and is not thread-safe: any host thread may use
+ *    it, one at a time; different handles (one per GPU / process) are independent.
  *  - After any CUDA failure the handle is poisoned: every later call except ckpt_destroy
  *    returns CKPT_ESTATE.
  *  - "stream" arguments are cudaStream_t values passed as void* (NULL = legacy default

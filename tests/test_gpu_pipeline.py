@@ -246,3 +246,25 @@ def test_pipelined_stress_tiny_lineages(oracle_mod):
             for k in range(len(bufs)):
                 assert ck.diff_to_host(k) == o.diff(k), (it, k)
         ck.close()
+
+
+def test_pipelined_with_profiling_events(oracle_mod):
+    """Profiling level 2 (events between every kernel, on both streams) with pipelined calls:
+    per-phase times are reported and the diffs are still the oracle's."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    bufs = list(W.lineage(2, 1 << 22, 128, 5, p=0.05))
+    o = oracle_mod.Oracle(128)
+    for b in bufs:
+        o.checkpoint(b)
+    for level in (1, 2):
+        ck = Checkpointer(128)
+        ck.set_profiling(level)
+        pipelined(ck, [_dev(b) for b in bufs], bufs[0].size)
+        for k in range(len(bufs)):
+            assert ck.diff_to_host(k) == o.diff(k), (level, k)
+            pt = ck.phase_times(k)
+            assert pt["leaf_hash"] > 0 and pt["total"] >= pt["leaf_hash"], (level, k, pt)
+            if level == 2:
+                assert pt["insert"] > 0 and pt["phase2"] > 0 and pt["phase3"] > 0 and pt["compact"] > 0, pt
+        ck.close()
