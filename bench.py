@@ -566,8 +566,7 @@ def run_ours(args):
     paper = None
     if not inplace:
         ckq = Checkpointer(C)
-        for k in range(Wm):
-            ckq.checkpoint(lin.get(k), nbytes=B, stream=stream)
+        run_steps(ckq, range(Wm), [], True)   # warm-up in the timed form (pipelined: first-call setup)
         sizes = [int(d["bytes"]) for d in steady]   # same lineage -> same diffs as the timed run
         offs = [0]
         for sz in sizes:
@@ -578,9 +577,21 @@ def run_ours(args):
         torch.cuda.synchronize()
         q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         q0.record(stream)
-        for i, k in enumerate(range(Wm, Wm + K)):
-            dq = ckq.checkpoint(lin.get(k), nbytes=B, stream=stream)   # returns with the diff complete
-            ckq.diff_to_host_async(k, hpipe[offs[i]:offs[i + 1]], d2h_stream, nbytes=dq["bytes"])
+        if pipe:   # pipelined calls: diff k's D2H is enqueued as soon as k is collected
+            pend = None
+            for i, k in enumerate(range(Wm, Wm + K)):
+                cid = ckq.submit(lin.get(k), nbytes=B, stream=stream)
+                if pend is not None:
+                    dq = ckq.wait(pend[1], stream=stream)
+                    ckq.diff_to_host_async(pend[1], hpipe[offs[pend[0]]:offs[pend[0] + 1]], d2h_stream,
+                                           nbytes=dq["bytes"])
+                pend = (i, cid)
+            dq = ckq.wait(pend[1], stream=stream)
+            ckq.diff_to_host_async(pend[1], hpipe[offs[pend[0]]:offs[pend[0] + 1]], d2h_stream, nbytes=dq["bytes"])
+        else:
+            for i, k in enumerate(range(Wm, Wm + K)):
+                dq = ckq.checkpoint(lin.get(k), nbytes=B, stream=stream)   # returns with the diff complete
+                ckq.diff_to_host_async(k, hpipe[offs[i]:offs[i + 1]], d2h_stream, nbytes=dq["bytes"])
         q1.record(d2h_stream)
         d2h_stream.synchronize()
         stream.synchronize()

@@ -232,7 +232,9 @@ CKPT_API int ckpt_diff_to_host(ckpt_handle h, uint32_t id, void* host_ptr, uint6
  * with the next de-duplication): enqueues the one device-to-host copy of diff `id` on
  * `stream` (cudaStream_t as void*) and returns. Diffs are immutable and never move, so the
  * copy may run while later ckpt_checkpoint calls de-duplicate on another stream; the host
- * data is valid once `stream` has completed the copy (the caller synchronises it).
+ * data is valid once `stream` has completed the copy (the caller synchronises it). A diff
+ * already collected (ckpt_checkpoint_wait) is copied without collecting the pipelined calls
+ * still in flight; the copy is ordered after that call's gather.
  *   host_ptr  caller-owned PINNED host memory of >= capacity bytes (pageable memory would make
  *             the copy synchronous), borrowed until the copy completes.
  * Errors: CKPT_ERANGE, CKPT_EINVAL (capacity < diff bytes), CKPT_ECUDA, CKPT_ESTATE. */

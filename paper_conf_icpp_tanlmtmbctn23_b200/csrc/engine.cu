@@ -1155,12 +1155,19 @@ int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t
   if (!h || !host_ptr) return CKPT_EINVAL;
   if (h->poisoned) return CKPT_ESTATE;
   BIND(h);
-  if (const int rd = drain(h)) return rd;   // calls in flight are collected first
+  // a collected diff is copied without collecting the calls still in flight (a pipelined
+  // lineage keeps overlapping); an uncollected one is collected first
+  if (id >= h->diffs.size())
+    if (const int rd = drain(h)) return rd;
   if (id >= h->diffs.size()) return CKPT_ERANGE;
   const DiffRec& d = h->diffs[id];
   if (capacity < d.info.bytes) return CKPT_EINVAL;
-  CK(after_last_checkpoint(h, static_cast<cudaStream_t>(stream)));
-  CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, static_cast<cudaStream_t>(stream)));
+  const cudaStream_t ds = static_cast<cudaStream_t>(stream);
+  // after the gather of call id: the event of its parity (re-recorded by a later call of the
+  // same parity at most, which is later still), or the latest call for a synchronous one
+  if (h->call_pipe[id & 3] && ds != h->cs) CK(cudaStreamWaitEvent(ds, h->ev_chain[id & 1], 0));
+  else CK(after_last_checkpoint(h, ds));
+  CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, ds));
   return CKPT_OK;
 }
 

@@ -268,3 +268,38 @@ def test_pipelined_with_profiling_events(oracle_mod):
             if level == 2:
                 assert pt["insert"] > 0 and pt["phase2"] > 0 and pt["phase3"] > 0 and pt["compact"] > 0, pt
         ck.close()
+
+
+def test_async_d2h_of_collected_diffs_keeps_pipelining(oracle_mod):
+    """diff_to_host_async of a collected diff while the next pipelined call is in flight (no
+    collection of that call): every host copy equals the oracle's diff, and the handle still
+    has the newer call outstanding afterwards (one host wait per call in total)."""
+    from paper_conf_icpp_tanlmtmbctn23_b200 import Checkpointer
+    bufs = dup_lineage(21, 3000 * 128 - 9, 128, K=7, alphabet=5, p_change=0.7)
+    o = oracle_mod.Oracle(128)
+    for b in bufs:
+        o.checkpoint(b)
+    ck = Checkpointer(128)
+    devs = [_dev(b) for b in bufs]
+    torch.cuda.synchronize()
+    d2h = torch.cuda.Stream()
+    cap = 64 + 12 * 3000 + 16 + bufs[0].size
+    hosts = [torch.empty(cap, dtype=torch.uint8).pin_memory() for _ in bufs]
+    sizes = {}
+    s0 = ck.host_syncs
+    pend = None
+    for k, t in enumerate(devs):
+        cid = ck.submit(t)
+        if pend is not None:
+            d = ck.wait(pend)
+            sizes[pend] = d["bytes"]
+            ck.diff_to_host_async(pend, hosts[pend], d2h, nbytes=cap)
+        pend = cid
+    assert ck.host_syncs - s0 == len(bufs) - 1          # the newest call is still outstanding
+    d = ck.wait(pend)
+    sizes[pend] = d["bytes"]
+    ck.diff_to_host_async(pend, hosts[pend], d2h, nbytes=cap)
+    d2h.synchronize()
+    for k in range(len(bufs)):
+        assert bytes(hosts[k][:sizes[k]].numpy()) == o.diff(k), k
+    ck.close()
