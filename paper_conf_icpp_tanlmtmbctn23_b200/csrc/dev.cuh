@@ -169,8 +169,27 @@ constexpr unsigned long long kEmpty = ~0ull;
 
 __device__ __forceinline__ uint64_t slot_home(uint64_t klo, uint64_t cap) { return __umul64hi(klo, cap); }
 
-__device__ __forceinline__ void ld_key_relaxed(const Slot* s, unsigned long long& lo, unsigned long long& hi) {
-  asm volatile("ld.relaxed.gpu.global.v2.u64 {%0, %1}, [%2];" : "=l"(lo), "=l"(hi) : "l"(s) : "memory");
+// The whole 32-B slot (key and value) in ONE 256-bit load (LDG.E.ENL2.256, sm_100). Two
+// loads of the same sector (key, then value) cost two random DRAM accesses when the slot
+// is not in L2: tools/rand_probe.cu measured 19.6 G slot reads/s with two loads against
+// 38.8 G/s with one, over a 2-GiB table (profiles/rand_probe_r2.txt). Key and value were
+// never read as one atomic unit (a concurrent claim can be seen torn), and the callers
+// handle that: a half equal to EMPTY sends the insert to the CAS, and a value still EMPTY
+// after its key was claimed reads as "not final" (phase 2 re-reads it).
+__device__ __forceinline__ void ld_slot_relaxed(const Slot* s, unsigned long long& lo, unsigned long long& hi,
+                                                unsigned long long& val) {
+  [[maybe_unused]] unsigned long long pad;
+  asm volatile("ld.relaxed.gpu.global.v4.u64 {%0, %1, %2, %3}, [%4];"
+               : "=l"(lo), "=l"(hi), "=l"(val), "=l"(pad)
+               : "l"(s)
+               : "memory");
+}
+
+// Same, through the L2-only path, for tables with no concurrent writer (phase 3 lookups).
+__device__ __forceinline__ void ld_slot_cg(const Slot* s, unsigned long long& lo, unsigned long long& hi,
+                                           unsigned long long& val) {
+  [[maybe_unused]] unsigned long long pad;
+  asm volatile("ld.global.cg.v4.u64 {%0, %1, %2, %3}, [%4];" : "=l"(lo), "=l"(hi), "=l"(val), "=l"(pad) : "l"(s));
 }
 
 __device__ __forceinline__ unsigned long long ld_val_relaxed(const Slot* s) {
@@ -207,9 +226,8 @@ __device__ __forceinline__ uint64_t table_find_or_claim(Slot* tab, uint64_t cap,
   if (val_seen) *val_seen = kEmpty;
   for (;;) {
     Slot* p = tab + s;
-    unsigned long long lo, hi;
-    ld_key_relaxed(p, lo, hi);
-    const unsigned long long v = val_seen ? ld_val_relaxed(p) : kEmpty;
+    unsigned long long lo, hi, v;
+    ld_slot_relaxed(p, lo, hi, v);
     if (lo == d.lo && hi == d.hi && lo != kEmpty && hi != kEmpty) {
       if (val_seen) *val_seen = v;
       return s;
@@ -265,11 +283,10 @@ __device__ __forceinline__ uint64_t table_insert_min(Slot* tab, uint64_t cap, co
 __device__ __forceinline__ unsigned long long table_lookup(const Slot* tab, uint64_t cap, const Digest& d) {
   uint64_t s = slot_home(d.lo, cap);
   for (;;) {
-    const Slot* p = tab + s;
-    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p));   // key and value: one sector,
-    const unsigned long long val = __ldcg(&p->val);                         // both loads in flight
-    if (kv.x == d.lo && kv.y == d.hi) return val;
-    if (kv.x == kEmpty && kv.y == kEmpty) return kEmpty;
+    unsigned long long klo, khi, val;
+    ld_slot_cg(tab + s, klo, khi, val);   // key and value: one sector, one load
+    if (klo == d.lo && khi == d.hi) return val;
+    if (klo == kEmpty && khi == kEmpty) return kEmpty;
     if (++s == cap) s = 0;
   }
 }
@@ -277,11 +294,10 @@ __device__ __forceinline__ unsigned long long table_lookup(const Slot* tab, uint
 // Lookup continuing at slot s (the caller already checked the home slot).
 __device__ __forceinline__ unsigned long long table_lookup_from(const Slot* tab, uint64_t cap, const Digest& d, uint64_t s) {
   for (;;) {
-    const Slot* p = tab + s;
-    const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p));
-    const unsigned long long val = __ldcg(&p->val);
-    if (kv.x == d.lo && kv.y == d.hi) return val;
-    if (kv.x == kEmpty && kv.y == kEmpty) return kEmpty;
+    unsigned long long klo, khi, val;
+    ld_slot_cg(tab + s, klo, khi, val);   // key and value: one sector, one load
+    if (klo == d.lo && khi == d.hi) return val;
+    if (klo == kEmpty && khi == kEmpty) return kEmpty;
     if (++s == cap) s = 0;
   }
 }

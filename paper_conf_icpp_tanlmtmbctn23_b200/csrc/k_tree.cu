@@ -673,10 +673,7 @@ __device__ void process_group(Ctx& c, WarpSmem& ws, unsigned long long& ins_cnt,
         if (PHASE == 2) {
           cas128(p.tab + sl[t], kEmpty, kEmpty, d[t].lo, d[t].hi, olo[t], ohi[t]);   // Alg.1 l.29 (new key)
         } else {
-          const ulonglong2 kv = __ldcg(reinterpret_cast<const ulonglong2*>(p.tab + sl[t]));  // Alg.1 l.39
-          olo[t] = kv.x;
-          ohi[t] = kv.y;
-          oval[t] = __ldcg(&p.tab[sl[t]].val);
+          ld_slot_cg(p.tab + sl[t], olo[t], ohi[t], oval[t]);   // Alg.1 l.39: key and value, one load
         }
       }
 #pragma unroll
