@@ -55,7 +55,10 @@ constexpr int kWarps = kTreeThreads / 32;
 #ifndef CKPT_TREE_CURSOR
 #define CKPT_TREE_CURSOR 1   // worklist entries beyond the first per warp from a cursor (0: static stride)
 #endif
-constexpr int kDigCap = 256;   // on-chip digests per warp (4 KB); dense groups spill to global
+#ifndef CKPT_DIGCAP
+#define CKPT_DIGCAP 256   // on-chip digests per warp (4 KB); dense groups spill to global
+#endif
+constexpr int kDigCap = CKPT_DIGCAP;
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;

@@ -2,8 +2,9 @@
 # Round-2 measurement pass: GPU tests, smoke, bench (config 2 pipelined and --sync, config 5 in place, config 1,
 # reference arm), pipelined vs synchronous lineages (tools/pipe_probe.py),
 # ncu launch list and full captures (config 2 steady + per-config), sweep (configs 2-5, variants, methods),
-# oracle timing, in-kernel trace, sanitizers.
+# oracle timing, in-kernel trace, sanitizers, random-sector probe of the record table's access pattern.
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu,power.draw --format=csv,noheader
+nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o /tmp/rand_probe tools/rand_probe.cu && timeout 300 /tmp/rand_probe > gpurun_out/rand_probe.txt 2>&1; echo "rand_probe rc=$?"
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"
 timeout 900 python bench.py > gpurun_out/bench.log 2>&1; echo "bench rc=$?"; tail -1 gpurun_out/bench.log | cut -c1-200

@@ -26,3 +26,4 @@ cp $G/trace_kernels.txt $P/trace_kernels_$R.txt
 cp $G/trace_view.txt $P/trace_tiles_$R.txt
 mkdir -p $P/sanitize_$R
 cp $G/sanitize_memcheck.log $G/sanitize_racecheck.log $G/sanitize_synccheck.log $P/sanitize_$R/
+cp $G/rand_probe.txt $P/rand_probe_$R.txt
