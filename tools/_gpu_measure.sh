@@ -31,6 +31,8 @@ python tools/trace_kernels.py gpurun_out/tr > gpurun_out/trace_kernels.txt 2>&1;
 python tools/trace_view.py gpurun_out/tr > gpurun_out/trace_view.txt 2>&1; tail -6 gpurun_out/trace_view.txt
 rm -f gpurun_out/tr.*.bin
 rm -f gpurun_out/*.ncu-rep   # summaries kept; the reports would exceed gpurun's 64 MiB copy-back
+# compute-sanitizer: closed on the GPU pool late in round 2 (the wrapper exits 86); the logs of the last pass
+# where it ran are kept in profiles/sanitize_r2/
 for t in memcheck racecheck synccheck; do
   big=1; [ $t != memcheck ] && big=0
   SAN_BIG=$big timeout 1500 compute-sanitizer --tool $t --print-limit 50 python tools/sanitize_driver.py > gpurun_out/sanitize_$t.log 2>&1; echo "sanitize $t rc=$?"; tail -1 gpurun_out/sanitize_$t.log

@@ -24,6 +24,9 @@ cp $G/oracle_time.json $P/oracle_time_$R.json
 cp $G/pipeline.txt $P/pipeline_$R.txt
 cp $G/trace_kernels.txt $P/trace_kernels_$R.txt
 cp $G/trace_view.txt $P/trace_tiles_$R.txt
-mkdir -p $P/sanitize_$R
-cp $G/sanitize_memcheck.log $G/sanitize_racecheck.log $G/sanitize_synccheck.log $P/sanitize_$R/
+# sanitizer logs only from a pass where compute-sanitizer ran (the pool closed it late in round 2)
+if ! grep -q "is closed on this pool" $G/sanitize_memcheck.log 2>/dev/null; then
+  mkdir -p $P/sanitize_$R
+  cp $G/sanitize_memcheck.log $G/sanitize_racecheck.log $G/sanitize_synccheck.log $P/sanitize_$R/
+fi
 cp $G/rand_probe.txt $P/rand_probe_$R.txt
