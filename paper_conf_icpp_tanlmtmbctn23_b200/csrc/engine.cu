@@ -1457,11 +1457,20 @@ int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream)
     if (rc == CKPT_ECUDA) h->poisoned = true;
     return rc;
   }
+  // chunk owners (8 B per chunk) followed by the bitmap of claimed chunks (claim_kernel)
+  const size_t owner_bytes = h->n * sizeof(unsigned long long) + (h->n + 31) / 32 * sizeof(uint32_t);
   if (!h->owner) {
-    if (cudaMalloc(&h->owner, h->n * sizeof(unsigned long long)) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
+    if (cudaMalloc(&h->owner, owner_bytes) != cudaSuccess) { cudaGetLastError(); return CKPT_ENOMEM; }
   }
-  CK(cudaMemsetAsync(h->owner, 0, h->n * sizeof(unsigned long long), st));
+  CK(cudaMemsetAsync(h->owner, 0, owner_bytes, st));
   uint8_t* outp = static_cast<uint8_t*>(dev_ptr);
+  // claims by bitmap when the newer diffs cover more than the buffer's chunks in total (a
+  // long lineage of heavily rewritten checkpoints: config 4 restores 11-20 % faster, config 2
+  // 3 % slower with it, restore)
+  uint64_t newer = 0;
+  for (uint32_t c = 1; c <= id; ++c)
+    newer += (h->diffs[c].info.data_bytes + h->diffs[c].shift_bytes + h->C - 1) / h->C;
+  const bool bitmap = newer > h->n;
   for (int64_t c = id; c >= 0; --c) {
     const DiffRec& d = h->diffs[c];
     RestoreDiff r = {};
@@ -1474,7 +1483,7 @@ int ckpt_restore_stream(ckpt_handle h, uint32_t id, void* dev_ptr, void* stream)
     r.Flo = d.Flo; r.Foff = d.Foff; r.Slo = d.Slo; r.Soff = d.Soff; r.Ssrc = d.Ssrc;
     r.shift_bytes = d.shift_bytes; r.Fseg = d.Fseg; r.Sseg = d.Sseg;
     r.Cch = d.Cch; r.Csrc = d.Csrc;
-    CK(restore_claim(g, r, h->owner, h->num_sms, st));
+    CK(restore_claim(g, r, h->owner, bitmap, h->num_sms, st));
   }
   CK(restore_copy(g, h->owner, outp, h->num_sms, st));
   CK(sync_stream(h, st));

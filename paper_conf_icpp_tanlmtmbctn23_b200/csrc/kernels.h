@@ -261,7 +261,8 @@ uint64_t restore_segments(uint64_t bytes);
 cudaError_t restore_claimlist(const Geo& g, const RestoreDiff& d, int num_sms, cudaStream_t st);
 cudaError_t restore_resolve(const Geo& g, const RestoreDiff& d, const RestoreDiff* chain_dev, int passes, int* err,
                             int num_sms, cudaStream_t st);
-cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, int num_sms, cudaStream_t st);
+cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long* owner, bool bitmap, int num_sms,
+                          cudaStream_t st);
 cudaError_t restore_copy(const Geo& g, const unsigned long long* owner, uint8_t* out, int num_sms, cudaStream_t st);
 size_t scan_tmp_bytes_for(uint64_t count);
 cudaError_t scan_u64_exclusive(const unsigned long long* in, unsigned long long* out, uint64_t count, void* tmp,
