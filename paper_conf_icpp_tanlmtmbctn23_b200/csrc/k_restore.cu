@@ -201,32 +201,41 @@ __global__ void __launch_bounds__(kRT) claim_kernel(RestoreDiff d, uint64_t ncl,
 // instead of the 8-B owner entry, and the source address is loaded only for a chunk still
 // unclaimed: an older diff of a long lineage, most of whose chunks newer diffs rewrote,
 // costs 4 B of claim list per covered chunk instead of 20 (restore).
+#ifndef CKPT_CLAIM_UNROLL
+#define CKPT_CLAIM_UNROLL 8   // claim entries per thread in flight (bitmap claims; 1 / 4 / 8: config 4 at 30 diffs 1.10 / 1.04 / 0.99 ms)
+#endif
 __global__ void __launch_bounds__(kRT) claim_bitmap_kernel(RestoreDiff d, uint64_t ncl, uint64_t n,
                                                            unsigned long long* owner, int last) {
+  constexpr int U = CKPT_CLAIM_UNROLL;
   pdl_launch_dependents();
   pdl_wait();   // the newer diffs' claims are complete
   uint32_t* const claimed = reinterpret_cast<uint32_t*>(owner + n);
   const int lane = threadIdx.x & 31;
-  const uint64_t wstride = (uint64_t)gridDim.x * kRT;
-  // warp-uniform trip count (the bitmap updates are combined across the warp)
-  for (uint64_t base = (uint64_t)blockIdx.x * kRT + (threadIdx.x & ~31u); base < ncl; base += wstride) {
-    const uint64_t t = base + lane;
-    const uint32_t ch = t < ncl ? __ldg(d.Cch + t) : 0xFFFFFFFFu;
-    bool take = false;
-    if (ch < n) {   // ch < n: guard against malformed plans
-      if (last) {   // the oldest diff (most of its chunks unclaimed): both loads in flight at once
-        const unsigned long long src = __ldg(d.Csrc + t);
-        if (!((__ldcg(claimed + (ch >> 5)) >> (ch & 31)) & 1u)) owner[ch] = src;
-      } else {
-        take = !((__ldcg(claimed + (ch >> 5)) >> (ch & 31)) & 1u);
-        if (take) owner[ch] = __ldg(d.Csrc + t);
-      }
+  const uint64_t wstride = (uint64_t)gridDim.x * kRT * U;
+  // warp-uniform trip count (the bitmap updates are combined across the warp); a warp takes
+  // 32 U consecutive entries per round, U per lane in flight (the bitmap reads are L2 round
+  // trips that depend on the entry's chunk)
+  for (uint64_t base = ((uint64_t)blockIdx.x * kRT + (threadIdx.x & ~31u)) * U; base < ncl; base += wstride) {
+    uint32_t ch[U], wd[U];
+    unsigned long long src[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t t = base + 32 * u + lane;
+      ch[u] = t < ncl ? __ldg(d.Cch + t) : 0xFFFFFFFFu;
+      if (last && ch[u] < n) src[u] = __ldg(d.Csrc + t);   // the oldest diff: mostly unclaimed
     }
-    if (last) continue;   // no later claim pass reads the bitmap
-    const uint32_t key = take ? (ch >> 5) : 0xFFFFFFFFu;
-    const unsigned grp = __match_any_sync(0xffffffffu, key);
-    const uint32_t bits = __reduce_or_sync(grp, take ? 1u << (ch & 31) : 0u);
-    if (take && lane == __ffs(grp) - 1) atomicOr(claimed + key, bits);
+#pragma unroll
+    for (int u = 0; u < U; ++u) wd[u] = ch[u] < n ? __ldcg(claimed + (ch[u] >> 5)) : ~0u;   // ch < n: malformed-plan guard
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool take = ch[u] < n && !((wd[u] >> (ch[u] & 31)) & 1u);
+      if (take) owner[ch[u]] = last ? src[u] : __ldg(d.Csrc + base + 32 * u + lane);
+      if (last) continue;   // no later claim pass reads the bitmap
+      const uint32_t key = take ? (ch[u] >> 5) : 0xFFFFFFFFu;
+      const unsigned grp = __match_any_sync(0xffffffffu, key);
+      const uint32_t bits = __reduce_or_sync(grp, take ? 1u << (ch[u] & 31) : 0u);
+      if (take && lane == __ffs(grp) - 1) atomicOr(claimed + key, bits);
+    }
   }
 }
 
@@ -493,8 +502,10 @@ cudaError_t restore_claim(const Geo& g, const RestoreDiff& d, unsigned long long
   uint64_t grid = (nx + kRT - 1) / kRT;
   const uint64_t cap = (uint64_t)num_sms * (g_claim_bps > 0 ? g_claim_bps : 4);
   if (grid > cap) grid = cap;
-  if (bitmap)
+  if (bitmap) {
+    grid = std::min<uint64_t>(cap, (nx + kRT * CKPT_CLAIM_UNROLL - 1) / (kRT * CKPT_CLAIM_UNROLL));
     return launch_pdl(claim_bitmap_kernel, (unsigned)grid, kRT, 0, st, d, nx, (uint64_t)g.n, owner, d.id == 0 ? 1 : 0);
+  }
   return launch_pdl(claim_kernel, (unsigned)grid, kRT, 0, st, d, nx, (uint64_t)g.n, owner);
 }
 
