@@ -55,6 +55,9 @@ struct Inflight {
   std::chrono::steady_clock::time_point t_entry, t_pre, t_launched;
 };
 
+#ifndef CKPT_GREEN_CAND_PER_SM
+#define CKPT_GREEN_CAND_PER_SM 2300   // candidates per chain SM up to which a pipelined call is partitioned
+#endif
 #ifndef CKPT_K1_C32_SMEM
 #define CKPT_K1_C32_SMEM 49152      // K1 stage budget per CTA when C = 32 (data + digests; 4 CTAs per SM)
 #endif
@@ -136,6 +139,22 @@ struct ckpt_ctx {
   bool call_pipe[4] = {};        // call k was submitted pipelined (index k & 3)
   cudaStream_t cs = nullptr;
   cudaEvent_t ev_k1[2] = {}, ev_chain[2] = {};   // after K1(k) / after gather(k), parity k & 1
+  // SM partitions of pipelined calls (green contexts): K1 on the SMs of one
+  // green context (stream k1s), the chain on the other m (stream cs), so that the next K1 and
+  // this call's chain run side by side instead of taking turns for the SMs. m is chosen per
+  // call from the candidate count of the last collected call; none when the chain is heavy.
+  struct Part {
+    int m = 0;
+    CUgreenCtx g[2] = {};
+    cudaStream_t k1s = nullptr, cs = nullptr;
+    int sm_k1 = 0, sm_chain = 0;
+  };
+  static constexpr int kMaxParts = 4;
+  Part parts[kMaxParts];
+  int nparts = 0;
+  cudaEvent_t ev_in[2] = {};
+  cudaStream_t prev_cs = nullptr;   // chain stream of the previous pipelined call
+  uint64_t last_cand = ~0ull;       // non-FIXED leaves of the last collected call (~0: none yet)
   uint8_t* staging = nullptr;
   uint64_t staging_size = 0;
   // restore state (lazy): chunk owners, plan scratch, the chain's plans on device
@@ -517,6 +536,78 @@ bool validate_import_body(const HostGeo& g, const uint8_t* hd, uint32_t id, int 
 
 }  // namespace
 
+// Green contexts (CUDA 12.4+ driver API, through cudaGetDriverEntryPoint): the device's SMs
+// split into m for the chain and the rest for K1; one stream in each. The kernels' attributes
+// (K1's dynamic shared memory) are set and the modules loaded in both contexts.
+template <class F>
+static F drv(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return reinterpret_cast<F>(fn);
+}
+
+static int make_green(ckpt_ctx* h, ckpt_ctx::Part& P, int m, int prio_hi) {
+  auto getres = drv<CUresult (*)(CUdevice, CUdevResource*, CUdevResourceType)>("cuDeviceGetDevResource");
+  auto split = drv<CUresult (*)(CUdevResource*, unsigned*, const CUdevResource*, CUdevResource*, unsigned, unsigned)>(
+      "cuDevSmResourceSplitByCount");
+  auto gendesc = drv<CUresult (*)(CUdevResourceDesc*, CUdevResource*, unsigned)>("cuDevResourceGenerateDesc");
+  auto gcreate = drv<CUresult (*)(CUgreenCtx*, CUdevResourceDesc, CUdevice, unsigned)>("cuGreenCtxCreate");
+  auto gstream = drv<CUresult (*)(CUstream*, CUgreenCtx, unsigned, int)>("cuGreenCtxStreamCreate");
+  auto fromgreen = drv<CUresult (*)(CUcontext*, CUgreenCtx)>("cuCtxFromGreenCtx");
+  auto getcur = drv<CUresult (*)(CUcontext*)>("cuCtxGetCurrent");
+  auto setcur = drv<CUresult (*)(CUcontext)>("cuCtxSetCurrent");
+  if (!getres || !split || !gendesc || !gcreate || !gstream || !fromgreen || !getcur || !setcur) return CKPT_ECUDA;
+  const CUdevice dev = (CUdevice)h->device;
+  CUdevResource all, grp, rest;
+  unsigned ng = 1;
+  CUdevResourceDesc dk, dc;
+  if (getres(dev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS ||
+      split(&grp, &ng, &all, &rest, 0, (unsigned)m) != CUDA_SUCCESS || ng != 1 ||
+      gendesc(&dk, &rest, 1) != CUDA_SUCCESS || gendesc(&dc, &grp, 1) != CUDA_SUCCESS ||
+      gcreate(&P.g[0], dk, dev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS ||
+      gcreate(&P.g[1], dc, dev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS)
+    return CKPT_ECUDA;
+  CUstream sk, sc;
+  if (gstream(&sk, P.g[0], CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS ||
+      gstream(&sc, P.g[1], CU_STREAM_NON_BLOCKING, prio_hi) != CUDA_SUCCESS)
+    return CKPT_ECUDA;
+  P.m = m;
+  P.k1s = reinterpret_cast<cudaStream_t>(sk);
+  P.cs = reinterpret_cast<cudaStream_t>(sc);
+  P.sm_k1 = (int)rest.sm.smCount;
+  P.sm_chain = (int)grp.sm.smCount;
+  CUcontext prim = nullptr;
+  if (getcur(&prim) != CUDA_SUCCESS) return CKPT_ECUDA;
+  for (int i = 0; i < 2; ++i) {
+    CUcontext c = nullptr;
+    if (fromgreen(&c, P.g[i]) != CUDA_SUCCESS || setcur(c) != CUDA_SUCCESS) return CKPT_ECUDA;
+    const bool ok = leaf_setup_attributes() == cudaSuccess && tree_setup_attributes() == cudaSuccess &&
+                    preload_leaf() == cudaSuccess && preload_tree() == cudaSuccess && preload_compact() == cudaSuccess;
+    setcur(prim);
+    if (!ok) { cudaGetLastError(); return CKPT_ECUDA; }
+  }
+  return CKPT_OK;
+}
+
+// The partition of a pipelined call: the chain's SMs from the candidate count of the last
+// collected call (the chain's work grows with it). Measured on config 2 (1 GiB, C = 128,
+// DESIGN.md §1a): ~6 K candidates run best with 16 chain SMs (0.176 ms per step against 0.206
+// without a partition), ~59 K with 20-32 (0.207 against 0.222), and ~300 K (p = 5 %) best
+// without one (a 32-SM chain took 0.44 ms). Below ~2 300 candidates per chain SM a partition
+// of that size keeps the chain within the next K1. K1 on 16 SMs fewer streams ~3 % slower,
+// which outweighs the hidden chain on long K1 passes (config 3, 4 GiB at C = 4096: 0.715 ->
+// 0.733 ms per step), so buffers above 2 GiB are not partitioned.
+static const ckpt_ctx::Part* pick_part(const ckpt_ctx* h) {
+  if (!h->nparts || h->last_cand == ~0ull || h->B > (2ull << 30)) return nullptr;
+  for (int i = 0; i < h->nparts; ++i)
+    if (h->last_cand <= (uint64_t)CKPT_GREEN_CAND_PER_SM * (uint64_t)h->parts[i].sm_chain) return &h->parts[i];
+  return nullptr;
+}
+
 extern "C" {
 
 static int drain(ckpt_ctx* h);   // collects the calls in flight (ckpt_checkpoint_submit)
@@ -609,6 +700,17 @@ int ckpt_destroy(ckpt_handle h) {
     if (h->ev_chain[i]) cudaEventDestroy(h->ev_chain[i]);
   }
   if (h->cs) cudaStreamDestroy(h->cs);
+  for (int i = 0; i < 2; ++i)
+    if (h->ev_in[i]) cudaEventDestroy(h->ev_in[i]);
+  {
+    auto gdestroy = drv<CUresult (*)(CUgreenCtx)>("cuGreenCtxDestroy");
+    for (auto& P : h->parts) {
+      if (P.k1s) cudaStreamDestroy(P.k1s);
+      if (P.cs) cudaStreamDestroy(P.cs);
+      for (int i = 0; i < 2; ++i)
+        if (P.g[i] && gdestroy) gdestroy(P.g[i]);
+    }
+  }
   if (h->staging) cudaFree(h->staging);
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r)
     for (int i = 0; i < 6; ++i) if (h->evr[r][i]) cudaEventDestroy(h->evr[r][i]);
@@ -736,6 +838,19 @@ static int ensure_pipe_state(ckpt_ctx* h) {
   // race and 0.4-2.4 ms when K1's CTAs starved the chain's statically partitioned K1b and
   // gather; with the highest priority 0.226-0.228 ms, every run)
   if (cudaStreamCreateWithPriority(&h->cs, cudaStreamNonBlocking, hi) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
+  // SM partitions (CKPT_GREEN=0 disables them): chain sizes 16, 24, 32, 40 SMs
+  const char* gm = getenv("CKPT_GREEN");
+  if (!(gm && atoi(gm) == 0) && h->num_sms >= 96) {
+    for (int m : {16, 24, 32, 40}) {
+      if (make_green(h, h->parts[h->nparts], m, hi) != CKPT_OK) {   // no partitions: the shared form
+        cudaGetLastError();
+        break;
+      }
+      ++h->nparts;
+    }
+    for (int i = 0; i < 2 && h->nparts; ++i)
+      if (cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming) != cudaSuccess) return CKPT_ECUDA;
+  }
   for (int i = 0; i < 2; ++i)
     if (cudaEventCreateWithFlags(&h->ev_k1[i], cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&h->ev_chain[i], cudaEventDisableTiming) != cudaSuccess) {
@@ -758,8 +873,13 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   }
   const uint32_t k = (uint32_t)(h->diffs.size() + h->inflight.size());
   int r = CKPT_OK;
-  // the stream of the tree phases and the gather
-  const cudaStream_t cst = pipe ? h->cs : st;
+  // the stream of the tree phases and the gather; with an SM partition (CKPT_GREEN), K1's
+  // stream too, and the SMs each side sizes its grids for
+  const ckpt_ctx::Part* part = pipe ? pick_part(h) : nullptr;
+  const bool green = part != nullptr;
+  const cudaStream_t cst = green ? part->cs : pipe ? h->cs : st;
+  const cudaStream_t kst = green ? part->k1s : st;
+  const int sms_k1 = green ? part->sm_k1 : h->num_sms, sms_chain = green ? part->sm_chain : h->num_sms;
   if (pipe) {
     if (!h->cdig2[0]) {
       if (dalloc(h, &h->cdig2[0], h->n) != cudaSuccess || dalloc(h, &h->cdig2[1], h->n) != cudaSuccess) return CKPT_ENOMEM;
@@ -773,12 +893,19 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
         CK(cudaEventRecord(h->done_ev, ls));
         if (st != ls) CK(cudaStreamWaitEvent(st, h->done_ev, 0));
         if (cst != ls) CK(cudaStreamWaitEvent(cst, h->done_ev, 0));
+        if (kst != st && kst != ls) CK(cudaStreamWaitEvent(kst, h->done_ev, 0));
       }
     } else {
       // K1(k) after K1(k - 1) (prev digests, possibly another stream) and after the chain of
       // call k - 2 (this parity's buffers); the chain follows call k - 1's on h->cs
-      CK(cudaStreamWaitEvent(st, h->ev_k1[(k - 1) & 1], 0));
-      if (k >= 2 && h->call_pipe[(k - 2) & 3]) CK(cudaStreamWaitEvent(st, h->ev_chain[k & 1], 0));
+      CK(cudaStreamWaitEvent(kst, h->ev_k1[(k - 1) & 1], 0));
+      if (k >= 2 && h->call_pipe[(k - 2) & 3]) CK(cudaStreamWaitEvent(kst, h->ev_chain[k & 1], 0));
+      // a chain on another stream than the previous call's follows that call's chain
+      if (cst != h->prev_cs) CK(cudaStreamWaitEvent(cst, h->ev_chain[(k - 1) & 1], 0));
+    }
+    if (green) {   // K1 after the caller's work on `st` (the input buffer)
+      CK(cudaEventRecord(h->ev_in[k & 1], st));
+      CK(cudaStreamWaitEvent(kst, h->ev_in[k & 1], 0));
     }
   }
   const auto t_tab = clk::now();
@@ -889,20 +1016,20 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   const bool pe = h->prof >= 2;
   const auto t_pre = clk::now();
   if (!pipe) CK(after_last_checkpoint(h, st));   // the previous call's gather may still be finishing
-  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 32 * kTraceLanes, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[0], st));
+  if (h->trace) CK(cudaMemsetAsync(h->trace_n, 0, 32 * kTraceLanes, kst));
+  if (h->prof) CK(cudaEventRecord(h->ev[0], kst));
   // K1 + K1t: hash, fixed test, candidate bits, digest update (Alg.1 l.1-5, l.21)
-  CK(launch_leaf_tail(lp, st));
-  CK(launch_leaf(&tmap, lp, h->num_sms, st));
-  if (h->prof) CK(cudaEventRecord(h->ev[1], st));
+  CK(launch_leaf_tail(lp, kst));
+  CK(launch_leaf(&tmap, lp, sms_k1, kst));
+  if (h->prof) CK(cudaEventRecord(h->ev[1], kst));
   if (pipe) {
-    CK(cudaEventRecord(h->ev_k1[k & 1], st));
+    CK(cudaEventRecord(h->ev_k1[k & 1], kst));
     CK(cudaStreamWaitEvent(cst, h->ev_k1[k & 1], 0));
   }
   // K1b: record insert + tie-break (l.6-19), dirty tiles
   // pipelined: a plain launch (the chain stream's previous kernel is the last call's gather,
   // which triggers early; see launch_insert)
-  CK(launch_insert(ip, h->num_sms, cst, !pipe));
+  CK(launch_insert(ip, sms_chain, cst, !pipe));
   if (pe) CK(cudaEventRecord(h->ev[2], cst));
 
   // ---- phase 2 (all stages, one launch), then phase 3 (all stages, one launch): R11
@@ -941,10 +1068,10 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   tp.shift_insert = h->mode == kModeTree && (h->variant & CKPT_VARIANT_SHIFT_INSERT);
   tp.sw_permille = ip.sw_permille;
   if (h->mode != kModeBasic) {   // Basic: no record, no tree
-    CK(launch_tree(tp, 2, h->num_sms, cst));
+    CK(launch_tree(tp, 2, sms_chain, cst));
     if (pe) CK(cudaEventRecord(h->ev[3], cst));
-    if (tp.shift_insert) CK(launch_tree(tp, 4, h->num_sms, cst));   // R24 inserts, before any lookup
-    CK(launch_tree(tp, 3, h->num_sms, cst));
+    if (tp.shift_insert) CK(launch_tree(tp, 4, sms_chain, cst));   // R24 inserts, before any lookup
+    CK(launch_tree(tp, 3, sms_chain, cst));
     if (pe) CK(cudaEventRecord(h->ev[4], cst));
   } else if (pe) {
     CK(cudaEventRecord(h->ev[3], cst));
@@ -969,12 +1096,15 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   cp.cand = h->cand;
   cp.nwords = h->nwords;
   cp.tcc = h->tcc;
-  cp.parts = gather_parts(h->ngroups[0], h->C, h->num_sms);
+  cp.parts = gather_parts(h->ngroups[0], h->C, sms_chain);
   cp.sw_permille = ip.sw_permille;
   cp.full_first = (h->variant & CKPT_VARIANT_FULL_FIRST) && k == 0;   // R22
-  CK(launch_compact(cp, h->num_sms, cst));
+  CK(launch_compact(cp, sms_chain, cst));
   if (h->prof) CK(cudaEventRecord(h->ev[5], cst));
-  if (pipe) CK(cudaEventRecord(h->ev_chain[k & 1], cst));
+  if (pipe) {
+    CK(cudaEventRecord(h->ev_chain[k & 1], cst));
+    h->prev_cs = cst;
+  }
   h->last_stream = cst;
   h->pending = true;
   h->call_pipe[k & 3] = pipe;
@@ -1034,6 +1164,7 @@ static int finish_call(ckpt_ctx* h, const Inflight& f, ckpt_diff* diff) {
     if (FILE* fp = fopen(path, "wb")) { fwrite(tr.data(), sizeof(ulonglong4), tr.size(), fp); fclose(fp); }
   }
   if (h->mode != kModeBasic && t.full_kind != 2) h->live += t.n_first + t.p2_inserts + t.p3_inserts;   // R23: no record op
+  h->last_cand = t.n_first + t.n_spatial + t.n_temporal;   // the next pipelined call's partition
   DiffRec rec;
   rec.ptr = f.out;
   fill_diff(h, k, t, f.out, &rec.info);
@@ -1121,7 +1252,7 @@ int ckpt_checkpoint_wait(ckpt_handle h, uint32_t id, void* stream, ckpt_diff* di
   // the rest of call id (its gather) before the caller's later work on `stream`: the event
   // of this parity follows call id's gather (or a later call's, at worst late)
   const cudaStream_t ws = static_cast<cudaStream_t>(stream);
-  if (h->call_pipe[id & 3] && ws != h->cs) CK(cudaStreamWaitEvent(ws, h->ev_chain[id & 1], 0));
+  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ws, h->ev_chain[id & 1], 0));
   *diff = h->diffs[id].info;
   return h->diffs[id].collided ? CKPT_ECOLLIDE : CKPT_OK;
 }
@@ -1165,7 +1296,7 @@ int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t
   const cudaStream_t ds = static_cast<cudaStream_t>(stream);
   // after the gather of call id: the event of its parity (re-recorded by a later call of the
   // same parity at most, which is later still), or the latest call for a synchronous one
-  if (h->call_pipe[id & 3] && ds != h->cs) CK(cudaStreamWaitEvent(ds, h->ev_chain[id & 1], 0));
+  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ds, h->ev_chain[id & 1], 0));
   else CK(after_last_checkpoint(h, ds));
   CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, ds));
   return CKPT_OK;
