@@ -838,9 +838,14 @@ static int ensure_pipe_state(ckpt_ctx* h) {
   // race and 0.4-2.4 ms when K1's CTAs starved the chain's statically partitioned K1b and
   // gather; with the highest priority 0.226-0.228 ms, every run)
   if (cudaStreamCreateWithPriority(&h->cs, cudaStreamNonBlocking, hi) != cudaSuccess) { cudaGetLastError(); return CKPT_ECUDA; }
-  // SM partitions (CKPT_GREEN=0 disables them): chain sizes 16, 24, 32, 40 SMs
+  // SM partitions (CKPT_GREEN=0 disables them): chain sizes 16, 24, 32, 40 SMs. Not under a
+  // profiling / injection tool: under ncu 2025.2 a pipelined lineage on green contexts failed
+  // at its first partitioned call ("Failed to prepare kernel for profiling")
   const char* gm = getenv("CKPT_GREEN");
-  if (!(gm && atoi(gm) == 0) && h->num_sms >= 96) {
+  bool tool = false;
+  for (const char* v : {"CUDA_INJECTION64_PATH", "NV_COMPUTE_PROFILER_PERFWORKS_DIR", "NVIDIA-PROCESS-TRACKING-CONFIGURATION"})
+    if (const char* e = getenv(v)) tool = tool || *e;
+  if (!(gm && atoi(gm) == 0) && !tool && h->num_sms >= 96) {
     for (int m : {16, 24, 32, 40}) {
       if (make_green(h, h->parts[h->nparts], m, hi) != CKPT_OK) {   // no partitions: the shared form
         cudaGetLastError();
