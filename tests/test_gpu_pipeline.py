@@ -303,3 +303,33 @@ def test_async_d2h_of_collected_diffs_keeps_pipelining(oracle_mod):
     for k in range(len(bufs)):
         assert bytes(hosts[k][:sizes[k]].numpy()) == o.diff(k), k
     ck.close()
+
+
+def _alternating_lineage(nbytes, C, K, seed=5):
+    """Checkpoints alternate between rewriting every chunk and changing ~1 % of them, so the
+    SM partition a pipelined call picks from the previous call's candidate count (DESIGN.md
+    §1a: none above 40 x 2 300 candidates, 16 chain SMs below 16 x 2 300) switches at every
+    call, and the chain stream changes from call to call."""
+    rng = np.random.default_rng(seed)
+    buf = rng.integers(0, 256, nbytes, dtype=np.uint8)
+    out = [buf.copy()]
+    for k in range(1, K):
+        if k % 2:
+            buf = rng.integers(0, 256, nbytes, dtype=np.uint8)
+        else:
+            n = nbytes // C
+            for c in rng.choice(n, size=max(1, n // 100), replace=False):
+                buf[c * C] ^= 0x5A
+        out.append(buf.copy())
+    return out
+
+
+@pytest.mark.parametrize("green", ["1", "0"])
+def test_partition_switching_pipelined(oracle_mod, monkeypatch, green):
+    # 16 MiB at C = 128: 131 072 leaves; a full rewrite is above the largest partition's
+    # threshold, a 1 % change below the smallest. green = "0": the unpartitioned form.
+    if green == "0":
+        monkeypatch.setenv("CKPT_GREEN", "0")
+    else:
+        monkeypatch.delenv("CKPT_GREEN", raising=False)
+    run_pipe_parity(oracle_mod, _alternating_lineage((16 << 20) + 48, 128, 8), 128)
