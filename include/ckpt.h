@@ -37,6 +37,9 @@ extern "C" {
 
 typedef struct ckpt_ctx* ckpt_handle;
 
+/* Pipelined calls in flight at most (ckpt_checkpoint_submit). */
+#define CKPT_PIPELINE_DEPTH 2
+
 enum {
   CKPT_OK = 0,
   CKPT_EINVAL = 1, /* bad argument / precondition violated; nothing changed           */
@@ -176,12 +179,13 @@ CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes,
  * bit-identical); only the overlap of consecutive calls differs.
  *   dev_ptr, bytes  as ckpt_checkpoint. BORROWED until ckpt_checkpoint_wait(id) returns AND
  *                   the caller's later work is ordered after the stream passed to it.
- *   stream          cudaStream_t (as void*) the leaf pass is enqueued on; the record and tree
- *                   phases and the gather run on an internal non-blocking stream of the handle,
- *                   ordered after it by events.
+ *   stream          cudaStream_t (as void*) the leaf pass is ordered after; the leaf pass runs
+ *                   on it, or (SM partitions) on an internal stream of a green
+ *                   context ordered after it by an event; the record and tree phases and the
+ *                   gather run on an internal non-blocking stream, ordered after the leaf pass.
  *   id              receives the checkpoint id (= the number of checkpoints before it).
- * At most two calls are in flight: a submit with two outstanding first collects the older
- * (a host wait). Every other call of this library (ckpt_checkpoint, diff access, restore,
+ * At most CKPT_PIPELINE_DEPTH (2) calls are in flight: a submit with that many outstanding
+ * first collects the oldest (a host wait). Every other call of this library (ckpt_checkpoint, diff access, restore,
  * import, introspection) first collects all outstanding calls, oldest first.
  * Errors: as ckpt_checkpoint (an error of the collected older call is returned here). */
 CKPT_API int ckpt_checkpoint_submit(ckpt_handle h, const void* dev_ptr, uint64_t bytes, void* stream, uint32_t* id);

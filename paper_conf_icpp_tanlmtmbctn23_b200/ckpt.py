@@ -34,6 +34,9 @@ ABI_FUNCTIONS = [
 ]
 
 
+PIPELINE_DEPTH = 2   # include/ckpt.h CKPT_PIPELINE_DEPTH: pipelined calls in flight at most
+
+
 class CkptDiff(ctypes.Structure):
     _fields_ = [
         ("id", ctypes.c_uint32),

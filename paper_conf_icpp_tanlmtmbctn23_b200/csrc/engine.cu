@@ -55,8 +55,16 @@ struct Inflight {
   std::chrono::steady_clock::time_point t_entry, t_pre, t_launched;
 };
 
+#ifndef CKPT_PIPE_DEPTH
+#define CKPT_PIPE_DEPTH CKPT_PIPELINE_DEPTH   // pipelined calls in flight (include/ckpt.h). A depth-3
+                                              // build (3 arenas, 4 counter sets) measured the same as 2
+                                              // with SM partitions: the chain's throughput on its SMs, not
+                                              // its latency, bounds the step
+#endif
+constexpr int kDepth = CKPT_PIPE_DEPTH;
+static_assert(kDepth >= 2 && kDepth <= 3, "pipeline depth");
 #ifndef CKPT_GREEN_CAND_PER_SM
-#define CKPT_GREEN_CAND_PER_SM 2300   // candidates per chain SM up to which a pipelined call is partitioned
+#define CKPT_GREEN_CAND_PER_SM 2600   // candidates per chain SM up to which a pipelined call is partitioned
 #endif
 #ifndef CKPT_K1_C32_SMEM
 #define CKPT_K1_C32_SMEM 49152      // K1 stage budget per CTA when C = 32 (data + digests; 4 CTAs per SM)
@@ -93,10 +101,10 @@ struct ckpt_ctx {
   uint64_t ngroups[kMaxStages] = {};
   // device state
   Digest* prev = nullptr;
-  uint32_t* cand = nullptr;       // = cand2[k & 1] of the current call
-  uint32_t* cand2[2] = {};        // candidate bits per call parity: a pipelined call's K1 writes its own
+  uint32_t* cand = nullptr;       // = cand2[k % kDepth] of the current call
+  uint32_t* cand2[kDepth] = {};        // candidate bits per call parity: a pipelined call's K1 writes its own
                                   // while the previous call's tree phases read theirs
-  Digest* cdig2[2] = {};          // pipelined calls: the candidates' digests of call k (parity k & 1), read
+  Digest* cdig2[kDepth] = {};          // pipelined calls: the candidates' digests of call k (slot k % kDepth), read
                                   // by its K1b / tree kernels while the next call's K1 updates prev in place
   uint64_t nwords = 0;
   unsigned long long* res_of = nullptr;   // per chunk (candidates only): K1b's resolution
@@ -116,29 +124,29 @@ struct ckpt_ctx {
   // Totals + per-stage counters, triple-buffered: call k uses ctr3[k % 3] and its last kernel
   // zeroes ctr3[(k + 2) % 3] (the previous call's, complete by then) for call k + 2, so no
   // memset precedes K1 and a pipelined call's K1 never meets a buffer still being zeroed.
-  uint8_t* ctr3[3] = {};
+  uint8_t* ctr3[kDepth + 1] = {};
   size_t ctr_bytes = 0;
   size_t ctr_dbits_off = 0, ctr_tcc_off = 0, ctr_bsum_off = 0, ctr_gsum_off = 0, ctr_stage_off[kMaxStages] = {};
   uint4* scratch = nullptr;
   uint4* tilecnt = nullptr;
   uint32_t* lmask = nullptr;
-  uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b (= defer2[k & 1])
-  uint32_t* defer2[2] = {};
+  uint32_t* defer = nullptr;     // 256-chunk leaf tiles whose inserts go to K1b (= defer2[k % kDepth])
+  uint32_t* defer2[kDepth] = {};
   unsigned long long* blocksum = nullptr;
   unsigned long long* gsum = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
-  Totals* tot_host2[2] = {};    // pinned + mapped, per call parity: written by the gather kernel
+  Totals* tot_host2[kDepth] = {};    // pinned + mapped, per call parity: written by the gather kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
   std::vector<void*> retired;    // record tables replaced by a growth (freed by ckpt_destroy)
-  DiffArena arena[2];            // diffs; pipelined calls alternate (call k: arena[k & 1])
-  bool arena1_ready = false;
+  DiffArena arena[kDepth];       // diffs; pipelined calls rotate (call k: arena[k % kDepth])
+  int arenas_ready = 1;          // arena[0] is set up with the geometry, the others at first use
   std::vector<DiffRec> diffs;
   // pipelining (ckpt_checkpoint_submit): K1 on the caller's stream, K1b .. gather on `cs`
   std::deque<Inflight> inflight;
   bool call_pipe[4] = {};        // call k was submitted pipelined (index k & 3)
   cudaStream_t cs = nullptr;
-  cudaEvent_t ev_k1[2] = {}, ev_chain[2] = {};   // after K1(k) / after gather(k), parity k & 1
+  cudaEvent_t ev_k1[kDepth] = {}, ev_chain[kDepth] = {};   // after K1(k) / after gather(k), slot k % kDepth
   // SM partitions of pipelined calls (green contexts): K1 on the SMs of one
   // green context (stream k1s), the chain on the other m (stream cs), so that the next K1 and
   // this call's chain run side by side instead of taking turns for the SMs. m is chosen per
@@ -152,7 +160,8 @@ struct ckpt_ctx {
   static constexpr int kMaxParts = 4;
   Part parts[kMaxParts];
   int nparts = 0;
-  cudaEvent_t ev_in[2] = {};
+  bool part_forced = false;         // CKPT_GREEN=m (m >= 8): every pipelined call on one m-SM partition (tuning)
+  cudaEvent_t ev_in[kDepth] = {};
   cudaStream_t prev_cs = nullptr;   // chain stream of the previous pipelined call
   uint64_t last_cand = ~0ull;       // non-FIXED leaves of the last collected call (~0: none yet)
   uint8_t* staging = nullptr;
@@ -286,8 +295,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
     if (e != cudaSuccess) return CKPT_ENOMEM; \
   } while (0)
   AL(h->prev, n);
-  AL(h->cand2[0], h->nwords + 32);
-  AL(h->cand2[1], h->nwords + 32);
+  for (int i = 0; i < kDepth; ++i) AL(h->cand2[i], h->nwords + 32);
   h->cand = h->cand2[0];
   AL(h->res_of, n);
   for (int s = 0; s < h->S; ++s) {
@@ -320,7 +328,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
       off[s] = bytes;
       bytes += (4 + 32 + 64 + 32) * h->ngroups[s] * sizeof(uint32_t);   // arr2 arr3 arr4 dcnt, gm2, gm3, gm4
     }
-    for (int i = 0; i < 3; ++i) {
+    for (int i = 0; i < kDepth + 1; ++i) {
       AL(h->ctr3[i], bytes);
       if (cudaMemsetAsync(h->ctr3[i], 0, bytes, st) != cudaSuccess) return CKPT_ECUDA;
     }
@@ -335,8 +343,7 @@ int setup_geometry(ckpt_ctx* h, uint64_t B, cudaStream_t st) {
   AL(h->tilecnt, n_tiles);
   AL(h->wl0, n_tiles);
   AL(h->lmask, n_tiles * kLmWords);
-  AL(h->defer2[0], n / 32 + 16);   // (tile << 3 | round) entries, one per 32 candidates
-  AL(h->defer2[1], n / 32 + 16);
+  for (int i = 0; i < kDepth; ++i) AL(h->defer2[i], n / 32 + 16);   // (tile << 3 | round), one per 32 candidates
   h->defer = h->defer2[0];
 #undef AL
   if (cudaMemsetAsync(h->tilecnt, 0, n_tiles * sizeof(uint4), st) != cudaSuccess) return CKPT_ECUDA;
@@ -370,7 +377,7 @@ int ensure_table(ckpt_ctx* h, cudaStream_t st, bool pipe) {
   // worst case: every node inserted, by this call and, for pipelined calls, by
   // the call that may still be in flight (its inserts are not counted in `live` yet); sized
   // for two from the first pipelined call on, so the growth happens there and not later
-  uint64_t need = h->live + (pipe ? 2 : 1) * (2 * h->n - 1);
+  uint64_t need = h->live + (pipe ? kDepth : 1) * (2 * h->n - 1);
   if (h->dbg & 256) need = h->live + h->n / 2;   // diagnostics only: undersized table experiment
   if (h->cap && (double)need <= kMaxLoad * (double)h->cap) return CKPT_OK;
   // geometric growth: at least double, so a lineage whose record keeps growing pays for a
@@ -597,11 +604,13 @@ static int make_green(ckpt_ctx* h, ckpt_ctx::Part& P, int m, int prio_hi) {
 // collected call (the chain's work grows with it). Measured on config 2 (1 GiB, C = 128,
 // DESIGN.md §1a): ~6 K candidates run best with 16 chain SMs (0.176 ms per step against 0.206
 // without a partition), ~59 K with 20-32 (0.207 against 0.222), and ~300 K (p = 5 %) best
-// without one (a 32-SM chain took 0.44 ms). Below ~2 300 candidates per chain SM a partition
-// of that size keeps the chain within the next K1. K1 on 16 SMs fewer streams ~3 % slower,
+// without one (a 32-SM chain took 0.44 ms). Below ~2 600 candidates per chain SM a partition
+// of that size keeps the chain within the next K1 (59 K on 24 SMs: 0.2054 ms; on 20: 0.2068;
+// on 16, 3 700 per SM, the chain no longer keeps up: 0.277). K1 on 16 SMs fewer streams ~3 % slower,
 // which outweighs the hidden chain on long K1 passes (config 3, 4 GiB at C = 4096: 0.715 ->
 // 0.733 ms per step), so buffers above 2 GiB are not partitioned.
 static const ckpt_ctx::Part* pick_part(const ckpt_ctx* h) {
+  if (h->part_forced) return &h->parts[0];
   if (!h->nparts || h->last_cand == ~0ull || h->B > (2ull << 30)) return nullptr;
   for (int i = 0; i < h->nparts; ++i)
     if (h->last_cand <= (uint64_t)CKPT_GREEN_CAND_PER_SM * (uint64_t)h->parts[i].sm_chain) return &h->parts[i];
@@ -666,10 +675,10 @@ int ckpt_create_mode(uint32_t chunk_bytes, int mode, ckpt_handle* out) {
   // default stream (torch's default) completes before ckpt_restore / ckpt_import /
   // ckpt_leaf_digests touch memory on it (ckpt.h ordering contract).
   if (cudaStreamCreateWithFlags(&h->internal, cudaStreamDefault) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < kDepth; ++i)
     if (cudaHostAlloc(&h->tot_host2[i], sizeof(Totals), cudaHostAllocMapped) != cudaSuccess) { delete h; return CKPT_ECUDA; }
   if (cudaEventCreateWithFlags(&h->done_ev, cudaEventDisableTiming) != cudaSuccess) { delete h; return CKPT_ECUDA; }
-  for (int i = 0; i < 2; ++i) std::memset(h->tot_host2[i], 0, sizeof(Totals));   // done = 0: epochs start at 1
+  for (int i = 0; i < kDepth; ++i) std::memset(h->tot_host2[i], 0, sizeof(Totals));   // done = 0: epochs start at 1
   for (int r = 0; r < ckpt_ctx::kEvRing; ++r) {
     h->ev_id[r] = -1;
     for (int i = 0; i < 6; ++i) cudaEventCreate(&h->evr[r][i]);
@@ -683,8 +692,7 @@ int ckpt_destroy(ckpt_handle h) {
   cudaSetDevice(h->device);
   cudaDeviceSynchronize();
   for (void* p : h->allocs) cudaFree(p);
-  h->arena[0].release_all();
-  if (h->arena1_ready) h->arena[1].release_all();
+  for (int i = 0; i < h->arenas_ready; ++i) h->arena[i].release_all();
   for (auto& d : h->diffs)
     for (void* q : {(void*)d.Flo, (void*)d.Foff, (void*)d.Slo, (void*)d.Soff, (void*)d.Ssrc, (void*)d.Fseg, (void*)d.Sseg,
                     (void*)d.Cch, (void*)d.Csrc})
@@ -693,14 +701,14 @@ int ckpt_destroy(ckpt_handle h) {
     if (q) cudaFree(q);
   if (h->tab) cudaFree(h->tab);
   for (void* q : h->retired) cudaFree(q);
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < kDepth; ++i)
     if (h->tot_host2[i]) cudaFreeHost(h->tot_host2[i]);
-  for (int i = 0; i < 2; ++i) {
+  for (int i = 0; i < kDepth; ++i) {
     if (h->ev_k1[i]) cudaEventDestroy(h->ev_k1[i]);
     if (h->ev_chain[i]) cudaEventDestroy(h->ev_chain[i]);
   }
   if (h->cs) cudaStreamDestroy(h->cs);
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < kDepth; ++i)
     if (h->ev_in[i]) cudaEventDestroy(h->ev_in[i]);
   {
     auto gdestroy = drv<CUresult (*)(CUgreenCtx)>("cuGreenCtxDestroy");
@@ -801,11 +809,11 @@ struct LaunchCount {
 };
 
 // Point the per-call views at call k's buffers: counters ctr3[k % 3], candidate bits and
-// deferred tiles of parity k & 1.
+// deferred tiles of slot k % kDepth.
 static void select_ctr(ckpt_ctx* h, uint32_t k) {
-  h->cand = h->cand2[k & 1];
-  h->defer = h->defer2[k & 1];
-  uint8_t* c = h->ctr3[k % 3];
+  h->cand = h->cand2[k % kDepth];
+  h->defer = h->defer2[k % kDepth];
+  uint8_t* c = h->ctr3[k % (kDepth + 1)];
   h->tot = reinterpret_cast<Totals*>(c);
   h->dbits = reinterpret_cast<uint32_t*>(c + h->ctr_dbits_off);
   h->tcc = reinterpret_cast<uint32_t*>(c + h->ctr_tcc_off);
@@ -846,17 +854,23 @@ static int ensure_pipe_state(ckpt_ctx* h) {
   for (const char* v : {"CUDA_INJECTION64_PATH", "NV_COMPUTE_PROFILER_PERFWORKS_DIR", "NVIDIA-PROCESS-TRACKING-CONFIGURATION"})
     if (const char* e = getenv(v)) tool = tool || *e;
   if (!(gm && atoi(gm) == 0) && !tool && h->num_sms >= 96) {
+    const int forced = gm ? atoi(gm) : 0;
     for (int m : {16, 24, 32, 40}) {
+      if (forced >= 8) m = forced;
       if (make_green(h, h->parts[h->nparts], m, hi) != CKPT_OK) {   // no partitions: the shared form
         cudaGetLastError();
         break;
       }
       ++h->nparts;
+      if (forced >= 8) {
+        h->part_forced = true;
+        break;
+      }
     }
-    for (int i = 0; i < 2 && h->nparts; ++i)
+    for (int i = 0; i < kDepth && h->nparts; ++i)
       if (cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming) != cudaSuccess) return CKPT_ECUDA;
   }
-  for (int i = 0; i < 2; ++i)
+  for (int i = 0; i < kDepth; ++i)
     if (cudaEventCreateWithFlags(&h->ev_k1[i], cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&h->ev_chain[i], cudaEventDisableTiming) != cudaSuccess) {
       cudaGetLastError();
@@ -887,7 +901,8 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   const int sms_k1 = green ? part->sm_k1 : h->num_sms, sms_chain = green ? part->sm_chain : h->num_sms;
   if (pipe) {
     if (!h->cdig2[0]) {
-      if (dalloc(h, &h->cdig2[0], h->n) != cudaSuccess || dalloc(h, &h->cdig2[1], h->n) != cudaSuccess) return CKPT_ENOMEM;
+      for (int i = 0; i < kDepth; ++i)
+        if (dalloc(h, &h->cdig2[i], h->n) != cudaSuccess) return CKPT_ENOMEM;
     }
     const bool prev_pipe = k > 0 && h->call_pipe[(k - 1) & 3];
     if (!prev_pipe) {
@@ -903,14 +918,16 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
     } else {
       // K1(k) after K1(k - 1) (prev digests, possibly another stream) and after the chain of
       // call k - 2 (this parity's buffers); the chain follows call k - 1's on h->cs
-      CK(cudaStreamWaitEvent(kst, h->ev_k1[(k - 1) & 1], 0));
-      if (k >= 2 && h->call_pipe[(k - 2) & 3]) CK(cudaStreamWaitEvent(kst, h->ev_chain[k & 1], 0));
+      CK(cudaStreamWaitEvent(kst, h->ev_k1[(k - 1) % kDepth], 0));
+      // K1(k) reuses the buffers of call k - kDepth (slot k % kDepth): after that call's chain
+      if (k >= (uint32_t)kDepth && h->call_pipe[(k - kDepth) & 3])
+        CK(cudaStreamWaitEvent(kst, h->ev_chain[k % kDepth], 0));
       // a chain on another stream than the previous call's follows that call's chain
-      if (cst != h->prev_cs) CK(cudaStreamWaitEvent(cst, h->ev_chain[(k - 1) & 1], 0));
+      if (cst != h->prev_cs) CK(cudaStreamWaitEvent(cst, h->ev_chain[(k - 1) % kDepth], 0));
     }
     if (green) {   // K1 after the caller's work on `st` (the input buffer)
-      CK(cudaEventRecord(h->ev_in[k & 1], st));
-      CK(cudaStreamWaitEvent(kst, h->ev_in[k & 1], 0));
+      CK(cudaEventRecord(h->ev_in[k % kDepth], st));
+      CK(cudaStreamWaitEvent(kst, h->ev_in[k % kDepth], 0));
     }
   }
   const auto t_tab = clk::now();
@@ -919,16 +936,17 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   if (r != CKPT_OK) return r;
   const auto t_arena = clk::now();
   const uint64_t worst = 64 + 12 * h->n + 16 + h->B;
-  // pipelined calls alternate between two arenas, so a call's place is known while the
-  // previous call's diff size is not yet; the other arena's last diff (call k - 2) is final
-  const int ai = pipe ? (int)(k & 1) : 0;
-  if (ai == 1 && !h->arena1_ready) {
-    if (!h->arena[1].init(h->device)) return CKPT_ECUDA;
+  // pipelined calls rotate over kDepth arenas, so a call's place is known while the sizes of
+  // the calls still in flight are not; that arena's last diff (call k - kDepth) is final
+  const int ai = pipe ? (int)(k % kDepth) : 0;
+  while (ai >= h->arenas_ready) {
+    DiffArena& A = h->arena[h->arenas_ready];
+    if (!A.init(h->device)) return CKPT_ECUDA;
     bool reserved = false;
     for (uint64_t va : kArenaVA)
-      if (va >= 4 * (h->B + 12 * h->n + 1024) && h->arena[1].reserve(va)) { reserved = true; break; }
+      if (va >= 4 * (h->B + 12 * h->n + 1024) && A.reserve(va)) { reserved = true; break; }
     if (!reserved) return CKPT_ENOMEM;
-    h->arena1_ready = true;
+    ++h->arenas_ready;
   }
   // pipelined: an arena's first mapping covers two diffs' worst case, so that its next
   // physical growth (a host cost of 0.5-2 ms, during which a pipelined lineage starves) comes
@@ -944,7 +962,7 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   select_ctr(h, k);
   // the leaf digests the chain reads: prev itself, or (pipelined) this call's copy of its
   // candidates' digests, since the next call's K1 rewrites prev meanwhile
-  Digest* const ldig = pipe ? h->cdig2[k & 1] : h->prev;
+  Digest* const ldig = pipe ? h->cdig2[k % kDepth] : h->prev;
 
   // ---- record-insert state (K1's insert warp and K1b)
   InsertParams ip;
@@ -1028,8 +1046,8 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   CK(launch_leaf(&tmap, lp, sms_k1, kst));
   if (h->prof) CK(cudaEventRecord(h->ev[1], kst));
   if (pipe) {
-    CK(cudaEventRecord(h->ev_k1[k & 1], kst));
-    CK(cudaStreamWaitEvent(cst, h->ev_k1[k & 1], 0));
+    CK(cudaEventRecord(h->ev_k1[k % kDepth], kst));
+    CK(cudaStreamWaitEvent(cst, h->ev_k1[k % kDepth], 0));
   }
   // K1b: record insert + tie-break (l.6-19), dirty tiles
   // pipelined: a plain launch (the chain stream's previous kernel is the last call's gather,
@@ -1092,9 +1110,9 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   cp.lmask = h->lmask;
   cp.out = out; cp.buf = buf;
   cp.trace = h->trace; cp.trace_n = h->trace_n;
-  cp.tot_host = h->tot_host2[k & 1];
+  cp.tot_host = h->tot_host2[k % kDepth];
   cp.dbg = h->dbg;
-  cp.ctr_next = reinterpret_cast<uint4*>(h->ctr3[(k + 2) % 3]);   // call k - 1's: complete
+  cp.ctr_next = reinterpret_cast<uint4*>(h->ctr3[(k + kDepth) % (kDepth + 1)]);   // call k - 1's: complete
   cp.ctr_next_words = h->ctr_bytes / 16;
   cp.mode = h->mode;
   cp.flags = tp.shift_insert ? CKPT_FLAGS_SHIFT_INSERT : h->mode;
@@ -1107,7 +1125,7 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
   CK(launch_compact(cp, sms_chain, cst));
   if (h->prof) CK(cudaEventRecord(h->ev[5], cst));
   if (pipe) {
-    CK(cudaEventRecord(h->ev_chain[k & 1], cst));
+    CK(cudaEventRecord(h->ev_chain[k % kDepth], cst));
     h->prev_cs = cst;
   }
   h->last_stream = cst;
@@ -1130,7 +1148,7 @@ static int launch_call(ckpt_ctx* h, const void* dev_ptr, uint64_t bytes, cudaStr
 static int finish_call(ckpt_ctx* h, const Inflight& f, ckpt_diff* diff) {
   const uint32_t k = f.k;
   const uint32_t epoch = k + 1;
-  Totals* const th = h->tot_host2[k & 1];
+  Totals* const th = h->tot_host2[k % kDepth];
   {
     ++h->host_syncs;
     volatile uint32_t* done = &th->done;
@@ -1228,8 +1246,8 @@ int ckpt_checkpoint_submit(ckpt_handle h, const void* dev_ptr, uint64_t bytes, v
   LaunchCount lc(h);
   int r = check_buffer(h, dev_ptr, bytes);
   if (r != CKPT_OK) return r;
-  // at most two calls in flight: collect the oldest first
-  while (h->inflight.size() >= 2) {
+  // at most kDepth calls in flight: collect the oldest first
+  while (h->inflight.size() >= (size_t)kDepth) {
     const Inflight f = h->inflight.front();
     h->inflight.pop_front();
     r = finish_call(h, f, nullptr);
@@ -1257,7 +1275,7 @@ int ckpt_checkpoint_wait(ckpt_handle h, uint32_t id, void* stream, ckpt_diff* di
   // the rest of call id (its gather) before the caller's later work on `stream`: the event
   // of this parity follows call id's gather (or a later call's, at worst late)
   const cudaStream_t ws = static_cast<cudaStream_t>(stream);
-  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ws, h->ev_chain[id & 1], 0));
+  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ws, h->ev_chain[id % kDepth], 0));
   *diff = h->diffs[id].info;
   return h->diffs[id].collided ? CKPT_ECOLLIDE : CKPT_OK;
 }
@@ -1301,7 +1319,7 @@ int ckpt_diff_to_host_async(ckpt_handle h, uint32_t id, void* host_ptr, uint64_t
   const cudaStream_t ds = static_cast<cudaStream_t>(stream);
   // after the gather of call id: the event of its parity (re-recorded by a later call of the
   // same parity at most, which is later still), or the latest call for a synchronous one
-  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ds, h->ev_chain[id & 1], 0));
+  if (h->call_pipe[id & 3]) CK(cudaStreamWaitEvent(ds, h->ev_chain[id % kDepth], 0));
   else CK(after_last_checkpoint(h, ds));
   CK(cudaMemcpyAsync(host_ptr, d.ptr, d.info.bytes, cudaMemcpyDeviceToHost, ds));
   return CKPT_OK;

@@ -333,3 +333,16 @@ def test_partition_switching_pipelined(oracle_mod, monkeypatch, green):
     else:
         monkeypatch.delenv("CKPT_GREEN", raising=False)
     run_pipe_parity(oracle_mod, _alternating_lineage((16 << 20) + 48, 128, 8), 128)
+
+
+@pytest.mark.parametrize("seed", [3, 11])
+def test_full_depth_in_flight(oracle_mod, seed):
+    # CKPT_PIPELINE_DEPTH calls in flight, submitted through the generic depth loop of bench.py
+    # (K1(k) reuses the buffers of call k - depth while the calls between are in their tree
+    # phases; a depth-3 build, CKPT_PIPE_DEPTH=3, passed the same tests)
+    from paper_conf_icpp_tanlmtmbctn23_b200 import workloads as W
+    from paper_conf_icpp_tanlmtmbctn23_b200.ckpt import PIPELINE_DEPTH
+    rng = np.random.default_rng(seed)
+    bufs = dup_lineage(seed, int(rng.integers(40_000, 400_000)), 128, K=9, alphabet=4, p_change=0.5)
+    run_pipe_parity(oracle_mod, bufs, 128, depth=PIPELINE_DEPTH)
+    run_pipe_parity(oracle_mod, list(W.lineage(2, (1 << 22) + 100, 128, 8, p=0.05)), 128, depth=PIPELINE_DEPTH)

@@ -37,22 +37,22 @@ def sync_run():
     return e0.elapsed_time(e1) / K
 
 
+DEPTH = int(os.environ.get("DEPTH", 2))   # calls in flight (the library's CKPT_PIPELINE_DEPTH or less)
+
+
 def pipe_run():
     ck = Checkpointer(C)
-    pend = None
+    pend = []
     for k in range(Wm):
-        cid = ck.submit(bufs[k], stream=st)
-        if pend is not None: ck.wait(pend, stream=st)
-        pend = cid
-    ck.wait(pend, stream=st)
-    pend = None
+        pend.append(ck.submit(bufs[k], stream=st))
+        if len(pend) >= DEPTH: ck.wait(pend.pop(0), stream=st)
+    while pend: ck.wait(pend.pop(0), stream=st)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(st)
     for k in range(Wm, Wm + K):
-        cid = ck.submit(bufs[k], stream=st)
-        if pend is not None: ck.wait(pend, stream=st, raw=True)
-        pend = cid
-    ck.wait(pend, stream=st, raw=True)
+        pend.append(ck.submit(bufs[k], stream=st))
+        if len(pend) >= DEPTH: ck.wait(pend.pop(0), stream=st, raw=True)
+    while pend: ck.wait(pend.pop(0), stream=st, raw=True)
     e1.record(st); st.synchronize()
     ck.close()
     return e0.elapsed_time(e1) / K
