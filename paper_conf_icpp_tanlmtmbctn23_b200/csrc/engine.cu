@@ -158,9 +158,11 @@ struct ckpt_ctx {
     int sm_k1 = 0, sm_chain = 0;
   };
   static constexpr int kMaxParts = 4;
-  Part parts[kMaxParts];
-  int nparts = 0;
-  bool part_forced = false;         // CKPT_GREEN=m (m >= 8): every pipelined call on one m-SM partition (tuning)
+  static constexpr int kPartSMs[kMaxParts] = {16, 24, 32, 40};   // chain SMs of each partition
+  Part parts[kMaxParts];            // created at first use (make_green: ~0.1-1 s of host time each)
+  bool green_ok = false;            // partitions allowed (no CKPT_GREEN=0, no profiling tool, a full GPU)
+  int forced_m = 0;                 // CKPT_GREEN=m (m >= 8): every pipelined call on one m-SM partition (tuning)
+  int prio_hi = 0;                  // the chain streams' priority
   cudaEvent_t ev_in[kDepth] = {};
   cudaStream_t prev_cs = nullptr;   // chain stream of the previous pipelined call
   uint64_t last_cand = ~0ull;       // non-FIXED leaves of the last collected call (~0: none yet)
@@ -610,11 +612,16 @@ static int make_green(ckpt_ctx* h, ckpt_ctx::Part& P, int m, int prio_hi) {
 // which outweighs the hidden chain on long K1 passes (config 3, 4 GiB at C = 4096: 0.715 ->
 // 0.733 ms per step), so buffers above 2 GiB are not partitioned.
 static const ckpt_ctx::Part* pick_part(const ckpt_ctx* h) {
-  if (h->part_forced) return &h->parts[0];
-  if (!h->nparts || h->last_cand == ~0ull || h->B > (2ull << 30)) return nullptr;
-  for (int i = 0; i < h->nparts; ++i)
-    if (h->last_cand <= (uint64_t)CKPT_GREEN_CAND_PER_SM * (uint64_t)h->parts[i].sm_chain) return &h->parts[i];
-  return nullptr;
+  if (!h->green_ok) return nullptr;
+  int i = -1;
+  if (h->forced_m) {
+    i = 0;
+  } else if (h->last_cand != ~0ull && h->B <= (2ull << 30)) {
+    for (int j = 0; j < ckpt_ctx::kMaxParts && i < 0; ++j)
+      if (h->last_cand <= (uint64_t)CKPT_GREEN_CAND_PER_SM * (uint64_t)ckpt_ctx::kPartSMs[j]) i = j;
+  }
+  if (i < 0) return nullptr;
+  return &h->parts[i];
 }
 
 extern "C" {
@@ -834,7 +841,7 @@ using clk = std::chrono::steady_clock;
 static float ms_since(clk::time_point a, clk::time_point b) { return std::chrono::duration<float, std::milli>(b - a).count(); }
 
 // Pipelined calls only: the chain stream, the events and the second arena (created once).
-static int ensure_pipe_state(ckpt_ctx* h) {
+static int ensure_pipe_state(ckpt_ctx* h, uint64_t bytes) {
   if (h->cs) return CKPT_OK;
   // non-blocking: work on the legacy default stream must not serialise against the chain.
   // Highest priority: when K1 of the next call and this chain's kernels both wait for SM
@@ -853,21 +860,19 @@ static int ensure_pipe_state(ckpt_ctx* h) {
   bool tool = false;
   for (const char* v : {"CUDA_INJECTION64_PATH", "NV_COMPUTE_PROFILER_PERFWORKS_DIR", "NVIDIA-PROCESS-TRACKING-CONFIGURATION"})
     if (const char* e = getenv(v)) tool = tool || *e;
-  if (!(gm && atoi(gm) == 0) && !tool && h->num_sms >= 96) {
-    const int forced = gm ? atoi(gm) : 0;
-    for (int m : {16, 24, 32, 40}) {
-      if (forced >= 8) m = forced;
-      if (make_green(h, h->parts[h->nparts], m, hi) != CKPT_OK) {   // no partitions: the shared form
-        cudaGetLastError();
-        break;
-      }
-      ++h->nparts;
-      if (forced >= 8) {
-        h->part_forced = true;
-        break;
-      }
-    }
-    for (int i = 0; i < kDepth && h->nparts; ++i)
+  // Created here, at the first pipelined call (host time once: a partition created when the
+  // candidate count first calls for it stalled that call by 10-25 ms, inside a timed lineage),
+  // and only for buffers that can use them (pick_part: <= 2 GiB)
+  const int forced = gm ? atoi(gm) : 0;
+  if (!(gm && forced == 0) && !tool && h->num_sms >= 96 && (bytes <= (2ull << 30) || forced >= 8)) {
+    h->prio_hi = hi;
+    if (forced >= 8 && forced <= h->num_sms - 64) h->forced_m = forced;
+    bool ok = true;
+    for (int j = 0; j < (h->forced_m ? 1 : ckpt_ctx::kMaxParts) && ok; ++j)
+      ok = make_green(h, h->parts[j], h->forced_m ? h->forced_m : ckpt_ctx::kPartSMs[j], hi) == CKPT_OK;
+    if (!ok) cudaGetLastError();   // no partitions on this device: the shared form
+    h->green_ok = ok;
+    for (int i = 0; i < kDepth; ++i)
       if (cudaEventCreateWithFlags(&h->ev_in[i], cudaEventDisableTiming) != cudaSuccess) return CKPT_ECUDA;
   }
   for (int i = 0; i < kDepth; ++i)
@@ -1253,7 +1258,7 @@ int ckpt_checkpoint_submit(ckpt_handle h, const void* dev_ptr, uint64_t bytes, v
     r = finish_call(h, f, nullptr);
     if (r != CKPT_OK && r != CKPT_ECOLLIDE) return r;
   }
-  if ((r = ensure_pipe_state(h)) != CKPT_OK) return r;
+  if ((r = ensure_pipe_state(h, bytes)) != CKPT_OK) return r;
   Inflight f;
   if ((r = launch_call(h, dev_ptr, bytes, static_cast<cudaStream_t>(stream), true, &f)) != CKPT_OK) return r;
   h->inflight.push_back(f);
