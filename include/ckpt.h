@@ -183,6 +183,10 @@ CKPT_API int ckpt_checkpoint(ckpt_handle h, const void* dev_ptr, uint64_t bytes,
  *                   on it, or (SM partitions) on an internal stream of a green
  *                   context ordered after it by an event; the record and tree phases and the
  *                   gather run on an internal non-blocking stream, ordered after the leaf pass.
+ *                   SM partitions: created at the handle's first submit when the buffer is at
+ *                   most 2 GiB (host time once); each call picks one from the candidate count of
+ *                   the last collected call, or none. Environment CKPT_GREEN=0 disables them;
+ *                   they are also off under a profiling tool (CUDA_INJECTION64_PATH set).
  *   id              receives the checkpoint id (= the number of checkpoints before it).
  * At most CKPT_PIPELINE_DEPTH (2) calls are in flight: a submit with that many outstanding
  * first collects the oldest (a host wait). Every other call of this library (ckpt_checkpoint, diff access, restore,
