@@ -102,7 +102,7 @@ struct ckpt_ctx {
   // device state
   Digest* prev = nullptr;
   uint32_t* cand = nullptr;       // = cand2[k % kDepth] of the current call
-  uint32_t* cand2[kDepth] = {};        // candidate bits per call parity: a pipelined call's K1 writes its own
+  uint32_t* cand2[kDepth] = {};   // candidate bits per call slot (k % kDepth): a pipelined call's K1 writes its own
                                   // while the previous call's tree phases read theirs
   Digest* cdig2[kDepth] = {};          // pipelined calls: the candidates' digests of call k (slot k % kDepth), read
                                   // by its K1b / tree kernels while the next call's K1 updates prev in place
@@ -135,7 +135,7 @@ struct ckpt_ctx {
   unsigned long long* blocksum = nullptr;
   unsigned long long* gsum = nullptr;
   Totals* tot = nullptr;         // = (Totals*)ctr
-  Totals* tot_host2[kDepth] = {};    // pinned + mapped, per call parity: written by the gather kernel
+  Totals* tot_host2[kDepth] = {};    // pinned + mapped, per call slot: written by the gather kernel
   Slot* tab = nullptr;
   uint64_t cap = 0, live = 0;
   std::vector<void*> retired;    // record tables replaced by a growth (freed by ckpt_destroy)
@@ -159,7 +159,7 @@ struct ckpt_ctx {
   };
   static constexpr int kMaxParts = 4;
   static constexpr int kPartSMs[kMaxParts] = {16, 24, 32, 40};   // chain SMs of each partition
-  Part parts[kMaxParts];            // created at first use (make_green: ~0.1-1 s of host time each)
+  Part parts[kMaxParts];            // created at the first pipelined call of a buffer <= 2 GiB (ensure_pipe_state)
   bool green_ok = false;            // partitions allowed (no CKPT_GREEN=0, no profiling tool, a full GPU)
   int forced_m = 0;                 // CKPT_GREEN=m (m >= 8): every pipelined call on one m-SM partition (tuning)
   int prio_hi = 0;                  // the chain streams' priority
